@@ -1,0 +1,375 @@
+#!/usr/bin/env python3
+"""bench.py -- bitBSR SpMV throughput on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload fem1p5m]
+                    [--dtype fp32|fp16] [--impl spaden|reference]
+
+A step is one iterated SpMV over the whole matrix: x_{k+1} = alpha * A x_k with
+alpha = 1/||A||_inf (bounded iterates).  With N > 1 (torchrun, NCCL) A is
+row-partitioned in 8-row-aligned slices, each rank computes its slice of
+x_{k+1} and an NCCL all-gather rebuilds the replicated x;
+total work is fixed ("strong" scaling).  The timed region is K steps between
+barrier + synchronize; the time is the max over ranks of CUDA-event time.
+
+Inputs are synthetic (workloads/, seeded) and resident in HBM; the matrix
+(480 MB for fem1p5m fp32) is larger than the 126 MB L2, so no L2 flush is
+needed between steps (x, 6 MB, is L2-resident as in any iterative solver).
+
+--impl reference times the CPU oracle (oracle/, fp64 CSR SpMV, single thread)
+on a bounded row sample per step -- this tier's reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+METRIC = "SpMV GFLOP/s (2*nnz/t) on bitBSR; achieved HBM GB/s and bytes/nnz alongside"
+UNIT = "GFLOP/s"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=2000)
+    p.add_argument("--warmup", type=int, default=20)
+    p.add_argument("--workload", default="fem1p5m", choices=sorted(W.CONFIGS))
+    p.add_argument("--dtype", default="fp32", choices=["fp32", "fp16"])
+    p.add_argument("--impl", default="spaden", choices=["spaden", "reference"])
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-cusparse", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=12.0)
+    return p.parse_args()
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def alg_bytes(m, n, nnz, Bnrow, Bnnz, sv, beta_nonzero=False):
+    """Algorithmic bytes of one SpMV: the bitBSR arrays once
+    (blk_rowptr, blk_col, bitmap, blk_offset, values), x once, y written once."""
+    return 4 * (Bnrow + 1) + (4 + 8 + 4) * Bnnz + sv * nnz + 4 * n + 4 * m + (4 * m if beta_nonzero else 0)
+
+
+class Clocks:
+    """NVML sampler of SM clock and throttle reasons during the timed region."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, index, period=0.02):
+        self.index, self.period = index, period
+        self.samples, self.reasons = [], set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._t = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.nv:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons - {"gpu_idle"}), "samples": len(self.samples)}
+
+
+def cpu_oracle_gflops(A, x, seconds):
+    """The oracle (fp64 CSR SpMV, single thread) on whole-matrix passes, bounded in time."""
+    import oracle
+    oracle.lib()
+    rp = np.ascontiguousarray(A.rowptr, np.int64)
+    v = np.ascontiguousarray(A.values.astype(np.float64))
+    xx = np.ascontiguousarray(x.astype(np.float64))
+    t0 = time.perf_counter()
+    passes = 0
+    while True:
+        oracle.spmv(rp, A.colidx, v, xx)
+        passes += 1
+        if time.perf_counter() - t0 >= seconds:
+            break
+    dt = time.perf_counter() - t0
+    return {"value": 2.0 * A.nnz * passes / dt / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{passes} full passes over the {A.m}x{A.n} matrix ({A.nnz} nnz), fp64, "
+                      f"{dt:.1f} s wall"}
+
+
+def reference_arm(args):
+    """--impl reference: the CPU oracle as this tier's reference arm."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    A = W.make(args.workload)
+    vals = A.values if args.dtype == "fp32" else oracle.f32_to_f16(A.values)
+    x = W.vector(A.n, 2)
+    oracle.lib()
+    # per-step budget so that K+W steps take ~90 s of CPU time in total
+    t0 = time.perf_counter()
+    oracle.spmv(A.rowptr, A.colidx, vals, x)
+    full = time.perf_counter() - t0
+    frac = min(1.0, 90.0 / max(1, args.steps + args.warmup) / max(full, 1e-6))
+    r1 = max(8, int(A.m * frac) // 8 * 8)
+    S = A.row_slice(0, r1)
+    sv = vals[: S.nnz]
+    rp = np.ascontiguousarray(S.rowptr, np.int64)
+    v = np.ascontiguousarray(sv.astype(np.float64))
+    xx = np.ascontiguousarray(x.astype(np.float64))
+    for _ in range(args.warmup):
+        oracle.spmv(rp, S.colidx, v, xx)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.spmv(rp, S.colidx, v, xx)
+    dt = time.perf_counter() - t0
+    val = 2.0 * S.nnz * args.steps / dt / 1e9
+    line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "impl": "reference",
+            "config": {"workload": args.workload, "m": A.m, "n": A.n, "nnz": A.nnz, "values": args.dtype,
+                       "sample_rows": r1, "sample_nnz": S.nnz},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"rows [0,{r1}) of {args.workload} ({S.nnz} nnz) per step"},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return reference_arm(args)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_cheny24_b200 as sp
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    # ---- workload (identical on every rank), this rank's 8-row-aligned slice
+    A = W.make(args.workload)
+    slice_rows = -(-A.m // (8 * world)) * 8
+    r0, r1 = rank * slice_rows, min(A.m, (rank + 1) * slice_rows)
+    S = A.row_slice(r0, r1)
+    csum = np.concatenate([[0.0], np.cumsum(np.abs(A.values.astype(np.float64)))])
+    a_inf = float((csum[A.rowptr[1:]] - csum[A.rowptr[:-1]]).max()) if A.m else 0.0
+    alpha = 1.0 / a_inf if a_inf > 0 else 1.0
+    sv = 2 if args.dtype == "fp16" else 4
+
+    rp = torch.from_numpy(S.rowptr).to(dev)
+    ci = torch.from_numpy(S.colidx).to(dev)
+    vv = torch.from_numpy(S.values).to(dev)
+    stream = torch.cuda.current_stream(dev)
+    torch.cuda.synchronize(dev)
+    t0 = time.perf_counter()
+    M = sp.convert(rp, ci, vv, A.n, storage=args.dtype)
+    torch.cuda.synchronize(dev)
+    convert_s = time.perf_counter() - t0
+    info = M.info
+    del rp, ci, vv
+
+    nx = slice_rows * world
+    x0 = np.zeros(nx, np.float32)
+    x0[: A.n] = W.vector(A.n, 2)
+    xa = torch.from_numpy(x0).to(dev)
+    xb = torch.zeros(nx, dtype=torch.float32, device=dev)
+    x_a, x_b = xa, xb
+
+    def step(ev_pair=None):
+        nonlocal x_a, x_b
+        ys = x_b[rank * slice_rows: rank * slice_rows + S.m]
+        if ev_pair is not None:
+            ev_pair[0].record(stream)
+        M.spmv(x_a[: A.n], ys, alpha=alpha, beta=0.0, stream=stream)
+        if ev_pair is not None:
+            ev_pair[1].record(stream)
+        if world > 1:
+            dist.all_gather_into_tensor(x_b, x_b[rank * slice_rows:(rank + 1) * slice_rows])
+        x_a, x_b = x_b, x_a
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize(dev)
+
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    start = torch.cuda.Event(enable_timing=True)
+    end = torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    with Clocks(local) as clk:
+        start.record(stream)
+        for i in range(args.steps):
+            step(evs[i])
+        end.record(stream)
+        torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    elapsed_ms = start.elapsed_time(end)
+    kernel_ms = [a.elapsed_time(b) for a, b in evs]
+    t = torch.tensor([elapsed_ms], device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    elapsed_ms = float(t.item())
+    ms_per_step = elapsed_ms / args.steps
+    gflops = 2.0 * A.nnz * args.steps / (elapsed_ms * 1e-3) / 1e9
+
+    # ---- roofline of the dominant kernel (the SpMV) on this rank
+    kavg_ms = float(np.mean(kernel_ms))
+    abytes = alg_bytes(S.m, A.n, S.nnz, info.Bnrow, info.Bnnz, sv)
+    peak, peak_kind = peaks()
+    achieved = abytes / (kavg_ms * 1e-3) / 1e9
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            tr = json.load(f)
+        key = f"{args.workload}/{args.dtype}"
+        if key in tr and world == 1:
+            traffic = tr[key]["dram_bytes_per_launch"]
+    except Exception:
+        pass
+
+    line = None
+    if rank == 0:
+        clocks = clk.summary()
+        # ---- e2e through the C ABI with host buffers (N=1 rank-local; H2D x, D2H y per step)
+        e2e = None
+        if world == 1:
+            xh = torch.from_numpy(x0[: A.n].copy()).pin_memory()
+            yh = torch.empty(S.m, dtype=torch.float32).pin_memory()
+            for _ in range(3):
+                M.spmv_host(xh, yh, alpha=alpha, stream=stream)
+            e2e_steps = max(20, min(args.steps, 200))
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize(dev)
+            e0.record(stream)
+            for _ in range(e2e_steps):
+                M.spmv_host(xh, yh, alpha=alpha, stream=stream)
+            e1.record(stream)
+            torch.cuda.synchronize(dev)
+            e2e_ms = e0.elapsed_time(e1) / e2e_steps
+            e2e = {"value": 2.0 * A.nnz / (e2e_ms * 1e-3) / 1e9, "unit": UNIT,
+                   "h2d_bytes_per_step": 4 * A.n, "d2h_bytes_per_step": 4 * S.m,
+                   "ms_per_step": e2e_ms, "steps": e2e_steps,
+                   "api": "spaden_spmv_host (pinned host x/y, stream-synchronous)"}
+
+        # ---- cuSPARSE CSR SpMV on the same matrix and GPU (north_star comparison)
+        cus = None
+        if not args.no_cusparse and world == 1:
+            try:
+                Ac = torch.sparse_csr_tensor(torch.from_numpy(A.rowptr).to(dev), torch.from_numpy(A.colidx).to(dev),
+                                             torch.from_numpy(A.values).to(dev), size=(A.m, A.n))
+                xv = xa[: A.n].contiguous()
+                for _ in range(5):
+                    yc = torch.mv(Ac, xv)
+                reps = max(20, min(args.steps, 500))
+                c0 = torch.cuda.Event(enable_timing=True)
+                c1 = torch.cuda.Event(enable_timing=True)
+                torch.cuda.synchronize(dev)
+                c0.record(stream)
+                for _ in range(reps):
+                    yc = torch.mv(Ac, xv)
+                c1.record(stream)
+                torch.cuda.synchronize(dev)
+                cms = c0.elapsed_time(c1) / reps
+                csr_bytes = 4 * (A.m + 1) + 8 * A.nnz
+                cus = {"impl": "torch.mv(sparse_csr fp32) -> cuSPARSE SpMV", "ms": cms,
+                       "gflops": 2.0 * A.nnz / (cms * 1e-3) / 1e9,
+                       "footprint_bytes": csr_bytes, "bytes_per_nnz": csr_bytes / A.nnz,
+                       "speedup_spaden_vs_cusparse": cms / kavg_ms,
+                       "footprint_saving": csr_bytes / info.format_bytes}
+                del Ac, yc
+            except Exception as e:  # pragma: no cover
+                cus = {"error": repr(e)[:200]}
+
+        cpu = None
+        if not args.no_cpu_baseline and world == 1:
+            cpu = cpu_oracle_gflops(A, x0[: A.n], args.cpu_seconds)
+
+        line = {
+            "metric": METRIC, "value": gflops, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": max(3, args.warmup), "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32" if args.dtype == "fp32" else "f16xf32->f32",
+            "data": "synthetic",
+            "config": {"workload": args.workload, "m": A.m, "n": A.n, "nnz": A.nnz, "Bnrow": int((A.m + 7) // 8),
+                       "Bnnz_rank0": int(info.Bnnz), "fill": A.nnz / max(1, info.Bnnz) if world == 1 else None,
+                       "values": args.dtype, "parallelism": f"row-partition x{world}" + (" + NCCL all-gather" if world > 1 else ""),
+                       "l2": "inputs larger than L2 (A > 126 MB), no flush", "step": "x <- A x / ||A||_inf"},
+            "hbm_gbs": achieved,
+            "bytes_per_nnz": {"stored": info.format_bytes / max(1, info.nnz),
+                              "moved": abytes / max(1, S.nnz)},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "peak_kind": f"{peak_kind} copy bandwidth (MEASURED_PEAKS.json hbm_gbs)",
+                         "kernel": "k_spmv (one launch per step)", "kernel_ms": kavg_ms,
+                         "alg_bytes_per_launch": abytes},
+            "convert": {"seconds": convert_s, "ns_per_nnz": convert_s * 1e9 / max(1, S.nnz)},
+            "cusparse_csr": cus,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": args.steps,
+            "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    M.free()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,160 @@
+/*
+ * spaden.h -- C ABI of the B200-native bitBSR SpMV library (libspaden.so).
+ *
+ * Method: Y. Chen, J. X. Yu, "Bitmap-Based Sparse Matrix-Vector Multiplication
+ * with Tensor Cores" (Spaden), ICPP '24.  Passages are cited as P:L<n> =
+ * line n of PAPER.md, with the section / algorithm they fall in.
+ *
+ * The library computes y = alpha * A x + beta * y for a sparse A that it first
+ * converts from CSR (§2.1) into bitBSR (§4.2, Fig. 4):
+ *   - A is cut into 8x8 blocks; Bnrow = ceil(m/8) block-rows.
+ *   - The non-empty blocks of a block-row are listed CSR-style
+ *     in ascending block column:            blk_rowptr int32[Bnrow+1],
+ *                                           blk_col    int32[Bnnz].
+ *   - Each block is one 64-bit occupancy bitmap, bit 8*(r%8)+(c%8),
+ *     LSB = top-left, MSB = bottom-right, row 0 in the low byte:
+ *                                           bitmap     uint64[Bnnz].
+ *   - Per-block nonzero counts, exclusive-scanned:
+ *                                           blk_offset int32[Bnnz+1] (last = nnz).
+ *   - The nonzeros, "stored consecutively" block after block and in
+ *     ascending bit order inside a block:   values     fp32|fp16[nnz].
+ *   The value of set bit `bit` of block b is values[blk_offset[b] +
+ *   popcount(bitmap[b] & ((1<<bit)-1))] (reading R1 of Alg. 2).
+ *
+ * Conventions for every entry point:
+ *   - Pointers named d_* are DEVICE pointers on the device that is current
+ *     when the call is made; h_* are HOST pointers (pinned recommended).
+ *     Inputs are borrowed: the caller keeps them alive until the stream work
+ *     that uses them has completed.  No entry point takes ownership of caller
+ *     memory.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *     All device work is stream-ordered on it.
+ *   - Every call returns a spaden_status_t; nothing aborts or throws across the
+ *     ABI.  On failure a thread-local message is available from
+ *     spaden_last_error_message() and output handles are set to NULL.
+ *   - Indices are int32 (nnz < 2^31, m, n < 2^31).
+ */
+#ifndef SPADEN_H_
+#define SPADEN_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define SPADEN_API __attribute__((visibility("default")))
+#else
+#define SPADEN_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    SPADEN_OK = 0,
+    SPADEN_ERR_INVALID_ARGUMENT = 1,     /* bad sizes, NULL pointers, host pointer where device expected,
+                                            rowptr[0] != 0, rowptr[m] != nnz, non-monotone rowptr */
+    SPADEN_ERR_INDEX_OUT_OF_RANGE = 2,   /* some colidx outside [0, n)                          */
+    SPADEN_ERR_UNSORTED_OR_DUPLICATE = 3,/* colidx not strictly ascending within a row           */
+    SPADEN_ERR_UNSUPPORTED = 4,          /* dtype combination / size limit not supported         */
+    SPADEN_ERR_OUT_OF_MEMORY = 5,        /* device allocation failed                             */
+    SPADEN_ERR_CUDA = 6                  /* any other CUDA runtime error                         */
+} spaden_status_t;
+
+typedef enum {
+    SPADEN_R_32F = 0,   /* IEEE binary32 */
+    SPADEN_R_16F = 1    /* IEEE binary16 */
+} spaden_dtype_t;
+
+/* Opaque handle: owns the device bitBSR arrays of one matrix on one device. */
+typedef struct spaden_matrix_s *spaden_matrix_t;
+
+typedef struct {
+    int64_t m, n, nnz;          /* matrix shape and stored entries                        */
+    int64_t Bnrow, Bnnz;        /* block-rows ceil(m/8), non-empty 8x8 blocks              */
+    int32_t storage_dtype;      /* spaden_dtype_t of values[]                              */
+    int32_t device;             /* CUDA device ordinal the arrays live on                 */
+    int64_t format_bytes;       /* 4(Bnrow+1) + 4Bnnz + 8Bnnz + 4(Bnnz+1) + s_v*nnz: the
+                                   bitBSR footprint (2.85 B/nnz with fp16 values) */
+    int64_t aux_bytes;          /* extra device bytes (SpMV work schedule, padding)       */
+    int64_t n_tiles;            /* SpMV work tiles in the schedule                         */
+} spaden_info_t;
+
+typedef struct {                /* borrowed device views; valid until spaden_free         */
+    const int32_t  *blk_rowptr; /* [Bnrow+1] */
+    const int32_t  *blk_col;    /* [Bnnz]    */
+    const uint64_t *bitmap;     /* [Bnnz]    */
+    const int32_t  *blk_offset; /* [Bnnz+1]  */
+    const void     *values;     /* [nnz] of storage_dtype */
+} spaden_arrays_t;
+
+/*
+ * spaden_convert_csr_to_bitmap -- CSR -> bitBSR on the GPU (§4.2).
+ *
+ *   m, n            matrix shape, 0 <= m, n < 2^31.
+ *   nnz             number of stored entries, 0 <= nnz < 2^31.
+ *   d_rowptr        int32[m+1], rowptr[0] == 0, non-decreasing, rowptr[m] == nnz.
+ *   d_colidx        int32[nnz], each row's columns strictly ascending, in [0, n).
+ *   d_values        [nnz] of values_dtype.
+ *   values_dtype    dtype of d_values.
+ *   storage_dtype   dtype of the stored bitBSR values: 32F->32F and 16F->16F move
+ *                   raw bits; 32F->16F rounds to nearest even; 16F->32F is exact.
+ *   stream          cudaStream_t (void*).
+ *   out             receives the new handle (NULL on error).
+ *
+ * Stream-ordered; performs exactly one host synchronisation of `stream` (to
+ * learn Bnnz and the validation result before allocating).  A stored 0.0 keeps
+ * its bit (the round trip bitBSR -> CSR is the identity).  Invalid CSR is
+ * reported as INVALID_ARGUMENT / INDEX_OUT_OF_RANGE / UNSORTED_OR_DUPLICATE;
+ * nothing is leaked on error.  m == 0, n == 0 or nnz == 0 give a valid handle.
+ */
+SPADEN_API spaden_status_t spaden_convert_csr_to_bitmap(int64_t m, int64_t n, int64_t nnz,
+                                             const int32_t *d_rowptr, const int32_t *d_colidx,
+                                             const void *d_values, spaden_dtype_t values_dtype,
+                                             spaden_dtype_t storage_dtype, void *stream,
+                                             spaden_matrix_t *out);
+
+/*
+ * spaden_spmv -- y = alpha * A x + beta * y on the GPU (§4.3: "takes bitBSR
+ * and a dense vector x as input and produces a dense vector y").
+ *
+ *   A         handle from spaden_convert_csr_to_bitmap (immutable; may be used by
+ *             several streams concurrently).
+ *   d_x       float32[n] (read-only; only entries referenced by a set bit are read,
+ *             structural zeros are never multiplied).
+ *   d_y       float32[m]; with beta == 0 it is write-only (its old contents, even
+ *             NaN, are ignored).  d_x and d_y must not overlap.
+ *   stream    cudaStream_t (void*).
+ *
+ * Accumulation is fp32 in a fixed order that depends only on each block-row's own
+ * blocks (deterministic; identical for any row partition aligned to 8 rows).
+ * Never allocates and never synchronises: CUDA-graph capturable.
+ */
+SPADEN_API spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const float *d_x, float beta,
+                            float *d_y, void *stream);
+
+/*
+ * spaden_spmv_host -- the same operation with HOST vectors: copies h_x (and h_y if
+ * beta != 0) to device staging buffers owned by the handle, runs spaden_spmv,
+ * copies y back to h_y and synchronises `stream`.  Not thread-safe per handle.
+ */
+SPADEN_API spaden_status_t spaden_spmv_host(spaden_matrix_t A, float alpha, const float *h_x, float beta,
+                                 float *h_y, void *stream);
+
+/* spaden_free -- synchronises the handle's device, then releases all device
+ * arrays owned by A.  spaden_free(NULL) returns SPADEN_OK. */
+SPADEN_API spaden_status_t spaden_free(spaden_matrix_t A);
+
+/* Introspection (tests, bench, the bytes-per-nnz metric). */
+SPADEN_API spaden_status_t spaden_get_info(spaden_matrix_t A, spaden_info_t *info);
+SPADEN_API spaden_status_t spaden_get_arrays(spaden_matrix_t A, spaden_arrays_t *arrays);
+
+/* Static strings; never NULL. */
+SPADEN_API const char *spaden_status_string(spaden_status_t s);
+SPADEN_API const char *spaden_last_error_message(void);
+SPADEN_API const char *spaden_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPADEN_H_ */

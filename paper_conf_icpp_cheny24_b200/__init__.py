@@ -1,0 +1,227 @@
+"""Thin Python binding (ctypes) over libspaden.so -- the C ABI in include/spaden.h.
+
+Argument marshalling only: every step of CSR->bitBSR conversion and SpMV runs
+in the library's CUDA kernels.  PyTorch supplies device memory and streams.
+There is no CPU fallback: importing this package on a machine without the
+built library raises ImportError, and every call on a missing device fails.
+
+Raw entry points keep the C names (spaden_convert_csr_to_bitmap, spaden_spmv,
+spaden_spmv_host, spaden_free, spaden_get_info, spaden_get_arrays,
+spaden_status_string, spaden_last_error_message, spaden_version); `convert`
+and `Matrix` wrap them for torch tensors.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libspaden.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_icpp_cheny24_b200.build` "
+                      "(or __graft_entry__.build()); there is no fallback implementation")
+
+_lib = ctypes.CDLL(LIB_PATH)
+
+SPADEN_OK = 0
+SPADEN_ERR_INVALID_ARGUMENT = 1
+SPADEN_ERR_INDEX_OUT_OF_RANGE = 2
+SPADEN_ERR_UNSORTED_OR_DUPLICATE = 3
+SPADEN_ERR_UNSUPPORTED = 4
+SPADEN_ERR_OUT_OF_MEMORY = 5
+SPADEN_ERR_CUDA = 6
+SPADEN_R_32F = 0
+SPADEN_R_16F = 1
+
+
+class spaden_info_t(ctypes.Structure):
+    _fields_ = [("m", ctypes.c_int64), ("n", ctypes.c_int64), ("nnz", ctypes.c_int64),
+                ("Bnrow", ctypes.c_int64), ("Bnnz", ctypes.c_int64),
+                ("storage_dtype", ctypes.c_int32), ("device", ctypes.c_int32),
+                ("format_bytes", ctypes.c_int64), ("aux_bytes", ctypes.c_int64),
+                ("n_tiles", ctypes.c_int64)]
+
+
+class spaden_arrays_t(ctypes.Structure):
+    _fields_ = [("blk_rowptr", ctypes.c_void_p), ("blk_col", ctypes.c_void_p),
+                ("bitmap", ctypes.c_void_p), ("blk_offset", ctypes.c_void_p),
+                ("values", ctypes.c_void_p)]
+
+
+_P = ctypes.c_void_p
+_I64 = ctypes.c_int64
+_ST = ctypes.c_int
+_F = ctypes.c_float
+
+spaden_convert_csr_to_bitmap = _lib.spaden_convert_csr_to_bitmap
+spaden_convert_csr_to_bitmap.argtypes = [_I64, _I64, _I64, _P, _P, _P, ctypes.c_int, ctypes.c_int, _P,
+                                         ctypes.POINTER(_P)]
+spaden_convert_csr_to_bitmap.restype = _ST
+spaden_spmv = _lib.spaden_spmv
+spaden_spmv.argtypes = [_P, _F, _P, _F, _P, _P]
+spaden_spmv.restype = _ST
+spaden_spmv_host = _lib.spaden_spmv_host
+spaden_spmv_host.argtypes = [_P, _F, _P, _F, _P, _P]
+spaden_spmv_host.restype = _ST
+spaden_free = _lib.spaden_free
+spaden_free.argtypes = [_P]
+spaden_free.restype = _ST
+spaden_get_info = _lib.spaden_get_info
+spaden_get_info.argtypes = [_P, ctypes.POINTER(spaden_info_t)]
+spaden_get_info.restype = _ST
+spaden_get_arrays = _lib.spaden_get_arrays
+spaden_get_arrays.argtypes = [_P, ctypes.POINTER(spaden_arrays_t)]
+spaden_get_arrays.restype = _ST
+spaden_status_string = _lib.spaden_status_string
+spaden_status_string.argtypes = [_ST]
+spaden_status_string.restype = ctypes.c_char_p
+spaden_last_error_message = _lib.spaden_last_error_message
+spaden_last_error_message.argtypes = []
+spaden_last_error_message.restype = ctypes.c_char_p
+spaden_version = _lib.spaden_version
+spaden_version.argtypes = []
+spaden_version.restype = ctypes.c_char_p
+
+EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_spmv", "spaden_spmv_host", "spaden_free",
+            "spaden_get_info", "spaden_get_arrays", "spaden_status_string",
+            "spaden_last_error_message", "spaden_version"]
+
+
+class SpadenError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        msg = spaden_last_error_message().decode(errors="replace")
+        super().__init__(f"{where}: {spaden_status_string(status).decode()} ({msg})")
+
+
+def _check(status: int, where: str):
+    if status != SPADEN_OK:
+        raise SpadenError(status, where)
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _stream_ptr(stream):
+    torch = _torch()
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _dtype_code(dt) -> int:
+    torch = _torch()
+    if dt in (torch.float32, "fp32", "f32", "float32", SPADEN_R_32F):
+        return SPADEN_R_32F
+    if dt in (torch.float16, "fp16", "f16", "float16", SPADEN_R_16F):
+        return SPADEN_R_16F
+    raise ValueError(f"unsupported dtype {dt!r}")
+
+
+class _CudaArray:
+    """__cuda_array_interface__ shim to view a library-owned device array."""
+
+    def __init__(self, ptr: int, shape, typestr: str, owner):
+        self.__cuda_array_interface__ = {"data": (ptr or 0, True), "shape": tuple(shape),
+                                         "typestr": typestr, "version": 3, "strides": None}
+        self._owner = owner
+
+
+class Matrix:
+    """Owning wrapper of a spaden_matrix_t (bitBSR on one device)."""
+
+    def __init__(self, handle: ctypes.c_void_p, device):
+        self._h = handle
+        self.device = device
+        self.info = self.get_info()
+
+    @property
+    def handle(self):
+        return self._h
+
+    def get_info(self) -> spaden_info_t:
+        inf = spaden_info_t()
+        _check(spaden_get_info(self._h, ctypes.byref(inf)), "spaden_get_info")
+        return inf
+
+    @property
+    def m(self):
+        return self.info.m
+
+    @property
+    def n(self):
+        return self.info.n
+
+    @property
+    def nnz(self):
+        return self.info.nnz
+
+    def arrays(self):
+        """Borrowed torch views (on device) of blk_rowptr, blk_col, bitmap, blk_offset, values."""
+        torch = _torch()
+        a = spaden_arrays_t()
+        _check(spaden_get_arrays(self._h, ctypes.byref(a)), "spaden_get_arrays")
+        i = self.info
+        vt = "<f2" if i.storage_dtype == SPADEN_R_16F else "<f4"
+        tdt = {"<i4": torch.int32, "<i8": torch.int64, "<f2": torch.float16, "<f4": torch.float32}
+
+        def mk(p, n, t):
+            if n == 0 or not p:
+                return torch.empty(0, dtype=tdt[t], device=self.device)
+            return torch.as_tensor(_CudaArray(p, (n,), t, self), device=self.device)
+        return {"blk_rowptr": mk(a.blk_rowptr, i.Bnrow + 1, "<i4"),
+                "blk_col": mk(a.blk_col, i.Bnnz, "<i4"),
+                "bitmap": mk(a.bitmap, i.Bnnz, "<i8"),       # uint64 bits viewed as int64
+                "blk_offset": mk(a.blk_offset, i.Bnnz + 1, "<i4"),
+                "values": mk(a.values, i.nnz, vt)}
+
+    def spmv(self, x, y=None, alpha: float = 1.0, beta: float = 0.0, stream=None):
+        """y = alpha * A x + beta * y on the device (x, y float32 CUDA tensors)."""
+        torch = _torch()
+        if y is None:
+            y = torch.empty(self.m, dtype=torch.float32, device=x.device)
+        assert x.dtype == torch.float32 and y.dtype == torch.float32
+        assert x.is_cuda and y.is_cuda and x.is_contiguous() and y.is_contiguous()
+        assert x.numel() == self.n and y.numel() == self.m
+        _check(spaden_spmv(self._h, alpha, ctypes.c_void_p(x.data_ptr()), beta,
+                           ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream)), "spaden_spmv")
+        return y
+
+    def spmv_host(self, x_host, y_host, alpha: float = 1.0, beta: float = 0.0, stream=None):
+        """Host-buffer variant (H2D x, SpMV, D2H y, stream sync) through the C ABI."""
+        _check(spaden_spmv_host(self._h, alpha, ctypes.c_void_p(x_host.data_ptr()), beta,
+                                ctypes.c_void_p(y_host.data_ptr()), _stream_ptr(stream)), "spaden_spmv_host")
+        return y_host
+
+    def free(self):
+        if self._h:
+            _check(spaden_free(self._h), "spaden_free")
+            self._h = None
+
+    def __del__(self):
+        try:
+            if self._h:
+                spaden_free(self._h)
+                self._h = None
+        except Exception:
+            pass
+
+
+def convert(rowptr, colidx, values, n: int, storage=None, stream=None) -> Matrix:
+    """CSR (int32 CUDA tensors + fp32/fp16 values) -> bitBSR Matrix."""
+    torch = _torch()
+    assert rowptr.dtype == torch.int32 and colidx.dtype == torch.int32
+    assert rowptr.is_cuda and colidx.is_cuda and values.is_cuda
+    vdt = _dtype_code(values.dtype)
+    sdt = vdt if storage is None else _dtype_code(storage)
+    m = rowptr.numel() - 1
+    h = ctypes.c_void_p()
+    st = spaden_convert_csr_to_bitmap(m, n, colidx.numel(), ctypes.c_void_p(rowptr.data_ptr()),
+                                      ctypes.c_void_p(colidx.data_ptr()),
+                                      ctypes.c_void_p(values.data_ptr()), vdt, sdt,
+                                      _stream_ptr(stream), ctypes.byref(h))
+    _check(st, "spaden_convert_csr_to_bitmap")
+    return Matrix(h, rowptr.device)

@@ -1,0 +1,214 @@
+// capi.cu -- the extern "C" boundary declared in include/spaden.h: argument
+// validation, handle lifetime, error strings.  All compute is in convert.cu /
+// spmv.cu kernels.
+#include <algorithm>
+#include <cstdio>
+#include <new>
+#include <string>
+
+#include "internal.cuh"
+
+namespace spaden {
+
+static thread_local std::string g_last_error;
+
+void set_error(const std::string &msg) { g_last_error = msg; }
+
+spaden_status_t cuda_status(cudaError_t e, const char *what) {
+    set_error(std::string(what) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")");
+    cudaGetLastError();  // clear sticky-free errors
+    if (e == cudaErrorMemoryAllocation) return SPADEN_ERR_OUT_OF_MEMORY;
+    return SPADEN_ERR_CUDA;
+}
+
+// device pointer on the current device (or managed), else INVALID_ARGUMENT
+static spaden_status_t check_device_ptr(const void *p, const char *name, int dev) {
+    cudaPointerAttributes at;
+    cudaError_t e = cudaPointerGetAttributes(&at, p);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_error(std::string(name) + " is not a CUDA device pointer");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (at.type != cudaMemoryTypeDevice && at.type != cudaMemoryTypeManaged) {
+        set_error(std::string(name) + " must be device memory");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (at.type == cudaMemoryTypeDevice && at.device != dev) {
+        set_error(std::string(name) + " lives on another device");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    return SPADEN_OK;
+}
+
+static void release(Matrix *A) {
+    if (!A) return;
+    void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap, A->blk_offset, A->values, A->stage_x, A->stage_y};
+    for (void *p : ptrs)
+        if (p) cudaFree(p);
+    delete A;
+}
+
+}  // namespace spaden
+
+using namespace spaden;
+
+extern "C" {
+
+const char *spaden_version(void) { return "spaden-b200 0.1 (sm_100a)"; }
+
+const char *spaden_status_string(spaden_status_t s) {
+    switch (s) {
+    case SPADEN_OK: return "SPADEN_OK";
+    case SPADEN_ERR_INVALID_ARGUMENT: return "SPADEN_ERR_INVALID_ARGUMENT";
+    case SPADEN_ERR_INDEX_OUT_OF_RANGE: return "SPADEN_ERR_INDEX_OUT_OF_RANGE";
+    case SPADEN_ERR_UNSORTED_OR_DUPLICATE: return "SPADEN_ERR_UNSORTED_OR_DUPLICATE";
+    case SPADEN_ERR_UNSUPPORTED: return "SPADEN_ERR_UNSUPPORTED";
+    case SPADEN_ERR_OUT_OF_MEMORY: return "SPADEN_ERR_OUT_OF_MEMORY";
+    case SPADEN_ERR_CUDA: return "SPADEN_ERR_CUDA";
+    }
+    return "SPADEN_ERR_UNKNOWN";
+}
+
+const char *spaden_last_error_message(void) { return g_last_error.c_str(); }
+
+spaden_status_t spaden_convert_csr_to_bitmap(int64_t m, int64_t n, int64_t nnz, const int32_t *d_rowptr,
+                                             const int32_t *d_colidx, const void *d_values,
+                                             spaden_dtype_t values_dtype, spaden_dtype_t storage_dtype,
+                                             void *stream, spaden_matrix_t *out) {
+    g_last_error.clear();
+    if (!out) {
+        set_error("out must not be NULL");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    *out = nullptr;
+    if (m < 0 || n < 0 || nnz < 0) {
+        set_error("m, n, nnz must be >= 0");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (m >= (1LL << 31) - 8 || n >= (1LL << 31) - 8 || nnz >= (1LL << 31) - 1) {
+        set_error("m, n, nnz must be < 2^31 (int32 indices)");
+        return SPADEN_ERR_UNSUPPORTED;
+    }
+    if ((values_dtype != SPADEN_R_32F && values_dtype != SPADEN_R_16F) ||
+        (storage_dtype != SPADEN_R_32F && storage_dtype != SPADEN_R_16F)) {
+        set_error("dtype must be SPADEN_R_32F or SPADEN_R_16F");
+        return SPADEN_ERR_UNSUPPORTED;
+    }
+    if (!d_rowptr || (nnz > 0 && (!d_colidx || !d_values))) {
+        set_error("NULL rowptr (or colidx/values with nnz > 0)");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_status(e, "cudaGetDevice");
+    spaden_status_t s = check_device_ptr(d_rowptr, "rowptr", dev);
+    if (s == SPADEN_OK && nnz > 0) s = check_device_ptr(d_colidx, "colidx", dev);
+    if (s == SPADEN_OK && nnz > 0) s = check_device_ptr(d_values, "values", dev);
+    if (s != SPADEN_OK) return s;
+
+    Matrix *A = new (std::nothrow) Matrix();
+    if (!A) {
+        set_error("host allocation failed");
+        return SPADEN_ERR_OUT_OF_MEMORY;
+    }
+    A->device = dev;
+    s = convert_csr(m, n, nnz, d_rowptr, d_colidx, d_values, values_dtype, storage_dtype,
+                    (cudaStream_t)stream, A);
+    if (s != SPADEN_OK) {
+        cudaStreamSynchronize((cudaStream_t)stream);
+        release(A);
+        return s;
+    }
+    *out = A;
+    return SPADEN_OK;
+}
+
+spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const float *d_x, float beta, float *d_y,
+                            void *stream) {
+    if (!A) {
+        set_error("NULL matrix handle");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if ((A->m > 0 && !d_y) || (A->Bnnz > 0 && !d_x)) {
+        set_error("NULL x or y");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (d_x && d_y && A->m > 0 && A->n > 0) {
+        const char *xb = (const char *)d_x, *xe = xb + 4 * A->n;
+        const char *yb = (const char *)d_y, *ye = yb + 4 * A->m;
+        if (xb < ye && yb < xe) {
+            set_error("x and y must not overlap");
+            return SPADEN_ERR_INVALID_ARGUMENT;
+        }
+    }
+    return spmv_launch(*A, alpha, d_x, beta, d_y, (cudaStream_t)stream);
+}
+
+spaden_status_t spaden_spmv_host(spaden_matrix_t A, float alpha, const float *h_x, float beta, float *h_y,
+                                 void *stream) {
+    if (!A || (A->n > 0 && !h_x) || (A->m > 0 && !h_y)) {
+        set_error("NULL handle or host vector");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    if (!A->stage_x && A->n > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->stage_x, pad16(4 * A->n)));
+    if (!A->stage_y && A->m > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->stage_y, pad16(4 * A->m)));
+    if (A->n > 0)
+        SPADEN_CUDA_TRY(cudaMemcpyAsync(A->stage_x, h_x, 4 * A->n, cudaMemcpyHostToDevice, st));
+    if (beta != 0.f && A->m > 0)
+        SPADEN_CUDA_TRY(cudaMemcpyAsync(A->stage_y, h_y, 4 * A->m, cudaMemcpyHostToDevice, st));
+    spaden_status_t s = spmv_launch(*A, alpha, A->stage_x, beta, A->stage_y, st);
+    if (s != SPADEN_OK) return s;
+    if (A->m > 0)
+        SPADEN_CUDA_TRY(cudaMemcpyAsync(h_y, A->stage_y, 4 * A->m, cudaMemcpyDeviceToHost, st));
+    SPADEN_CUDA_TRY(cudaStreamSynchronize(st));
+    return SPADEN_OK;
+}
+
+spaden_status_t spaden_free(spaden_matrix_t A) {
+    if (!A) return SPADEN_OK;
+    int cur = 0;
+    const int dev = A->device;
+    cudaGetDevice(&cur);
+    if (cur != dev) cudaSetDevice(dev);
+    cudaError_t e = cudaDeviceSynchronize();
+    release(A);
+    if (cur != dev) cudaSetDevice(cur);
+    if (e != cudaSuccess) return cuda_status(e, "cudaDeviceSynchronize in spaden_free");
+    return SPADEN_OK;
+}
+
+spaden_status_t spaden_get_info(spaden_matrix_t A, spaden_info_t *info) {
+    if (!A || !info) {
+        set_error("NULL handle or info");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    const int64_t sv = A->storage == SPADEN_R_16F ? 2 : 4;
+    info->m = A->m;
+    info->n = A->n;
+    info->nnz = A->nnz;
+    info->Bnrow = A->Bnrow;
+    info->Bnnz = A->Bnnz;
+    info->storage_dtype = (int32_t)A->storage;
+    info->device = A->device;
+    info->format_bytes = 4 * (A->Bnrow + 1) + 4 * A->Bnnz + 8 * A->Bnnz + 4 * (A->Bnnz + 1) + sv * A->nnz;
+    info->aux_bytes = A->aux_bytes;
+    info->n_tiles = A->n_tiles;
+    return SPADEN_OK;
+}
+
+spaden_status_t spaden_get_arrays(spaden_matrix_t A, spaden_arrays_t *v) {
+    if (!A || !v) {
+        set_error("NULL handle or arrays");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    v->blk_rowptr = A->blk_rowptr;
+    v->blk_col = A->blk_col;
+    v->bitmap = A->bitmap;
+    v->blk_offset = A->blk_offset;
+    v->values = A->values;
+    return SPADEN_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,408 @@
+// convert.cu -- GPU CSR -> bitBSR converter (
+// PAPER.md §4.2, Fig. 4).
+//
+// Work unit: a "chunk" = (block-row br, block-column range [bcl, bch)).  A
+// block-row holding more than kChunkNnz entries is split into several column
+// ranges so hub rows (R-MAT) spread over many warps.  One warp owns a chunk and
+// walks it in windows of 32 block columns, lane j <-> block column wbase+j:
+//   1. lanes 0..7 hold the cursor of row 8br+r; the window starts at the smallest
+//      pending block column of the 8 rows (so empty column ranges are skipped);
+//   2. each row with entries in the window is read coalesced (32 entries per
+//      load) and every entry ORs bit 8*(r%8)+(c%8) into its lane's
+//      bitmap word in shared memory;                                   [C3]
+//   3. lanes with a non-empty bitmap are blocks; ballot+popc ranks them
+//      (ascending block column, reading R5), a warp scan of popcounts gives
+//      blk_offset (P:L138 exclusive scan);                            [C3, C4]
+//   4. each entry is stored at blk_offset + popc(bitmap & ((1<<bit)-1))
+//      (ascending bit order = "stored consecutively", reading R4).  [C5]
+// The same walk runs twice: a count pass (which also validates the CSR) and,
+// after exclusive scans of the per-chunk block / value counts [C2] and the one
+// host sync that sizes the arrays, a fill pass.
+#include <climits>
+
+#include "internal.cuh"
+
+namespace spaden {
+namespace {
+
+constexpr int kChunkNnz = 4096;
+constexpr int kWarps = 8;
+constexpr unsigned kFull = 0xffffffffu;
+
+// per block-row: validate rowptr of its rows and decide the number of chunks
+__global__ void k_brinfo(int64_t m, int64_t nnz, int64_t NBC, const int32_t *__restrict__ rowptr,
+                         int32_t *__restrict__ nch, uint32_t *err) {
+    const int64_t Bnrow = (m + 7) / 8;
+    const int64_t br = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (br > Bnrow) return;
+    if (br == Bnrow) {  // global ends of rowptr
+        if (rowptr[0] != 0 || (int64_t)rowptr[m] != nnz) atomicOr(err, ERRF_ROWPTR);
+        return;
+    }
+    const int64_t r0 = 8 * br, r1 = min(r0 + 8, m);
+    int first = rowptr[r0], prev = first;
+    bool ok = first >= 0;
+    for (int64_t r = r0; r < r1; ++r) {
+        int nx = rowptr[r + 1];
+        ok = ok && nx >= prev;
+        prev = nx;
+    }
+    ok = ok && (int64_t)prev <= nnz;
+    if (!ok) {
+        atomicOr(err, ERRF_ROWPTR);
+        nch[br] = 1;
+        return;
+    }
+    int64_t c = ((int64_t)(prev - first) + kChunkNnz - 1) / kChunkNnz;
+    if (c < 1) c = 1;
+    if (NBC > 0 && c > NBC) c = NBC;
+    nch[br] = (int32_t)c;
+}
+
+__global__ void k_chunk_owner(int64_t Bnrow, const int32_t *__restrict__ chunk_start,
+                              int32_t *__restrict__ chunk_br) {
+    const int64_t br = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (br >= Bnrow) return;
+    for (int j = chunk_start[br]; j < chunk_start[br + 1]; ++j) chunk_br[j] = (int32_t)br;
+}
+
+__device__ __forceinline__ int lower_bound_col(const int32_t *__restrict__ col, int lo, int hi,
+                                               int64_t key) {
+    while (lo < hi) {
+        int mid = lo + ((hi - lo) >> 1);
+        if ((int64_t)col[mid] < key) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+// value movement: MODE 0 = 32-bit raw, 1 = 16-bit raw, 2 = f32 -> f16 RNE, 3 = f16 -> f32
+template <int MODE> struct VMove;
+template <> struct VMove<0> {
+    using In = uint32_t; using Out = uint32_t;
+    static __device__ __forceinline__ Out mv(In v) { return v; }
+};
+template <> struct VMove<1> {
+    using In = uint16_t; using Out = uint16_t;
+    static __device__ __forceinline__ Out mv(In v) { return v; }
+};
+template <> struct VMove<2> {
+    using In = float; using Out = __half;
+    static __device__ __forceinline__ Out mv(In v) { return __float2half_rn(v); }
+};
+template <> struct VMove<3> {
+    using In = __half; using Out = float;
+    static __device__ __forceinline__ Out mv(In v) { return __half2float(v); }
+};
+
+template <bool FILL, int MODE>
+__global__ void __launch_bounds__(kWarps * 32)
+k_tiles(int64_t m, int64_t n, int64_t NBC, const int32_t *__restrict__ rowptr,
+        const int32_t *__restrict__ colidx, const typename VMove<MODE>::In *__restrict__ vin,
+        const int32_t *__restrict__ chunk_start, const int32_t *__restrict__ chunk_br,
+        const int32_t *__restrict__ total_chunks, int32_t *__restrict__ cnt_blk,
+        int32_t *__restrict__ cnt_val, const int32_t *__restrict__ blk_start,
+        const int32_t *__restrict__ val_start, int32_t *__restrict__ blk_col,
+        uint64_t *__restrict__ bitmap, int32_t *__restrict__ blk_offset,
+        typename VMove<MODE>::Out *__restrict__ vout, uint32_t *err) {
+    __shared__ uint32_t words[kWarps][64];  // [0,32): bits 0-31, [32,64): bits 32-63 of lane j's block
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int64_t w = (int64_t)blockIdx.x * kWarps + wid;
+    if (!FILL && (*(volatile uint32_t *)err & ERRF_ROWPTR)) return;
+    if (w >= *total_chunks) return;  // warp-uniform
+    uint32_t *wd = words[wid];
+
+    const int br = chunk_br[w];
+    const int c0 = chunk_start[br];
+    const int nch = chunk_start[br + 1] - c0;
+    const int c = (int)(w - c0);
+    const int64_t wdt = (NBC + nch - 1) / nch;
+    const int64_t bcl = (int64_t)c * wdt;
+    const int64_t bch = min(NBC, bcl + wdt);
+    const int64_t lo_col = 8 * bcl, hi_col = 8 * bch;
+
+    // lanes 0..7: slice [cur, end) of row 8br+lane inside the chunk's column range
+    int cur = 0, end = 0;
+    const int64_t row = 8 * (int64_t)br + lane;
+    if (lane < 8 && row < m) {
+        const int rs = rowptr[row], re = rowptr[row + 1];
+        cur = (c == 0) ? rs : lower_bound_col(colidx, rs, re, lo_col);
+        end = (c == nch - 1) ? re : lower_bound_col(colidx, rs, re, hi_col);
+        if (end < cur) end = cur;
+    }
+    int carry = INT_MIN;  // lanes 0..7: last column seen in the row (sortedness check)
+    int bcur = 0, vcur = 0, nblk = 0;
+    if (FILL) {
+        bcur = blk_start[w];
+        vcur = val_start[w];
+    }
+
+    while (true) {
+        const int nxt = (lane < 8 && cur < end) ? (colidx[cur] >> 3) : INT_MAX;
+        const int wbase = warp_min_i32(nxt);
+        if (wbase == INT_MAX) break;
+        wd[lane] = 0u;
+        wd[lane + 32] = 0u;
+        __syncwarp();
+        const unsigned rows = __ballot_sync(kFull, nxt != INT_MAX && nxt < wbase + 32);
+        int adv = 0;
+        // ---- pass A: OR every in-window entry into its block's bitmap word
+        for (unsigned rm = rows; rm; rm &= rm - 1) {
+            const int r = __ffs(rm) - 1;
+            int s = __shfl_sync(kFull, cur, r);
+            const int e = __shfl_sync(kFull, end, r);
+            int prevc = __shfl_sync(kFull, carry, r);
+            const int s0 = s;
+            while (s < e) {
+                const int k = s + lane;
+                const bool in = k < e;
+                const int col = in ? colidx[k] : INT_MAX;
+                const int bc = col >> 3;
+                const bool inwin = in && bc < wbase + 32;
+                if (!FILL) {
+                    if (in && (col < 0 || (int64_t)col >= n)) atomicOr(err, ERRF_RANGE);
+                    // a binary-searched slice holding columns outside its chunk's
+                    // range can only come from an unsorted row
+                    else if (in && ((int64_t)col < lo_col || (int64_t)col >= hi_col))
+                        atomicOr(err, ERRF_UNSORTED);
+                    int pc = __shfl_up_sync(kFull, col, 1);
+                    if (lane == 0) pc = prevc;
+                    if (inwin && col <= pc) atomicOr(err, ERRF_UNSORTED);
+                }
+                const unsigned wm = __ballot_sync(kFull, inwin);
+                const int t = bc - wbase;
+                if (inwin && col >= 0 && t >= 0 && t < 32) {
+                    const int bit = 8 * r + (col & 7);
+                    atomicOr(&wd[t + (bit & 32)], 1u << (bit & 31));
+                }
+                const int nin = __popc(wm);
+                if (nin) prevc = __shfl_sync(kFull, col, 31 - __clz(wm));
+                s += nin;
+                if (nin < 32) break;
+            }
+            if (lane == r) {
+                adv = s - s0;
+                carry = prevc;
+            }
+        }
+        __syncwarp();
+        const uint64_t bmp = (uint64_t)wd[lane] | ((uint64_t)wd[lane + 32] << 32);
+        const unsigned nem = __ballot_sync(kFull, bmp != 0ull);
+        if (FILL) {
+            const int rank = __popc(nem & ((1u << lane) - 1u));
+            int vtot;
+            const int vex = warp_excl_scan_i32(__popcll(bmp), lane, &vtot);
+            const int myoff = vcur + vex;
+            if (bmp != 0ull) {
+                const int idx = bcur + rank;
+                blk_col[idx] = wbase + lane;
+                bitmap[idx] = bmp;
+                blk_offset[idx] = myoff;
+            }
+            const uint32_t blo = (uint32_t)bmp, bhi = (uint32_t)(bmp >> 32);
+            // ---- pass B: place every in-window value at its popcount rank
+            for (unsigned rm = rows; rm; rm &= rm - 1) {
+                const int r = __ffs(rm) - 1;
+                const int s0 = __shfl_sync(kFull, cur, r);
+                const int e = s0 + __shfl_sync(kFull, adv, r);
+                for (int s = s0; s < e; s += 32) {
+                    const int k = s + lane;
+                    const bool in = k < e;
+                    const int col = in ? colidx[k] : 0;
+                    const int t = ((col >> 3) - wbase) & 31;
+                    const uint32_t tl = __shfl_sync(kFull, blo, t);
+                    const uint32_t th = __shfl_sync(kFull, bhi, t);
+                    const int toff = __shfl_sync(kFull, myoff, t);
+                    if (in) {
+                        const int bit = 8 * r + (col & 7);
+                        const uint64_t below = (((uint64_t)th << 32) | tl) & ((1ull << bit) - 1ull);
+                        vout[toff + __popcll(below)] = VMove<MODE>::mv(vin[k]);
+                    }
+                }
+            }
+            vcur += vtot;
+        }
+        bcur += __popc(nem);
+        nblk += __popc(nem);
+        if (lane < 8) cur += adv;
+        __syncwarp();
+    }
+    if (!FILL && lane == 0) cnt_blk[w] = nblk;
+}
+
+// per-chunk value counts (independent of the walk so the scan is exact)
+__global__ void k_chunk_vals(int64_t m, int64_t NBC, const int32_t *__restrict__ rowptr,
+                             const int32_t *__restrict__ colidx, const int32_t *__restrict__ chunk_start,
+                             const int32_t *__restrict__ chunk_br, const int32_t *__restrict__ total_chunks,
+                             int32_t *__restrict__ cnt_val, const uint32_t *err) {
+    const int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (*(volatile const uint32_t *)err & ERRF_ROWPTR) return;
+    if (w >= *total_chunks) return;
+    const int br = chunk_br[w];
+    const int c0 = chunk_start[br];
+    const int nch = chunk_start[br + 1] - c0;
+    const int c = (int)(w - c0);
+    const int64_t wdt = (NBC + nch - 1) / nch;
+    const int64_t bcl = (int64_t)c * wdt;
+    const int64_t bch = min(NBC, bcl + wdt);
+    int total = 0;
+    for (int r = 0; r < 8; ++r) {
+        const int64_t row = 8 * (int64_t)br + r;
+        if (row >= m) break;
+        const int rs = rowptr[row], re = rowptr[row + 1];
+        const int cur = (c == 0) ? rs : lower_bound_col(colidx, rs, re, 8 * bcl);
+        int end = (c == nch - 1) ? re : lower_bound_col(colidx, rs, re, 8 * bch);
+        if (end < cur) end = cur;
+        total += end - cur;
+    }
+    cnt_val[w] = total;
+}
+
+__global__ void k_summary(const uint32_t *err, const int32_t *total_chunks, const int32_t *bnnz,
+                          const int32_t *nvals, int32_t *out4) {
+    out4[0] = (int32_t)*err;
+    out4[1] = *total_chunks;
+    out4[2] = *bnnz;
+    out4[3] = *nvals;
+}
+
+__global__ void k_finalize(int64_t Bnrow, int64_t Bnnz, int64_t nnz, const int32_t *__restrict__ chunk_start,
+                           const int32_t *__restrict__ blk_start, int32_t *__restrict__ blk_rowptr,
+                           int32_t *__restrict__ blk_offset) {
+    const int64_t br = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (br < Bnrow) blk_rowptr[br] = blk_start[chunk_start[br]];
+    if (br == Bnrow) {
+        blk_rowptr[Bnrow] = (int32_t)Bnnz;
+        blk_offset[Bnnz] = (int32_t)nnz;
+    }
+}
+
+inline unsigned grid_for(int64_t threads, int per) { return (unsigned)((threads + per - 1) / per); }
+
+struct TempPool {
+    void *base = nullptr;
+    cudaStream_t s = nullptr;
+    ~TempPool() {
+        if (base) cudaFreeAsync(base, s);
+    }
+};
+
+template <int MODE>
+void launch_fill(int64_t m, int64_t n, int64_t NBC, const int32_t *rowptr, const int32_t *colidx,
+                 const void *vin, const int32_t *chunk_start, const int32_t *chunk_br,
+                 const int32_t *total_chunks, int64_t nchunks, const int32_t *blk_start,
+                 const int32_t *val_start, Matrix *A, uint32_t *err, cudaStream_t st) {
+    using M = VMove<MODE>;
+    k_tiles<true, MODE><<<grid_for(nchunks, kWarps), kWarps * 32, 0, st>>>(
+        m, n, NBC, rowptr, colidx, (const typename M::In *)vin, chunk_start, chunk_br, total_chunks,
+        nullptr, nullptr, blk_start, val_start, A->blk_col, A->bitmap, A->blk_offset,
+        (typename M::Out *)A->values, err);
+}
+
+}  // namespace
+
+spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *rowptr,
+                            const int32_t *colidx, const void *values, spaden_dtype_t vdt,
+                            spaden_dtype_t sdt, cudaStream_t st, Matrix *A) {
+    const int64_t Bnrow = (m + 7) / 8;
+    const int64_t NBC = (n + 7) / 8;
+    const int64_t max_chunks = Bnrow + nnz / kChunkNnz + 1;
+    const size_t sv = (sdt == SPADEN_R_16F) ? 2 : 4;
+
+    // ---- temporaries (stream-ordered)
+    const size_t n_nch = (size_t)Bnrow + 1;
+    const size_t n_cnt = (size_t)max_chunks + 1;
+    const size_t n_tmp = scan_tmp_ints(std::max<int64_t>(max_chunks, Bnrow) + 1);
+    const size_t ints = n_nch + (size_t)max_chunks + 2 * n_cnt + n_tmp + 8;
+    TempPool pool;
+    pool.s = st;
+    SPADEN_CUDA_TRY(cudaMallocAsync(&pool.base, ints * sizeof(int32_t), st));
+    int32_t *p = (int32_t *)pool.base;
+    int32_t *chunk_start = p; p += n_nch;
+    int32_t *chunk_br = p; p += max_chunks;
+    int32_t *cnt_blk = p; p += n_cnt;
+    int32_t *cnt_val = p; p += n_cnt;
+    int32_t *scan_tmp = p; p += n_tmp;
+    uint32_t *err = (uint32_t *)p; p += 4;
+    int32_t *summary = p;
+    SPADEN_CUDA_TRY(cudaMemsetAsync(err, 0, sizeof(uint32_t), st));
+    SPADEN_CUDA_TRY(cudaMemsetAsync(cnt_blk, 0, 2 * n_cnt * sizeof(int32_t), st));
+
+    // C1: per block-row chunking + rowptr validation, chunk owners
+    k_brinfo<<<grid_for(Bnrow + 1, 256), 256, 0, st>>>(m, nnz, NBC, rowptr, chunk_start, err);
+    SPADEN_CUDA_TRY(exclusive_scan_i32(chunk_start, chunk_start, Bnrow, scan_tmp, st));
+    const int32_t *total_chunks = chunk_start + Bnrow;
+    if (Bnrow > 0) k_chunk_owner<<<grid_for(Bnrow, 256), 256, 0, st>>>(Bnrow, chunk_start, chunk_br);
+    // C1/C3 count pass (+ colidx validation)
+    if (Bnrow > 0) {
+        k_tiles<false, 0><<<grid_for(max_chunks, kWarps), kWarps * 32, 0, st>>>(
+            m, n, NBC, rowptr, colidx, nullptr, chunk_start, chunk_br, total_chunks, cnt_blk, cnt_val,
+            nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, err);
+        k_chunk_vals<<<grid_for(max_chunks, 256), 256, 0, st>>>(m, NBC, rowptr, colidx, chunk_start,
+                                                                 chunk_br, total_chunks, cnt_val, err);
+    }
+    SPADEN_CUDA_TRY(cudaGetLastError());
+    // C2/C4: chunk -> first block / first value
+    SPADEN_CUDA_TRY(exclusive_scan_i32(cnt_blk, cnt_blk, max_chunks, scan_tmp, st));
+    SPADEN_CUDA_TRY(exclusive_scan_i32(cnt_val, cnt_val, max_chunks, scan_tmp, st));
+    k_summary<<<1, 1, 0, st>>>(err, total_chunks, cnt_blk + max_chunks, cnt_val + max_chunks, summary);
+    int32_t h[4] = {0, 0, 0, 0};
+    SPADEN_CUDA_TRY(cudaMemcpyAsync(h, summary, sizeof(h), cudaMemcpyDeviceToHost, st));
+    SPADEN_CUDA_TRY(cudaStreamSynchronize(st));  // the converter's one host sync
+    const uint32_t eflags = (uint32_t)h[0];
+    if (eflags & ERRF_ROWPTR) {
+        set_error("rowptr must satisfy rowptr[0]==0, non-decreasing, rowptr[m]==nnz");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (eflags & ERRF_RANGE) {
+        set_error("colidx outside [0, n)");
+        return SPADEN_ERR_INDEX_OUT_OF_RANGE;
+    }
+    if (eflags & ERRF_UNSORTED) {
+        set_error("colidx not strictly ascending within a row (unsorted or duplicate)");
+        return SPADEN_ERR_UNSORTED_OR_DUPLICATE;
+    }
+    const int64_t nchunks = h[1];
+    const int64_t Bnnz = h[2];
+    if ((int64_t)h[3] != nnz) {
+        set_error("internal: chunk value count mismatch");
+        return SPADEN_ERR_CUDA;
+    }
+
+    // ---- owned arrays
+    A->m = m; A->n = n; A->nnz = nnz; A->Bnrow = Bnrow; A->Bnnz = Bnnz; A->storage = sdt;
+    auto alloc = [&](void **ptr, size_t bytes) -> cudaError_t {
+        cudaError_t e = cudaMalloc(ptr, pad16(bytes));
+        if (e == cudaSuccess) e = cudaMemsetAsync(*ptr, 0, pad16(bytes), st);
+        return e;
+    };
+    cudaError_t e = cudaSuccess;
+    if (e == cudaSuccess) e = alloc((void **)&A->blk_rowptr, sizeof(int32_t) * (Bnrow + 1));
+    if (e == cudaSuccess) e = alloc((void **)&A->blk_col, sizeof(int32_t) * Bnnz);
+    if (e == cudaSuccess) e = alloc((void **)&A->bitmap, sizeof(uint64_t) * Bnnz);
+    if (e == cudaSuccess) e = alloc((void **)&A->blk_offset, sizeof(int32_t) * (Bnnz + 1));
+    if (e == cudaSuccess) e = alloc(&A->values, sv * nnz);
+    if (e != cudaSuccess) return cuda_status(e, "allocating bitBSR arrays");
+
+    // C3-C5 fill pass
+    if (nchunks > 0 && nnz > 0) {
+        if (vdt == SPADEN_R_32F && sdt == SPADEN_R_32F)
+            launch_fill<0>(m, n, NBC, rowptr, colidx, values, chunk_start, chunk_br, total_chunks, nchunks,
+                           cnt_blk, cnt_val, A, err, st);
+        else if (vdt == SPADEN_R_16F && sdt == SPADEN_R_16F)
+            launch_fill<1>(m, n, NBC, rowptr, colidx, values, chunk_start, chunk_br, total_chunks, nchunks,
+                           cnt_blk, cnt_val, A, err, st);
+        else if (vdt == SPADEN_R_32F && sdt == SPADEN_R_16F)
+            launch_fill<2>(m, n, NBC, rowptr, colidx, values, chunk_start, chunk_br, total_chunks, nchunks,
+                           cnt_blk, cnt_val, A, err, st);
+        else
+            launch_fill<3>(m, n, NBC, rowptr, colidx, values, chunk_start, chunk_br, total_chunks, nchunks,
+                           cnt_blk, cnt_val, A, err, st);
+    }
+    k_finalize<<<grid_for(Bnrow + 1, 256), 256, 0, st>>>(Bnrow, Bnnz, nnz, chunk_start, cnt_blk,
+                                                         A->blk_rowptr, A->blk_offset);
+    SPADEN_CUDA_TRY(cudaGetLastError());
+    return SPADEN_OK;
+}
+
+}  // namespace spaden

@@ -1,0 +1,387 @@
+"""Parity of the CUDA path (through the C ABI) against the CPU oracle.
+
+Conversion: bit-exact (memcmp of all five bitBSR arrays against oracle/'s
+reference converter, plus oracle decode back to the input CSR).
+SpMV: fp32 values componentwise |y - y*| / s <= 1e-5; fp16 values componentwise
+1e-5 against the oracle on the stored fp16 values and normwise 1e-2 against the
+original fp32 values (BASELINE north_star).  Closed
+forms (identity / permutation / diagonal / small integers / H1 / H2) bitwise.
+"""
+import ctypes
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+TOL32 = 1e-5
+TOL16_NORM = 1e-2
+
+
+@pytest.fixture(scope="module")
+def sp():
+    import paper_conf_icpp_cheny24_b200 as sp
+    return sp
+
+
+@pytest.fixture(scope="module")
+def torch():
+    import torch
+    assert torch.cuda.is_available()
+    return torch
+
+
+def dev(torch, A, values=None):
+    vals = A.values if values is None else values
+    return (torch.from_numpy(np.ascontiguousarray(A.rowptr)).cuda(),
+            torch.from_numpy(np.ascontiguousarray(A.colidx)).cuda(),
+            torch.from_numpy(np.ascontiguousarray(vals)).cuda())
+
+
+def convert(sp, torch, A, values=None, storage=None):
+    rp, ci, v = dev(torch, A, values)
+    M = sp.convert(rp, ci, v, A.n, storage=storage)
+    torch.cuda.synchronize()
+    return M
+
+
+def host_arrays(torch, M):
+    return {k: t.cpu().numpy() for k, t in M.arrays().items()}
+
+
+def assert_format_parity(torch, M, A, values):
+    st, B = oracle.csr_to_bitbsr(A.m, A.n, A.rowptr, A.colidx, values)
+    assert st == 0
+    h = host_arrays(torch, M)
+    i = M.info
+    assert (i.m, i.n, i.nnz, i.Bnrow, i.Bnnz) == (A.m, A.n, A.nnz, B.Bnrow, B.Bnnz)
+    assert np.array_equal(h["blk_rowptr"].astype(np.int64), B.blk_rowptr)
+    if B.Bnnz:
+        assert np.array_equal(h["blk_col"], B.blk_col)
+        assert np.array_equal(h["bitmap"].view(np.uint64), B.bitmap)
+    assert np.array_equal(h["blk_offset"].astype(np.int64), B.blk_offset)
+    if A.nnz:
+        ub = np.uint16 if values.dtype == np.float16 else np.uint32
+        assert np.array_equal(h["values"].view(ub), np.ascontiguousarray(B.values).view(ub))
+    # footprint formula
+    assert i.format_bytes == oracle.bitbsr_bytes(A.m, B.Bnnz, A.nnz, values.dtype.itemsize)
+    # decode(GPU arrays) == input CSR, bit for bit
+    G = oracle.BitBSR(A.m, A.n, h["blk_rowptr"].astype(np.int64), h["blk_col"] if B.Bnnz else B.blk_col,
+                      h["bitmap"].view(np.uint64) if B.Bnnz else B.bitmap,
+                      h["blk_offset"].astype(np.int64), h["values"] if A.nnz else values[:0])
+    rp, ci, vv = oracle.bitbsr_to_csr(G)
+    assert np.array_equal(rp, A.rowptr.astype(np.int64))
+    assert np.array_equal(ci, A.colidx)
+    ub = np.uint16 if values.dtype == np.float16 else np.uint32
+    assert np.array_equal(np.ascontiguousarray(vv).view(ub), np.ascontiguousarray(values).view(ub))
+    return B
+
+
+def gpu_spmv(torch, M, x, alpha=1.0, beta=0.0, y0=None):
+    xd = torch.from_numpy(np.ascontiguousarray(x, dtype=np.float32)).cuda()
+    yd = torch.from_numpy(np.ascontiguousarray(y0, dtype=np.float32)).cuda() if y0 is not None else None
+    y = M.spmv(xd, yd, alpha=alpha, beta=beta)
+    torch.cuda.synchronize()
+    return y.cpu().numpy()
+
+
+CASES = {
+    "h1": lambda: W.h1(),
+    "h2": lambda: W.h2(),
+    "identity1": lambda: W.identity(1),
+    "identity7": lambda: W.identity(7),
+    "identity9": lambda: W.identity(9),
+    "identity1023": lambda: W.identity(1023),
+    "reversal64": lambda: W.reversal(64),
+    "perm1000": lambda: W.permutation(W.random_perm(1000, 3)),
+    "diag1024": lambda: W.diagonal(1024, 1),
+    "dense8": lambda: W.dense_block(8, 8),
+    "dense64": lambda: W.dense_block(64, 64, 2),
+    "corner": lambda: W.from_coo(13, 21, [12], [20], [3.0]),
+    "empty_middle_last": lambda: W.from_coo(40, 40, [0, 30], [39, 0], [1.0, 2.0]),
+    "rand_rect": lambda: W.random_sparse(333, 517, 0.02, 5),
+    "rand_dense": lambda: W.random_sparse(129, 65, 0.6, 6),
+    "tiny": lambda: W.tiny(0),
+    "hub": lambda: hub_matrix(),
+}
+
+
+def hub_matrix(m=64, n=100_003, hub_rows=(3, 9, 60), hub_nnz=30_000, seed=7):
+    """A few hub rows spanning many block columns (forces the chunked converter path)."""
+    rng = np.random.default_rng(seed)
+    rows, cols = [], []
+    for r in hub_rows:
+        c = rng.choice(n, hub_nnz, replace=False)
+        rows.append(np.full(c.size, r))
+        cols.append(c)
+    for r in range(m):
+        c = rng.choice(n, 5, replace=False)
+        rows.append(np.full(5, r))
+        cols.append(c)
+    rows = np.concatenate(rows)
+    cols = np.concatenate(cols)
+    key = np.unique(rows.astype(np.int64) * n + cols)
+    r, c = np.divmod(key, n)
+    return W.from_coo(m, n, r, c, rng.uniform(-1, 1, key.size))
+
+
+@pytest.mark.parametrize("name", sorted(CASES))
+@pytest.mark.parametrize("mode", ["f32>f32", "f32>f16", "f16>f16", "f16>f32"])
+def test_conversion_bit_exact(sp, torch, name, mode):
+    A = CASES[name]()
+    vin = A.values.astype(np.float16) if mode.startswith("f16") else A.values
+    if mode == "f32>f16":
+        stored = oracle.f32_to_f16(A.values)
+    elif mode == "f16>f32":
+        stored = vin.astype(np.float32)
+    else:
+        stored = vin
+    M = convert(sp, torch, A, values=vin, storage="fp16" if mode.endswith("f16") else "fp32")
+    h = host_arrays(torch, M)
+    # the reference converter applied to the oracle-rounded values
+    Aref = W.CSR(A.m, A.n, A.rowptr, A.colidx, stored)
+    assert_format_parity(torch, M, Aref, stored)
+    M.free()
+
+
+@pytest.mark.parametrize("m,n", [(0, 0), (0, 7), (7, 0), (8, 8), (17, 3)])
+def test_empty_matrices(sp, torch, m, n):
+    A = W.CSR(m, n, np.zeros(m + 1, np.int32), np.zeros(0, np.int32), np.zeros(0, np.float32))
+    rp = torch.zeros(m + 1, dtype=torch.int32, device="cuda")
+    ci = torch.zeros(1, dtype=torch.int32, device="cuda")
+    v = torch.zeros(1, dtype=torch.float32, device="cuda")
+    h = ctypes.c_void_p()
+    st = sp.spaden_convert_csr_to_bitmap(m, n, 0, rp.data_ptr(), ci.data_ptr(), v.data_ptr(), 0, 0,
+                                         torch.cuda.current_stream().cuda_stream, ctypes.byref(h))
+    assert st == 0
+    M = sp.Matrix(h, rp.device)
+    assert M.info.Bnnz == 0 and M.info.Bnrow == (m + 7) // 8
+    if m:
+        x = torch.ones(max(n, 1), device="cuda")[:n].contiguous() if n else torch.zeros(0, device="cuda")
+        y0 = torch.full((m,), float("nan"), device="cuda")
+        st = sp.spaden_spmv(M.handle, 1.0, x.data_ptr() or None, 0.0, y0.data_ptr(), None)
+        torch.cuda.synchronize()
+        assert st == 0 and (y0 == 0).all()
+        y1 = torch.full((m,), 2.0, device="cuda")
+        sp.spaden_spmv(M.handle, 1.0, x.data_ptr() or None, 0.5, y1.data_ptr(), None)
+        torch.cuda.synchronize()
+        assert (y1 == 1.0).all()
+    M.free()
+
+
+def bad_inputs():
+    rp = np.array([0, 2, 4], np.int32)
+    ci = np.array([1, 3, 0, 2], np.int32)
+    yield "unsorted", rp, np.array([3, 1, 0, 2], np.int32), 3
+    yield "dup", rp, np.array([1, 1, 0, 2], np.int32), 3
+    yield "col_n", rp, np.array([1, 4, 0, 2], np.int32), 2
+    yield "col_neg", rp, np.array([-1, 3, 0, 2], np.int32), 2
+    yield "rowptr_nonmono", np.array([0, 3, 2], np.int32), ci, 1
+    yield "rowptr_end", np.array([0, 2, 3], np.int32), ci, 1
+    yield "rowptr_start", np.array([1, 2, 4], np.int32), ci, 1
+
+
+@pytest.mark.parametrize("case", list(bad_inputs()), ids=lambda c: c[0])
+def test_rejects_invalid_csr(sp, torch, case):
+    _, rp, ci, code = case
+    rpd, cid = torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda()
+    v = torch.ones(4, device="cuda")
+    h = ctypes.c_void_p()
+    st = sp.spaden_convert_csr_to_bitmap(2, 4, 4, rpd.data_ptr(), cid.data_ptr(), v.data_ptr(), 0, 0,
+                                         None, ctypes.byref(h))
+    assert st == code and h.value is None
+
+
+def test_rejects_unsorted_hub_row_and_host_pointer(sp, torch):
+    A = hub_matrix()
+    ci = A.colidx.copy()
+    k = int(A.rowptr[9]) + 20_000          # inside a chunked hub row
+    ci[k], ci[k + 1] = ci[k + 1], ci[k]
+    h = ctypes.c_void_p()
+    rp, cid, v = dev(torch, A)
+    cid.copy_(torch.from_numpy(ci))
+    st = sp.spaden_convert_csr_to_bitmap(A.m, A.n, A.nnz, rp.data_ptr(), cid.data_ptr(), v.data_ptr(), 0, 0,
+                                         None, ctypes.byref(h))
+    assert st == sp.SPADEN_ERR_UNSORTED_OR_DUPLICATE
+    host_rp = np.zeros(A.m + 1, np.int32)
+    st = sp.spaden_convert_csr_to_bitmap(A.m, A.n, 0, host_rp.ctypes.data, None, None, 0, 0, None,
+                                         ctypes.byref(h))
+    assert st == sp.SPADEN_ERR_INVALID_ARGUMENT
+
+
+# ------------------------------------------------------------------ SpMV
+def check_spmv(A, y, stored, x):
+    ys, s = oracle.spmv(A.rowptr, A.colidx, stored, x)
+    err = oracle.componentwise_error(y, ys, s)
+    assert err <= TOL32, err
+    return ys
+
+
+@pytest.mark.parametrize("name", sorted(CASES))
+def test_spmv_fp32(sp, torch, name):
+    A = CASES[name]()
+    M = convert(sp, torch, A)
+    x = W.vector(A.n, 11)
+    y = gpu_spmv(torch, M, x)
+    check_spmv(A, y, A.values, x)
+
+
+@pytest.mark.parametrize("name", sorted(CASES))
+def test_spmv_fp16(sp, torch, name):
+    A = CASES[name]()
+    M = convert(sp, torch, A, storage="fp16")
+    x = W.vector(A.n, 12)
+    y = gpu_spmv(torch, M, x)
+    stored = oracle.f32_to_f16(A.values)
+    check_spmv(A, y, stored, x)
+    y32, _ = oracle.spmv(A.rowptr, A.colidx, A.values, x)
+    nerr = oracle.normwise_error(y, y32, oracle.csr_inf_norm(A.rowptr, A.values), float(np.abs(x).max(initial=0)))
+    assert nerr <= TOL16_NORM
+
+
+@pytest.mark.parametrize("name", ["h1", "h2"])
+def test_spmv_hand_worked_exact(sp, torch, name):
+    import json, os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", name + ".json")))
+    A = CASES[name]()
+    M = convert(sp, torch, A)
+    y = gpu_spmv(torch, M, np.arange(1, A.n + 1, dtype=np.float32))
+    assert y.tolist() == [float(v) for v in g["y"]]
+
+
+def test_spmv_closed_forms_bitwise(sp, torch):
+    for n in (1, 7, 8, 9, 1023, 1024):
+        x = W.vector(n, n)
+        assert np.array_equal(gpu_spmv(torch, convert(sp, torch, W.identity(n)), x), x)
+        perm = W.random_perm(n, n)
+        assert np.array_equal(gpu_spmv(torch, convert(sp, torch, W.permutation(perm)), x), x[perm])
+        D = W.diagonal(n, n)
+        assert np.array_equal(gpu_spmv(torch, convert(sp, torch, D), x), (D.values * x).astype(np.float32))
+    A = W.random_sparse(300, 280, 0.2, 1, dist="int")
+    x = np.random.default_rng(2).integers(-8, 9, 280).astype(np.float32)
+    y = gpu_spmv(torch, convert(sp, torch, A), x)
+    ys, _ = oracle.spmv(A.rowptr, A.colidx, A.values, x)
+    assert np.array_equal(y.astype(np.float64), ys)
+
+
+def test_alpha_beta_and_nan_semantics(sp, torch):
+    A = W.random_sparse(200, 190, 0.05, 4)
+    M = convert(sp, torch, A)
+    x = W.vector(190, 1)
+    y0 = W.vector(200, 2)
+    y = gpu_spmv(torch, M, x, alpha=2.0, beta=0.5, y0=y0)
+    ys, s = oracle.spmv(A.rowptr, A.colidx, A.values, x)
+    ref = 2.0 * ys + 0.5 * y0.astype(np.float64)
+    assert oracle.componentwise_error(y, ref, 2.0 * s + 0.5 * np.abs(y0)) <= TOL32
+    # beta == 0: y's old contents (NaN) are ignored
+    y = gpu_spmv(torch, M, x, beta=0.0, y0=np.full(200, np.nan, np.float32))
+    assert np.isfinite(y).all()
+    # a NaN in x only reaches rows that reference that column (structural zeros never multiplied)
+    j = int(A.colidx[0])
+    xn = x.copy()
+    xn[j] = np.nan
+    y = gpu_spmv(torch, M, xn)
+    dense_ref = np.zeros(200, bool)
+    for i in range(200):
+        dense_ref[i] = j in A.colidx[A.rowptr[i]:A.rowptr[i + 1]]
+    assert np.array_equal(np.isnan(y), dense_ref)
+
+
+def test_unaligned_x(sp, torch):
+    A = W.random_sparse(100, 97, 0.1, 3)
+    M = convert(sp, torch, A)
+    x = W.vector(97, 4)
+    buf = torch.zeros(98, device="cuda")
+    buf[1:].copy_(torch.from_numpy(x))
+    xv = buf[1:]
+    y = M.spmv(xv)
+    torch.cuda.synchronize()
+    check_spmv(A, y.cpu().numpy(), A.values, x)
+
+
+def test_deterministic_and_partition_invariant(sp, torch):
+    A = W.make("fem62k")
+    x = W.vector(A.n, 5)
+    M = convert(sp, torch, A)
+    y1 = gpu_spmv(torch, M, x)
+    y2 = gpu_spmv(torch, M, x)
+    assert np.array_equal(y1, y2)
+    parts = []
+    bounds = [0, 8 * 1000, 8 * 3001, 8 * 5000, A.m]
+    for r0, r1 in zip(bounds[:-1], bounds[1:]):
+        S = A.row_slice(r0, r1)
+        parts.append(gpu_spmv(torch, convert(sp, torch, S), x))
+    assert np.array_equal(np.concatenate(parts), y1)
+    check_spmv(A, y1, A.values, x)
+
+
+def test_spmv_host_matches_device(sp, torch):
+    A = W.tiny(0)
+    M = convert(sp, torch, A)
+    x = W.vector(A.n, 8)
+    yd = gpu_spmv(torch, M, x)
+    xh = torch.from_numpy(x).pin_memory()
+    yh = torch.empty(A.m, dtype=torch.float32).pin_memory()
+    M.spmv_host(xh, yh)
+    assert np.array_equal(yh.numpy(), yd)
+
+
+def test_cuda_graph_capture(sp, torch):
+    A = W.tiny(1)
+    M = convert(sp, torch, A)
+    x = torch.from_numpy(W.vector(A.n, 9)).cuda()
+    y = torch.empty(A.m, device="cuda")
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        M.spmv(x, y)
+    torch.cuda.synchronize()
+    ref = y.clone()
+    y.zero_()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        M.spmv(x, y, stream=s)
+    g.replay()
+    torch.cuda.synchronize()
+    assert torch.equal(y, ref)
+
+
+@pytest.mark.parametrize("name", ["fem62k", "powerlaw1m"])
+def test_configs_full(sp, torch, name):
+    A = W.make(name)
+    M = convert(sp, torch, A)
+    assert_format_parity(torch, M, A, A.values)
+    x = W.vector(A.n, 21)
+    check_spmv(A, gpu_spmv(torch, M, x), A.values, x)
+    M16 = convert(sp, torch, A, storage="fp16")
+    y = gpu_spmv(torch, M16, x)
+    check_spmv(A, y, oracle.f32_to_f16(A.values), x)
+
+
+@pytest.mark.slow
+def test_fem1p5m_full(sp, torch):
+    """BASELINE configs[3] at full size, in the launch configuration bench.py times."""
+    A = W.make("fem1p5m")
+    x = W.vector(A.n, 31)
+    for storage, stored in (("fp32", A.values), ("fp16", oracle.f32_to_f16(A.values))):
+        M = convert(sp, torch, A, storage=storage)
+        i = M.info
+        assert i.nnz == A.nnz and i.Bnrow == (A.m + 7) // 8
+        assert i.format_bytes == oracle.bitbsr_bytes(A.m, i.Bnnz, A.nnz, 2 if storage == "fp16" else 4)
+        check_spmv(A, gpu_spmv(torch, M, x), stored, x)
+        # sampled block-rows of the format against the reference converter on a row slice
+        h = M.arrays()
+        rng = np.random.default_rng(0)
+        for br in rng.choice(i.Bnrow, 64, replace=False):
+            S = A.row_slice(8 * int(br), 8 * int(br) + 8)
+            st, B = oracle.csr_to_bitbsr(S.m, S.n, S.rowptr, S.colidx, stored[A.rowptr[8 * br]:A.rowptr[min(8 * br + 8, A.m)]])
+            b0, b1 = [int(v) for v in h["blk_rowptr"][br:br + 2].cpu()]
+            assert b1 - b0 == B.Bnnz
+            assert np.array_equal(h["blk_col"][b0:b1].cpu().numpy(), B.blk_col)
+            assert np.array_equal(h["bitmap"][b0:b1].cpu().numpy().view(np.uint64), B.bitmap)
+            off = h["blk_offset"][b0:b1 + 1].cpu().numpy().astype(np.int64)
+            assert np.array_equal(off - off[0], B.blk_offset)
+            assert off[0] == A.rowptr[8 * br]
+        M.free()
