@@ -125,7 +125,7 @@ class _CudaArray:
     """__cuda_array_interface__ shim to view a library-owned device array."""
 
     def __init__(self, ptr: int, shape, typestr: str, owner):
-        self.__cuda_array_interface__ = {"data": (ptr or 0, True), "shape": tuple(shape),
+        self.__cuda_array_interface__ = {"data": (ptr or 0, False), "shape": tuple(shape),
                                          "typestr": typestr, "version": 3, "strides": None}
         self._owner = owner
 

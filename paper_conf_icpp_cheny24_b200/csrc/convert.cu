@@ -402,7 +402,8 @@ spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *ro
     k_finalize<<<grid_for(Bnrow + 1, 256), 256, 0, st>>>(Bnrow, Bnnz, nnz, chunk_start, cnt_blk,
                                                          A->blk_rowptr, A->blk_offset);
     SPADEN_CUDA_TRY(cudaGetLastError());
-    return SPADEN_OK;
+    // SpMV tile schedule (second and last host sync: tile / long-row counts)
+    return build_schedule(A, st);
 }
 
 }  // namespace spaden

@@ -9,6 +9,11 @@
 
 #include "spaden.h"
 
+// One SpMV tile: block-rows [br0, br1), their blocks [b0, b1), values [v0, v1).
+struct alignas(32) spaden_tile_desc_s {
+    int32_t br0, br1, b0, b1, v0, v1, pad0, pad1;
+};
+
 // ------------------------------------------------------------------ handle
 struct spaden_matrix_s {
     int64_t m = 0, n = 0, nnz = 0;
@@ -23,9 +28,13 @@ struct spaden_matrix_s {
     int32_t *blk_offset = nullptr;   // [Bnnz+1]
     void *values = nullptr;          // [nnz]
 
-    // SpMV schedule (aux)
+    // SpMV schedule (aux, schedule.cu)
     int64_t aux_bytes = 0;
-    int64_t n_tiles = 0;
+    int64_t n_tiles = 0;                       // whole-block-row tiles
+    int64_t n_long = 0;                        // block-rows too large for a tile
+    int tile_cfg = 0;                          // spaden::tile_cfg index the schedule was built for
+    struct spaden_tile_desc_s *tiles = nullptr; // [n_tiles] (spaden::TileDesc)
+    int32_t *long_rows = nullptr;              // [n_long]
 
     // host-API staging buffers (lazily allocated)
     float *stage_x = nullptr;
@@ -33,6 +42,8 @@ struct spaden_matrix_s {
 };
 
 namespace spaden {
+
+using Matrix = ::spaden_matrix_s;
 
 // ---------------------------------------------------------------- errors
 void set_error(const std::string &msg);
@@ -52,15 +63,36 @@ enum : uint32_t {
 };
 
 // ------------------------------------------------------------ SpMV schedule
-// A tile is a run of whole block-rows [br_begin, br_end) processed by one warp
-// group, or (long block-rows) one chunk [b_begin, b_end) of a single block-row
-// whose partial row sums go to a carry slot and are combined by a fix-up pass.
-struct Tile {
-    int32_t br_begin;
-    int32_t br_end;
+// Launch shape of the tiled SpMV kernel: CTAs per SM, consumer warps per CTA,
+// pipeline stages and bytes per stage.  A tile (whole block-rows) must fit one
+// stage including the 16-byte alignment slack of its regions.
+struct TileCfg {
+    int ctas_per_sm, consumers, stages, stage_bytes;
 };
+constexpr int kMaxStages = 4;
+constexpr int kNumTileCfgs = 4;
+__host__ __device__ inline TileCfg tile_cfg(int i) {
+    switch (i) {
+    case 1: return TileCfg{2, 16, 3, 36 * 1024};
+    case 2: return TileCfg{3, 8, 3, 24 * 1024};
+    case 3: return TileCfg{4, 8, 2, 27 * 1024};
+    default: return TileCfg{1, 16, 3, 64 * 1024};
+    }
+}
+int default_tile_cfg();  // SPADEN_TILE_CFG env override, else the measured best
+constexpr int kStageSlack = 384;
+// shared-memory bytes a block occupies in a stage: bitmap 8 + blk_col 4 +
+// blk_offset 4 (copied) + 8 fp32 row partials at a 9-word stride (scratch)
+constexpr int kBlockStageBytes = 16 + 36;
+// mean nonzeros per block from which the predicated-slot decode is used
+constexpr int kSlotsMinFill = 8;
+// decode used above that fill (1 = lane per block, 2 = lane per block row)
+constexpr int kDenseDecode = 1;
 
-using Matrix = ::spaden_matrix_s;
+using TileDesc = ::spaden_tile_desc_s;
+
+spaden_status_t build_schedule(Matrix *A, cudaStream_t stream);
+
 
 // converter (convert.cu)
 spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *rowptr,

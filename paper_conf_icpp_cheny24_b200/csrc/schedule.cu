@@ -1,0 +1,147 @@
+// schedule.cu -- SpMV work schedule, built once at conversion time.
+//
+// The v1 SpMV kernel streams the bitBSR arrays through shared memory in
+// "tiles": runs of WHOLE block-rows [br0, br1) whose blocks, values and
+// blk_rowptr slice fit one pipeline stage (TileCfg::stage_bytes).  Keeping block-rows
+// whole keeps each row's summation order a function of that block-row alone
+// (deterministic and independent of how rows are partitioned across GPUs).
+// A block-row too large for half a stage is "long": it is listed separately
+// and processed straight from global memory by the long-row kernel with the
+// same lane mapping and summation order.
+//
+// Tiles are packed greedily inside segments of kSeg block-rows (one thread per
+// segment; two passes: count, then write after a scan of the counts).
+#include <cstdlib>
+
+#include "internal.cuh"
+
+namespace spaden {
+namespace {
+
+constexpr int kSeg = 256;
+
+__device__ __forceinline__ int64_t br_cost(const int32_t *brp, const int32_t *boff, int64_t br, int sv,
+                                           int32_t *nb_out, int32_t *nv_out) {
+    const int b0 = brp[br], b1 = brp[br + 1];
+    const int nv = boff[b1] - boff[b0];
+    *nb_out = b1 - b0;
+    *nv_out = nv;
+    return (int64_t)kBlockStageBytes * (b1 - b0) + (int64_t)sv * nv + 4;
+}
+
+template <bool WRITE>
+__global__ void k_pack(int64_t Bnrow, const int32_t *__restrict__ brp, const int32_t *__restrict__ boff,
+                       int sv, int64_t cap, int64_t long_cost, int32_t *__restrict__ seg_tiles,
+                       int32_t *__restrict__ seg_long, const int32_t *__restrict__ tile_start,
+                       const int32_t *__restrict__ long_start, TileDesc *__restrict__ tiles,
+                       int32_t *__restrict__ long_rows) {
+    const int64_t seg = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t nseg = (Bnrow + kSeg - 1) / kSeg;
+    if (seg >= nseg) return;
+    const int64_t s0 = seg * kSeg, s1 = min(Bnrow, s0 + kSeg);
+    int nt = 0, nl = 0;
+    int64_t open_br = -1, open_cost = 0;
+    int32_t tbase = WRITE ? tile_start[seg] : 0;
+    int32_t lbase = WRITE ? long_start[seg] : 0;
+    auto close = [&](int64_t br_end) {
+        if (open_br >= 0) {
+            if (WRITE) {
+                TileDesc d;
+                d.br0 = (int32_t)open_br;
+                d.br1 = (int32_t)br_end;
+                d.b0 = brp[open_br];
+                d.b1 = brp[br_end];
+                d.v0 = boff[d.b0];
+                d.v1 = boff[d.b1];
+                d.pad0 = d.pad1 = 0;
+                tiles[tbase + nt] = d;
+            }
+            ++nt;
+            open_br = -1;
+            open_cost = 0;
+        }
+    };
+    for (int64_t br = s0; br < s1; ++br) {
+        int32_t nb, nv;
+        const int64_t c = br_cost(brp, boff, br, sv, &nb, &nv);
+        if (c > long_cost) {
+            close(br);
+            if (WRITE) long_rows[lbase + nl] = (int32_t)br;
+            ++nl;
+            continue;
+        }
+        if (open_br >= 0 && open_cost + c > cap) close(br);
+        if (open_br < 0) open_br = br;
+        open_cost += c;
+    }
+    close(s1);
+    if (!WRITE) {
+        seg_tiles[seg] = nt;
+        seg_long[seg] = nl;
+    }
+}
+
+__global__ void k_sched_summary(const int32_t *tile_total, const int32_t *long_total, int32_t *out) {
+    out[0] = *tile_total;
+    out[1] = *long_total;
+}
+
+}  // namespace
+
+int default_tile_cfg() {
+    const char *e = getenv("SPADEN_TILE_CFG");
+    if (e && e[0] >= '0' && e[0] < '0' + kNumTileCfgs) return e[0] - '0';
+    return 3;  // measured best on fem1p5m: 4 CTAs/SM x 8 consumers x 2 x 27 KB
+}
+
+spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
+    const int64_t Bnrow = A->Bnrow;
+    const int sv = A->storage == SPADEN_R_16F ? 2 : 4;
+    const int64_t nseg = (Bnrow + kSeg - 1) / kSeg;
+    A->tile_cfg = default_tile_cfg();
+    const TileCfg cfg = tile_cfg(A->tile_cfg);
+    const int64_t cap = cfg.stage_bytes - kStageSlack;
+    const int64_t long_cost = cfg.stage_bytes / 2;
+    if (Bnrow == 0) return SPADEN_OK;
+
+    const size_t n_tmp = scan_tmp_ints(nseg + 1);
+    const size_t ints = 2 * (size_t)(nseg + 1) + n_tmp + 4;
+    int32_t *tmp = nullptr;
+    SPADEN_CUDA_TRY(cudaMallocAsync(&tmp, ints * sizeof(int32_t), st));
+    int32_t *seg_tiles = tmp, *seg_long = tmp + (nseg + 1), *scan_tmp = tmp + 2 * (nseg + 1);
+    int32_t *summary = scan_tmp + n_tmp;
+    const unsigned grid = (unsigned)((nseg + 127) / 128);
+    k_pack<false><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, seg_tiles,
+                                        seg_long, nullptr, nullptr, nullptr, nullptr);
+    cudaError_t e = exclusive_scan_i32(seg_tiles, seg_tiles, nseg, scan_tmp, st);
+    if (e == cudaSuccess) e = exclusive_scan_i32(seg_long, seg_long, nseg, scan_tmp, st);
+    int32_t h[2] = {0, 0};
+    if (e == cudaSuccess) {
+        k_sched_summary<<<1, 1, 0, st>>>(seg_tiles + nseg, seg_long + nseg, summary);
+        e = cudaMemcpyAsync(h, summary, sizeof(h), cudaMemcpyDeviceToHost, st);
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) {
+        cudaFreeAsync(tmp, st);
+        return cuda_status(e, "building SpMV schedule");
+    }
+    A->n_tiles = h[0];
+    A->n_long = h[1];
+    const size_t tile_bytes = sizeof(TileDesc) * (size_t)std::max<int64_t>(1, A->n_tiles + 1);
+    const size_t long_bytes = sizeof(int32_t) * (size_t)std::max<int64_t>(1, A->n_long);
+    e = cudaMalloc(&A->tiles, tile_bytes);
+    if (e == cudaSuccess) e = cudaMalloc(&A->long_rows, long_bytes);
+    if (e != cudaSuccess) {
+        cudaFreeAsync(tmp, st);
+        return cuda_status(e, "allocating SpMV schedule");
+    }
+    A->aux_bytes = (int64_t)(tile_bytes + long_bytes);
+    k_pack<true><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, nullptr,
+                                       nullptr, seg_tiles, seg_long, A->tiles, A->long_rows);
+    e = cudaGetLastError();
+    cudaFreeAsync(tmp, st);
+    if (e != cudaSuccess) return cuda_status(e, "packing SpMV schedule");
+    return SPADEN_OK;
+}
+
+}  // namespace spaden

@@ -1,18 +1,23 @@
 // spmv.cu -- y = alpha*A*x + beta*y over bitBSR on sm_100a CUDA cores
 // (§4.3).
 //
-// v0 mapping ("row-byte lanes"): one warp per block-row ("each row of
-// blocks ... is computed with a segment of x with length 8, producing a segment
-// of y with length 8").  The warp walks the block-row four blocks at a time; the
-// 8 lanes of group g = lane/8 take block b0+g+4i and lane r = lane%8 owns row r of
-// that block, i.e. byte r of the bitmap.  Its first value sits at
-// blk_offset[b] + popc(bitmap & ((1<<8r)-1)) (popcount rank, reading R1 of
-// Alg. 2); the 8 bit slots are unrolled and predicated on the byte,
-// so structural zeros are neither loaded nor multiplied (reading R11).
-// x[8*bc .. 8*bc+7] is one 32-byte sector read as two float4 broadcasts
-// (Alg. 2 lines 7-10).  Each lane accumulates its row over the
-// block-row in fp32; the four groups are combined with two xor-shuffles in a
-// fixed order, so the result depends only on the block-row's own blocks.
+// Two kernels:
+//   k_spmv_tiled  (default)  persistent CTAs fed by a TMA bulk-copy pipeline;
+//   k_spmv_v0     (SPADEN_KERNEL=v0) the first, simple row-byte kernel, kept as
+//                 the measured baseline of DESIGN.md.
+// and k_spmv_long for block-rows too large for a pipeline stage.
+//
+// Decode (both kernels follow PAPER.md §4.3.1 / Alg. 2 semantics):
+// bit 8r+c of a block's bitmap is entry (r, c); its value is the
+// next one in the block's packed run because values are stored in ascending
+// bit order ("stored consecutively") -- i.e. the value index of a set
+// bit is blk_offset + popcount of the lower bits (reading R1 of Alg. 2 lines
+// 5-6).  Only set bits load a value or touch x ("zero elements are calculated
+// instead of loading from memory"): structural zeros are never
+// multiplied (reading R11).  x[8bc .. 8bc+7] is the block's 8-element segment
+// (Alg. 2 lines 7-10).
+#include <cstdlib>
+
 #include "internal.cuh"
 
 namespace spaden {
@@ -26,6 +31,10 @@ template <> __device__ __forceinline__ float ldv<__half>(const __half *p) {
     return __half2float(__ldg(p));
 }
 
+// ==========================================================================
+// v0: one warp per block-row; 8 lanes per block (lane r = row r = bitmap byte
+// r), four blocks per warp step; 8 predicated bit slots per lane.
+// ==========================================================================
 template <typename V>
 __global__ void __launch_bounds__(256)
 k_spmv_v0(int64_t m, int64_t n, int64_t Bnrow, const int32_t *__restrict__ blk_rowptr,
@@ -75,22 +84,543 @@ k_spmv_v0(int64_t m, int64_t n, int64_t Bnrow, const int32_t *__restrict__ blk_r
     }
 }
 
+// ==========================================================================
+// Tiled kernel: persistent CTAs, TMA bulk-copy pipeline through shared memory.
+//
+// Warp 0 (one elected lane) is the producer; warps 1..CONSUMERS consume.
+// Tiles (schedule.cu: runs of whole block-rows) go round-robin to CTAs,
+// tile t -> CTA t % gridDim.x.  Per tile the producer waits for the ring slot
+// (mbarrier "empty"), writes a header, and issues cp.async.bulk copies of the
+// bitmap, blk_col, blk_offset, blk_rowptr and value slices (16-byte-aligned
+// supersets) completing on the slot's "full" mbarrier (complete_tx), with an
+// L2 evict-first policy (the matrix is streamed once; x stays resident).
+//
+// Phase 1 (decode): the tile's blocks are cut into units of 32 consecutive
+// blocks, grabbed dynamically by the consumer warps (shared counter).  One
+// lane per block: it walks the 64 bit slots in ascending bit order (predicated,
+// or a set-bit loop for low-fill matrices -- same arithmetic) and writes the
+// block's 8 row partials to a scratch area of the stage.
+// Phase 2 (reduce): the warp whose completion count finishes the tile sums, for each
+// block-row and row, the block partials in a fixed order (4 interleaved chains
+// by block index within the block-row, then (c0+c1)+(c2+c3)) and stores y.
+// The summation order depends only on the block-row, so any 8-row-aligned row
+// partition of A produces bitwise identical y.
+// ==========================================================================
+
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint32_t bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(ok)
+        : "r"(bar), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+    while (!mbar_try_wait(bar, parity)) {
+    }
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar,
+                                         uint64_t policy) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], "
+        "%4;" ::"r"(dst),
+        "l"(src), "r"(bytes), "r"(bar), "l"(policy)
+        : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint2 lds_u2(uint32_t a) {
+    uint2 v;
+    asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ int lds_i32(uint32_t a) {
+    int v;
+    asm("ld.shared.s32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ float lds_f32(uint32_t a) {
+    float v;
+    asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ float lds_f16(uint32_t a) {
+    unsigned short h;
+    asm("ld.shared.u16 %0, [%1];" : "=h"(h) : "r"(a));
+    return __half2float(__ushort_as_half(h));
+}
+// header loads must stay below the full-barrier wait: volatile + memory clobber
+__device__ __forceinline__ int4 lds_i4_volatile(uint32_t a) {
+    int4 v;
+    asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ int atom_add_shared(uint32_t a, int v) {
+    int old;
+    asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(a), "r"(v) : "memory");
+    return old;
+}
+__device__ __forceinline__ void sts_f32(uint32_t a, float v) {
+    asm volatile("st.shared.f32 [%0], %1;" ::"r"(a), "f"(v) : "memory");
+}
+// row partials of a block: 8 floats at a 9-word stride (bank-conflict-free
+// per-lane stores and phase-2 reads)
+constexpr uint32_t kPartStride = 36;
+
+// Value source of a block's packed run: shared-memory stage or global memory.
+template <typename V> struct SmemVals {
+    using P = uint32_t;  // shared byte address
+    static __device__ __forceinline__ float get(P p) {
+        if constexpr (sizeof(V) == 2) return lds_f16(p);
+        else return lds_f32(p);
+    }
+    static constexpr uint32_t step = sizeof(V);
+};
+template <typename V> struct GlobalVals {
+    using P = const V *;
+    static __device__ __forceinline__ float get(P p) { return ldv<V>(p); }
+    static constexpr int step = 1;
+};
+
+struct XSeg {
+    float v[8];
+};
+
+// nbc_vec = number of leading block columns whose x segment may be read as one
+// 32-byte vector (n/8 when x is 32-byte aligned, else 0); other segments read only the
+// columns referenced by `cols` (bit c set = column c used by the block).
+__device__ __forceinline__ void load_x(XSeg &xs, const float *__restrict__ x, int bc, int nbc_vec, uint32_t cols) {
+    const float *p = x + 8 * (int64_t)bc;
+    if (bc < nbc_vec) {  // one 32-byte sector, one 256-bit load (LDG.E.ENL2.256)
+        asm("ld.global.nc.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+            : "=f"(xs.v[0]), "=f"(xs.v[1]), "=f"(xs.v[2]), "=f"(xs.v[3]), "=f"(xs.v[4]), "=f"(xs.v[5]),
+              "=f"(xs.v[6]), "=f"(xs.v[7])
+            : "l"(p));
+    } else {
+#pragma unroll
+        for (int c = 0; c < 8; ++c) xs.v[c] = ((cols >> c) & 1u) ? __ldg(p + c) : 0.f;
+    }
+}
+
+__device__ __forceinline__ uint32_t used_cols(uint2 bm) {
+    uint32_t w = bm.x | bm.y;
+    w |= w >> 16;
+    w |= w >> 8;
+    return w & 0xffu;
+}
+
+// Row partials of one block, 64 predicated slots in ascending bit order.  Each
+// row starts at its own popcount rank (P:L138 exclusive counts), so the eight
+// rows are independent dependency chains of at most 8 slots.
+template <class VS>
+__device__ __forceinline__ void block_slots(uint2 bm, typename VS::P p0, const XSeg &xs, float acc[8]) {
+    const int plo = __popc(bm.x);
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+        const uint32_t w = r < 4 ? bm.x : bm.y;
+        const uint32_t byte = (w >> (8 * (r & 3))) & 0xffu;
+        const int below = ((r & 3) == 0 ? 0 : __popc(w & ((1u << (8 * (r & 3))) - 1u))) + (r < 4 ? 0 : plo);
+        typename VS::P p = p0 + below * VS::step;
+        float a = 0.f;
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+            if ((byte >> c) & 1u) {
+                a = fmaf(VS::get(p), xs.v[c], a);
+                p += VS::step;
+            }
+        }
+        acc[r] = a;
+    }
+}
+
+// The same partials by iterating the set bits (fewer instructions when the
+// block holds few nonzeros); identical fma sequence per row.
+template <class VS>
+__device__ __forceinline__ void block_bits(uint2 bm, typename VS::P p, const float *__restrict__ xseg,
+                                           float acc[8]) {
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+        uint32_t byte = ((r < 4 ? bm.x : bm.y) >> (8 * (r & 3))) & 0xffu;
+        float a = 0.f;
+        while (byte) {
+            const int c = __ffs(byte) - 1;
+            byte &= byte - 1;
+            a = fmaf(VS::get(p), __ldg(xseg + c), a);
+            p += VS::step;
+        }
+        acc[r] = a;
+    }
+}
+
+struct alignas(16) StageHdr {
+    int br0, nbr, b0, v0;                      // tile
+    int nb, units, u_next, done;               // blocks, 32-block units, next unit to grab, units done
+    uint32_t a_bmp, a_col, a_off, a_rp;        // shared addresses of the copied slices
+    uint32_t a_val, a_part, pad0, pad1;        // values, row-partial scratch
+};
+
+// DEC: 0 = set-bit loop, 1 = 64 predicated slots per lane (lane = block),
+//      2 = 8 predicated slots per lane (lane = one row of a block, 4 blocks per
+//          warp step: value loads of a step stay inside 4 consecutive runs).
+template <typename V, int DEC, int CONSUMERS, int MINB>
+__global__ void __launch_bounds__(32 * (CONSUMERS + 1), MINB)
+k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int ntiles, const int32_t *__restrict__ blk_rowptr,
+             const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
+             const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
+             int nbc_vec, float alpha, float beta, float *__restrict__ y) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t full_bar[kMaxStages], empty_bar[kMaxStages];
+    __shared__ StageHdr hdr[kMaxStages];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < stages; ++s) {
+            mbar_init(smem_u32(&full_bar[s]), 1);
+            mbar_init(smem_u32(&empty_bar[s]), CONSUMERS);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const uint32_t sbase = smem_u32(smem);
+
+    if (warp == 0) {  // ---------------------------------------------- producer
+        if (lane == 0) {
+            const uint64_t pol = policy_evict_first();
+            int i = 0;
+            for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+                const int s = i % stages;
+                const uint32_t ph = (uint32_t)(i / stages) & 1u;
+                const int4 d0 = __ldg(reinterpret_cast<const int4 *>(tiles + t));
+                const int4 d1 = __ldg(reinterpret_cast<const int4 *>(tiles + t) + 1);
+                const int br0 = d0.x, br1 = d0.y, b0 = d0.z, b1 = d0.w, v0 = d1.x, v1 = d1.y;
+                if (i >= stages) mbar_wait(smem_u32(&empty_bar[s]), ph ^ 1u);
+                const uint32_t stage = sbase + (uint32_t)s * (uint32_t)stage_bytes;
+                uint32_t cur = stage;
+                struct Reg {
+                    uintptr_t src;
+                    uint32_t sz;
+                };
+                auto region = [&](const void *lo_p, size_t len, uint32_t *addr_out) {
+                    const uintptr_t lo = (uintptr_t)lo_p, hi = lo + len;
+                    const uintptr_t alo = lo & ~(uintptr_t)15, ahi = (hi + 15) & ~(uintptr_t)15;
+                    *addr_out = cur + (uint32_t)(lo - alo);
+                    const Reg r{alo, len > 0 ? (uint32_t)(ahi - alo) : 0u};
+                    cur += r.sz;
+                    return r;
+                };
+                StageHdr h;
+                h.br0 = br0;
+                h.nbr = br1 - br0;
+                h.b0 = b0;
+                h.v0 = v0;
+                h.nb = b1 - b0;
+                h.units = max(1, (h.nb + 31) >> 5);
+                h.u_next = 0;
+                h.done = 0;
+                h.pad0 = h.pad1 = 0;
+                const Reg rs[5] = {region(bitmap + b0, 8u * (b1 - b0), &h.a_bmp),
+                                   region(blk_col + b0, 4u * (b1 - b0), &h.a_col),
+                                   region(blk_offset + b0, 4u * (b1 - b0), &h.a_off),
+                                   region(blk_rowptr + br0, 4u * (br1 - br0 + 1), &h.a_rp),
+                                   region(vals + v0, sizeof(V) * (size_t)(v1 - v0), &h.a_val)};
+                const uint32_t bytes = cur - stage;
+                h.a_part = cur;  // kPartStride bytes of row partials per block (not copied)
+                hdr[s] = h;
+                const uint32_t fb = smem_u32(&full_bar[s]);
+                mbar_arrive_expect_tx(fb, bytes);
+                uint32_t dst = stage;
+#pragma unroll
+                for (int k = 0; k < 5; ++k) {
+                    if (rs[k].sz) bulk_g2s(dst, (const void *)rs[k].src, rs[k].sz, fb, pol);
+                    dst += rs[k].sz;
+                }
+            }
+        }
+        return;
+    }
+
+    // ------------------------------------------------------------ consumers
+    int i = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+        const int s = i % stages;
+        const uint32_t ph = (uint32_t)(i / stages) & 1u;
+        mbar_wait(smem_u32(&full_bar[s]), ph);
+        const int4 h0 = lds_i4_volatile(smem_u32(&hdr[s].br0));
+        const int4 h1 = lds_i4_volatile(smem_u32(&hdr[s].nb));
+        const int4 h2 = lds_i4_volatile(smem_u32(&hdr[s].a_bmp));
+        const int4 h3 = lds_i4_volatile(smem_u32(&hdr[s].a_val));
+        const int v0 = h0.w, nb = h1.x, units = h1.y;
+        const uint32_t a_bmp = h2.x, a_col = h2.y, a_off = h2.z, a_val = h3.x, a_part = h3.y;
+        // units of 32 blocks are grabbed dynamically (shared counter per stage)
+        const uint32_t a_next = smem_u32(&hdr[s].u_next);
+        int mine = 0;
+        while (true) {
+            int ul = 0;
+            if (lane == 0) ul = atom_add_shared(a_next, 1);
+            ul = __shfl_sync(kFull, ul, 0);
+            if (ul >= units) break;
+            ++mine;
+            if constexpr (DEC == 2) {
+                const int g = lane >> 3, r = lane & 7;
+                const uint32_t mlo = r == 0 ? 0u : (r < 4 ? (1u << (8 * r)) - 1u : 0xffffffffu);
+                const uint32_t mhi = r <= 4 ? 0u : (1u << (8 * (r - 4))) - 1u;
+                const int sh = 8 * (r & 3);
+#pragma unroll 2
+                for (int st = 0; st < 8; ++st) {
+                    const int lb = ul * 32 + st * 4 + g;
+                    if (lb < nb) {
+                        const uint2 bm = lds_u2(a_bmp + 8u * lb);
+                        const int bc = lds_i32(a_col + 4u * lb);
+                        const uint32_t byte = ((r < 4 ? bm.x : bm.y) >> sh) & 0xffu;
+                        uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0 + __popc(bm.x & mlo) +
+                                                        __popc(bm.y & mhi)) *
+                                                 (uint32_t)sizeof(V);
+                        XSeg xs;
+                        load_x(xs, x, bc, nbc_vec, used_cols(bm));
+                        float a = 0.f;
+#pragma unroll
+                        for (int c = 0; c < 8; ++c) {
+                            if ((byte >> c) & 1u) {
+                                a = fmaf(SmemVals<V>::get(p), xs.v[c], a);
+                                p += SmemVals<V>::step;
+                            }
+                        }
+                        sts_f32(a_part + kPartStride * lb + 4u * r, a);
+                    }
+                }
+            } else {
+                const int lb = ul * 32 + lane;
+                if (lb < nb) {  // phase 1: one block per lane
+                    const uint2 bm = lds_u2(a_bmp + 8u * lb);
+                    const int bc = lds_i32(a_col + 4u * lb);
+                    const uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
+                    float acc[8];
+                    if constexpr (DEC == 1) {
+                        XSeg xs;
+                        load_x(xs, x, bc, nbc_vec, used_cols(bm));
+                        block_slots<SmemVals<V>>(bm, p, xs, acc);
+                    } else {
+                        block_bits<SmemVals<V>>(bm, p, x + 8 * (int64_t)bc, acc);
+                    }
+                    const uint32_t q = a_part + kPartStride * lb;
+#pragma unroll
+                    for (int r = 0; r < 8; ++r) sts_f32(q + 4u * r, acc[r]);
+                }
+            }
+        }
+        if (mine) {
+            __syncwarp();
+            int last = 0;
+            if (lane == 0) {
+                __threadfence_block();
+                last = (atom_add_shared(smem_u32(&hdr[s].done), mine) + mine == units);
+            }
+            if (__shfl_sync(kFull, last, 0)) {  // phase 2: this warp completed the tile
+                __threadfence_block();
+                const int br0 = h0.x, nbr = h0.y, b0 = h0.z;
+                const uint32_t a_rp = h2.w;
+                const int r = lane & 7;
+                for (int base = 0; base < nbr; base += 4) {
+                    const int brl = base + (lane >> 3);
+                    if (brl < nbr) {
+                        const int k0 = lds_i32(a_rp + 4u * brl) - b0;
+                        const int k1 = lds_i32(a_rp + 4u * (brl + 1)) - b0;
+                        float c0 = 0.f, c1 = 0.f, c2 = 0.f, c3 = 0.f;
+                        uint32_t q = a_part + kPartStride * k0 + 4u * r;
+                        int k = k0;
+                        for (; k + 3 < k1; k += 4, q += 4 * kPartStride) {
+                            c0 += lds_f32(q);
+                            c1 += lds_f32(q + kPartStride);
+                            c2 += lds_f32(q + 2 * kPartStride);
+                            c3 += lds_f32(q + 3 * kPartStride);
+                        }
+                        if (k < k1) c0 += lds_f32(q);
+                        if (k + 1 < k1) c1 += lds_f32(q + kPartStride);
+                        if (k + 2 < k1) c2 += lds_f32(q + 2 * kPartStride);
+                        const float sum = (c0 + c1) + (c2 + c3);
+                        const int64_t row = 8 * ((int64_t)br0 + brl) + r;
+                        if (row < m) {
+                            float o = alpha * sum;
+                            if (beta != 0.f) o = fmaf(beta, y[row], o);
+                            y[row] = o;
+                        }
+                    }
+                }
+            }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(smem_u32(&empty_bar[s]));
+    }
+}
+
+// Long block-rows (too large for a stage): one warp per block-row straight from
+// global memory; lane j takes blocks j, j+32, ... (one lane per block, same
+// per-block arithmetic as the tiled kernel), then a fixed xor tree over lanes.
+template <typename V, bool SLOTS>
+__global__ void __launch_bounds__(256)
+k_spmv_long(int64_t m, const int32_t *__restrict__ long_rows, int nlong, const int32_t *__restrict__ blk_rowptr,
+            const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
+            const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
+            int nbc_vec, float alpha, float beta, float *__restrict__ y) {
+    const int w = (int)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    const int lane = threadIdx.x & 31;
+    if (w >= nlong) return;
+    const int br = long_rows[w];
+    const int b0 = blk_rowptr[br], b1 = blk_rowptr[br + 1];
+    float tot[8];
+#pragma unroll
+    for (int r = 0; r < 8; ++r) tot[r] = 0.f;
+    for (int b = b0 + lane; b < b1; b += 32) {
+        const uint64_t w64 = __ldg(bitmap + b);
+        const uint2 bm = make_uint2((uint32_t)w64, (uint32_t)(w64 >> 32));
+        const int bc = __ldg(blk_col + b);
+        const V *p = vals + __ldg(blk_offset + b);
+        float acc[8];
+        if constexpr (SLOTS) {
+            XSeg xs;
+            load_x(xs, x, bc, nbc_vec, used_cols(bm));
+            block_slots<GlobalVals<V>>(bm, p, xs, acc);
+        } else {
+            block_bits<GlobalVals<V>>(bm, p, x + 8 * (int64_t)bc, acc);
+        }
+#pragma unroll
+        for (int r = 0; r < 8; ++r) tot[r] += acc[r];
+    }
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) tot[r] += __shfl_xor_sync(kFull, tot[r], o);
+    }
+    if (lane < 8) {
+        const int64_t row = 8 * (int64_t)br + lane;
+        float sum = tot[0];
+#pragma unroll
+        for (int r = 1; r < 8; ++r)
+            if (lane == r) sum = tot[r];
+        if (row < m) {
+            float o = alpha * sum;
+            if (beta != 0.f) o = fmaf(beta, y[row], o);
+            y[row] = o;
+        }
+    }
+}
+
+int kernel_variant() {
+    static int v = [] {
+        const char *e = getenv("SPADEN_KERNEL");
+        if (e && e[0] == 'v' && e[1] == '0') return 0;
+        return 1;
+    }();
+    return v;
+}
+
+int sm_count() {
+    static int c = [] {
+        int dev = 0, n = 148;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        return n;
+    }();
+    return c;
+}
+
+template <typename V, int DEC, int CONSUMERS, int MINB>
+cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, const float *x, float beta,
+                             float *y, cudaStream_t st) {
+    const int nbc_vec = ((uintptr_t)x & 31u) == 0 ? (int)(A.n / 8) : 0;
+    const size_t smem = (size_t)cfg.stages * cfg.stage_bytes;
+    static int occ = 0;  // resident CTAs per SM actually achievable (registers, smem)
+    if (occ == 0) {
+        auto kern = k_spmv_tiled<V, DEC, CONSUMERS, MINB>;
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e == cudaSuccess)
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * (CONSUMERS + 1), smem);
+        if (e != cudaSuccess) return e;
+        occ = std::max(1, std::min(occ, MINB));
+    }
+    if (A.n_tiles > 0) {
+        const int grid = (int)std::min<int64_t>(A.n_tiles, (int64_t)sm_count() * occ);
+        k_spmv_tiled<V, DEC, CONSUMERS, MINB><<<grid, 32 * (CONSUMERS + 1), smem, st>>>(
+            cfg.stages, cfg.stage_bytes, A.m, A.tiles, (int)A.n_tiles, A.blk_rowptr, A.blk_col, A.bitmap,
+            A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y);
+    }
+    if (A.n_long > 0) {
+        const int64_t threads = 32 * A.n_long;
+        k_spmv_long<V, (DEC != 0)><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+            A.m, A.long_rows, (int)A.n_long, A.blk_rowptr, A.blk_col, A.bitmap, A.blk_offset, (const V *)A.values,
+            x, nbc_vec, alpha, beta, y);
+    }
+    return cudaGetLastError();
+}
+
+template <typename V, int DEC>
+cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st) {
+    const TileCfg cfg = tile_cfg(A.tile_cfg);
+    switch (A.tile_cfg) {
+    case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st);
+    case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st);
+    case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
+    default: return launch_tiled_cfg<V, DEC, 16, 1>(A, cfg, alpha, x, beta, y, st);
+    }
+}
+
 }  // namespace
 
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,
                             cudaStream_t st) {
     if (A.m == 0) return SPADEN_OK;
-    const int threads = 256;
-    const int64_t want = (A.Bnrow + 7) / 8;
-    const unsigned grid = (unsigned)std::min<int64_t>(want, 148LL * 64);
     const bool x_vec = ((uintptr_t)x & 15u) == 0;
+    if (kernel_variant() == 0) {
+        const int threads = 256;
+        const int64_t want = (A.Bnrow + 7) / 8;
+        const unsigned grid = (unsigned)std::min<int64_t>(want, 148LL * 64);
+        if (A.storage == SPADEN_R_16F)
+            k_spmv_v0<__half><<<grid, threads, 0, st>>>(A.m, A.n, A.Bnrow, A.blk_rowptr, A.blk_col, A.bitmap,
+                                                       A.blk_offset, (const __half *)A.values, x, x_vec, alpha,
+                                                       beta, y);
+        else
+            k_spmv_v0<float><<<grid, threads, 0, st>>>(A.m, A.n, A.Bnrow, A.blk_rowptr, A.blk_col, A.bitmap,
+                                                      A.blk_offset, (const float *)A.values, x, x_vec, alpha,
+                                                      beta, y);
+        SPADEN_CUDA_TRY(cudaGetLastError());
+        return SPADEN_OK;
+    }
+    // decode style from the mean block fill (predicated slots for dense-ish blocks)
+    static const int decode_env = [] {  // SPADEN_DECODE=bits|slots|rows overrides (ablation)
+        const char *e = getenv("SPADEN_DECODE");
+        if (e && e[0] == 'b') return 0;
+        if (e && e[0] == 's') return 1;
+        if (e && e[0] == 'r') return 2;
+        return -1;
+    }();
+    const int dec = decode_env >= 0 ? decode_env
+                                    : ((A.Bnnz == 0 || A.nnz >= (int64_t)kSlotsMinFill * A.Bnnz) ? kDenseDecode : 0);
+    cudaError_t e;
     if (A.storage == SPADEN_R_16F)
-        k_spmv_v0<__half><<<grid, threads, 0, st>>>(A.m, A.n, A.Bnrow, A.blk_rowptr, A.blk_col, A.bitmap,
-                                                   A.blk_offset, (const __half *)A.values, x, x_vec, alpha, beta, y);
+        e = dec == 0 ? launch_tiled<__half, 0>(A, alpha, x, beta, y, st)
+                     : (dec == 1 ? launch_tiled<__half, 1>(A, alpha, x, beta, y, st)
+                                 : launch_tiled<__half, 2>(A, alpha, x, beta, y, st));
     else
-        k_spmv_v0<float><<<grid, threads, 0, st>>>(A.m, A.n, A.Bnrow, A.blk_rowptr, A.blk_col, A.bitmap,
-                                                  A.blk_offset, (const float *)A.values, x, x_vec, alpha, beta, y);
-    SPADEN_CUDA_TRY(cudaGetLastError());
+        e = dec == 0 ? launch_tiled<float, 0>(A, alpha, x, beta, y, st)
+                     : (dec == 1 ? launch_tiled<float, 1>(A, alpha, x, beta, y, st)
+                                 : launch_tiled<float, 2>(A, alpha, x, beta, y, st));
+    if (e != cudaSuccess) return cuda_status(e, "launching k_spmv_tiled");
     return SPADEN_OK;
 }
 
