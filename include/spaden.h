@@ -118,8 +118,10 @@ SPADEN_API spaden_status_t spaden_convert_csr_to_bitmap(int64_t m, int64_t n, in
  * spaden_spmv -- y = alpha * A x + beta * y on the GPU (§4.3: "takes bitBSR
  * and a dense vector x as input and produces a dense vector y").
  *
- *   A         handle from spaden_convert_csr_to_bitmap (immutable; may be used by
- *             several streams concurrently).
+ *   A         handle from spaden_convert_csr_to_bitmap.  The bitBSR arrays are
+ *             immutable, but block-rows too large for a pipeline stage use a
+ *             per-handle scratch buffer: calls on one handle must be ordered
+ *             (same stream, or synchronised across streams).
  *   d_x       float32[n] (read-only; only entries referenced by a set bit are read,
  *             structural zeros are never multiplied).
  *   d_y       float32[m]; with beta == 0 it is write-only (its old contents, even

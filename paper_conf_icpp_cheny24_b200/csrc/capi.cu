@@ -44,7 +44,8 @@ static spaden_status_t check_device_ptr(const void *p, const char *name, int dev
 static void release(Matrix *A) {
     if (!A) return;
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap, A->blk_offset, A->values,
-                    A->stage_x,     A->stage_y,  A->tiles,  A->long_rows};
+                    A->stage_x,     A->stage_y,  A->tiles,  A->long_rows, A->chunk_start,
+                    A->chunk_row,   A->carry};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     delete A;

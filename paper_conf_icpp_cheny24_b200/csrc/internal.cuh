@@ -35,6 +35,10 @@ struct spaden_matrix_s {
     int tile_cfg = 0;                          // spaden::tile_cfg index the schedule was built for
     struct spaden_tile_desc_s *tiles = nullptr; // [n_tiles] (spaden::TileDesc)
     int32_t *long_rows = nullptr;              // [n_long]
+    int64_t n_chunks = 0;                      // kLongChunk-block chunks of the long rows
+    int32_t *chunk_start = nullptr;            // [n_long+1] first chunk of each long row
+    int32_t *chunk_row = nullptr;              // [n_chunks] index into long_rows
+    float *carry = nullptr;                    // [n_chunks*8] per-chunk row partials
 
     // host-API staging buffers (lazily allocated)
     float *stage_x = nullptr;
@@ -84,6 +88,9 @@ constexpr int kStageSlack = 384;
 // shared-memory bytes a block occupies in a stage: bitmap 8 + blk_col 4 +
 // blk_offset 4 (copied) + 8 fp32 row partials at a 9-word stride (scratch)
 constexpr int kBlockStageBytes = 16 + 36;
+// long block-rows are split into chunks of this many blocks (relative to the
+// block-row start, so the split depends only on the row itself)
+constexpr int kLongChunk = 1024;
 // mean nonzeros per block from which the predicated-slot decode is used
 constexpr int kSlotsMinFill = 8;
 // decode used above that fill (1 = lane per block, 2 = lane per block row)

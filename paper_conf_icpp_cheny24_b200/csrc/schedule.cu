@@ -5,9 +5,10 @@
 // blk_rowptr slice fit one pipeline stage (TileCfg::stage_bytes).  Keeping block-rows
 // whole keeps each row's summation order a function of that block-row alone
 // (deterministic and independent of how rows are partitioned across GPUs).
-// A block-row too large for half a stage is "long": it is listed separately
-// and processed straight from global memory by the long-row kernel with the
-// same lane mapping and summation order.
+// A block-row too large for half a stage is "long": it is listed separately,
+// cut into kLongChunk-block chunks (counted from the row start) processed
+// straight from global memory by k_spmv_long_chunks, and its chunk partials are
+// summed in chunk order by k_spmv_long_fixup.
 //
 // Tiles are packed greedily inside segments of kSeg block-rows (one thread per
 // segment; two passes: count, then write after a scan of the counts).
@@ -81,6 +82,21 @@ __global__ void k_pack(int64_t Bnrow, const int32_t *__restrict__ brp, const int
     }
 }
 
+__global__ void k_long_chunks(int nlong, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ brp,
+                              int32_t *__restrict__ cnt) {
+    const int j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j < nlong) {
+        const int br = long_rows[j];
+        cnt[j] = (brp[br + 1] - brp[br] + kLongChunk - 1) / kLongChunk;
+    }
+}
+
+__global__ void k_chunk_rows(int nlong, const int32_t *__restrict__ chunk_start, int32_t *__restrict__ chunk_row) {
+    const int j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j < nlong)
+        for (int c = chunk_start[j]; c < chunk_start[j + 1]; ++c) chunk_row[c] = j;
+}
+
 __global__ void k_sched_summary(const int32_t *tile_total, const int32_t *long_total, int32_t *out) {
     out[0] = *tile_total;
     out[1] = *long_total;
@@ -141,6 +157,33 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     e = cudaGetLastError();
     cudaFreeAsync(tmp, st);
     if (e != cudaSuccess) return cuda_status(e, "packing SpMV schedule");
+    if (A->n_long == 0) return SPADEN_OK;
+
+    // long block-rows -> fixed kLongChunk-block chunks (+ carry slots)
+    const int nl = (int)A->n_long;
+    int32_t *ltmp = nullptr;
+    const size_t lt = scan_tmp_ints(nl + 1);
+    SPADEN_CUDA_TRY(cudaMallocAsync(&ltmp, (lt + 4) * sizeof(int32_t), st));
+    e = cudaMalloc(&A->chunk_start, sizeof(int32_t) * (nl + 1));
+    if (e == cudaSuccess) {
+        k_long_chunks<<<(nl + 255) / 256, 256, 0, st>>>(nl, A->long_rows, A->blk_rowptr, A->chunk_start);
+        e = exclusive_scan_i32(A->chunk_start, A->chunk_start, nl, ltmp, st);
+    }
+    int32_t nch = 0;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&nch, A->chunk_start + nl, sizeof(int32_t), cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    cudaFreeAsync(ltmp, st);
+    if (e == cudaSuccess) {
+        A->n_chunks = nch;
+        e = cudaMalloc(&A->chunk_row, sizeof(int32_t) * std::max(1, nch));
+    }
+    if (e == cudaSuccess) e = cudaMalloc(&A->carry, sizeof(float) * 8 * std::max(1, nch));
+    if (e == cudaSuccess) {
+        k_chunk_rows<<<(nl + 255) / 256, 256, 0, st>>>(nl, A->chunk_start, A->chunk_row);
+        e = cudaGetLastError();
+    }
+    if (e != cudaSuccess) return cuda_status(e, "long-row chunk schedule");
+    A->aux_bytes += (int64_t)sizeof(int32_t) * (nl + 1 + nch) + (int64_t)sizeof(float) * 8 * nch;
     return SPADEN_OK;
 }
 

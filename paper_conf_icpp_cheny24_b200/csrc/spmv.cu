@@ -5,7 +5,8 @@
 //   k_spmv_tiled  (default)  persistent CTAs fed by a TMA bulk-copy pipeline;
 //   k_spmv_v0     (SPADEN_KERNEL=v0) the first, simple row-byte kernel, kept as
 //                 the measured baseline of DESIGN.md.
-// and k_spmv_long for block-rows too large for a pipeline stage.
+// and k_spmv_long_chunks + k_spmv_long_fixup for block-rows too large for a
+// pipeline stage.
 //
 // Decode (both kernels follow PAPER.md §4.3.1 / Alg. 2 semantics):
 // bit 8r+c of a block's bitmap is entry (r, c); its value is the
@@ -469,24 +470,30 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
     }
 }
 
-// Long block-rows (too large for a stage): one warp per block-row straight from
-// global memory; lane j takes blocks j, j+32, ... (one lane per block, same
-// per-block arithmetic as the tiled kernel), then a fixed xor tree over lanes.
+// Long block-rows (too large for a stage), straight from global memory.
+// k_spmv_long_chunks: one warp per kLongChunk-block chunk; lane j takes blocks
+// j, j+32, ... of the chunk (same per-block arithmetic as the tiled kernel),
+// sums them in that order, then a fixed xor tree over the lanes gives the
+// chunk's 8 row partials (carry).  k_spmv_long_fixup: the chunks of a row are
+// added in chunk order.  The order depends only on the block-row.
 template <typename V, bool SLOTS>
 __global__ void __launch_bounds__(256)
-k_spmv_long(int64_t m, const int32_t *__restrict__ long_rows, int nlong, const int32_t *__restrict__ blk_rowptr,
-            const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
-            const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
-            int nbc_vec, float alpha, float beta, float *__restrict__ y) {
+k_spmv_long_chunks(int nchunks, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
+                   const int32_t *__restrict__ chunk_row, const int32_t *__restrict__ blk_rowptr,
+                   const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
+                   const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
+                   int nbc_vec, float *__restrict__ carry) {
     const int w = (int)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
     const int lane = threadIdx.x & 31;
-    if (w >= nlong) return;
-    const int br = long_rows[w];
-    const int b0 = blk_rowptr[br], b1 = blk_rowptr[br + 1];
+    if (w >= nchunks) return;
+    const int j = chunk_row[w];
+    const int br = long_rows[j];
+    const int cb0 = blk_rowptr[br] + (w - chunk_start[j]) * kLongChunk;
+    const int cb1 = min(blk_rowptr[br + 1], cb0 + kLongChunk);
     float tot[8];
 #pragma unroll
     for (int r = 0; r < 8; ++r) tot[r] = 0.f;
-    for (int b = b0 + lane; b < b1; b += 32) {
+    for (int b = cb0 + lane; b < cb1; b += 32) {
         const uint64_t w64 = __ldg(bitmap + b);
         const uint2 bm = make_uint2((uint32_t)w64, (uint32_t)(w64 >> 32));
         const int bc = __ldg(blk_col + b);
@@ -507,17 +514,26 @@ k_spmv_long(int64_t m, const int32_t *__restrict__ long_rows, int nlong, const i
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) tot[r] += __shfl_xor_sync(kFull, tot[r], o);
     }
-    if (lane < 8) {
-        const int64_t row = 8 * (int64_t)br + lane;
-        float sum = tot[0];
-#pragma unroll
-        for (int r = 1; r < 8; ++r)
-            if (lane == r) sum = tot[r];
-        if (row < m) {
-            float o = alpha * sum;
-            if (beta != 0.f) o = fmaf(beta, y[row], o);
-            y[row] = o;
-        }
+    if (lane == 0) {
+        float4 *c4 = reinterpret_cast<float4 *>(carry + 8 * (int64_t)w);
+        c4[0] = make_float4(tot[0], tot[1], tot[2], tot[3]);
+        c4[1] = make_float4(tot[4], tot[5], tot[6], tot[7]);
+    }
+}
+
+__global__ void k_spmv_long_fixup(int64_t m, int nlong, const int32_t *__restrict__ long_rows,
+                                  const int32_t *__restrict__ chunk_start, const float *__restrict__ carry, float alpha,
+                                  float beta, float *__restrict__ y) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= 8 * (int64_t)nlong) return;
+    const int j = (int)(t >> 3), r = (int)(t & 7);
+    float sum = 0.f;
+    for (int c = chunk_start[j]; c < chunk_start[j + 1]; ++c) sum += carry[8 * (int64_t)c + r];
+    const int64_t row = 8 * (int64_t)long_rows[j] + r;
+    if (row < m) {
+        float o = alpha * sum;
+        if (beta != 0.f) o = fmaf(beta, y[row], o);
+        y[row] = o;
     }
 }
 
@@ -561,10 +577,12 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
             A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y);
     }
     if (A.n_long > 0) {
-        const int64_t threads = 32 * A.n_long;
-        k_spmv_long<V, (DEC != 0)><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
-            A.m, A.long_rows, (int)A.n_long, A.blk_rowptr, A.blk_col, A.bitmap, A.blk_offset, (const V *)A.values,
-            x, nbc_vec, alpha, beta, y);
+        const int64_t threads = 32 * A.n_chunks;
+        k_spmv_long_chunks<V, (DEC != 0)><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+            (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
+            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry);
+        k_spmv_long_fixup<<<(unsigned)((8 * A.n_long + 255) / 256), 256, 0, st>>>(
+            A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y);
     }
     return cudaGetLastError();
 }
