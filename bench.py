@@ -44,7 +44,8 @@ def parse():
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=2000)
     p.add_argument("--warmup", type=int, default=20)
-    p.add_argument("--workload", default="fem1p5m", choices=sorted(W.CONFIGS))
+    p.add_argument("--workload", default="fem1p5m",
+                   help="one of %s, or rmatNN (PageRank on R-MAT scale NN, e.g. rmat25)" % sorted(W.CONFIGS))
     p.add_argument("--dtype", default="fp32", choices=["fp32", "fp16"])
     p.add_argument("--impl", default="spaden", choices=["spaden", "reference"])
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -146,9 +147,18 @@ def reference_arm(args):
     if rank != 0:
         return 0
     import oracle
-    A = W.make(args.workload)
+    if args.workload.startswith("rmat"):  # GPU-generated (same stream as the CUDA arm), host sample
+        import torch
+        scale = int(args.workload[4:])
+        dev = "cuda" if torch.cuda.is_available() else "cpu"
+        k = max(8, (1 << scale) // 64)
+        rp, ci, v, n, _ = W.pagerank_slice_torch(scale, 32, 0, k, seed=0, device=dev)
+        A = W.CSR(k, n, rp.cpu().numpy(), ci.cpu().numpy(), v.cpu().numpy())
+        x = np.full(n, 1.0 / n, np.float32)
+    else:
+        A = W.make(args.workload)
+        x = W.vector(A.n, 2)
     vals = A.values if args.dtype == "fp32" else oracle.f32_to_f16(A.values)
-    x = W.vector(A.n, 2)
     oracle.lib()
     # per-step budget so that K+W steps take ~90 s of CPU time in total
     t0 = time.perf_counter()
@@ -181,6 +191,44 @@ def reference_arm(args):
     return 0
 
 
+class Workload:
+    """This rank's slice of the benchmark matrix plus the iteration it runs."""
+
+    def __init__(self, name, rank, world, dev):
+        import torch
+
+        from paper_conf_icpp_cheny24_b200.dist import RowPartition
+
+        self.name = name
+        if name.startswith("rmat"):  # PageRank on R-MAT (generated on the GPU)
+            scale = int(name[4:])
+            self.m = self.n = 1 << scale
+            self.part = RowPartition(self.m, world)
+            r0, r1 = self.part.range(rank)
+            rp, ci, v, _, self.nnz = W.pagerank_slice_torch(scale, 32, r0, r1, seed=0, device=dev)
+            self.local = (rp, ci, v)
+            self.local_nnz = int(ci.numel())
+            self.alpha, self.c = 0.85, 0.15 / self.n
+            self.x0 = torch.full((self.n,), 1.0 / self.n, dtype=torch.float32, device=dev)
+            self.host = None
+            self.step_desc = "PageRank x <- 0.85 A x + 0.15/n"
+        else:
+            A = W.make(name)
+            self.host = A
+            self.m, self.n, self.nnz = A.m, A.n, A.nnz
+            self.part = RowPartition(A.m, world)
+            r0, r1 = self.part.range(rank)
+            S = A.row_slice(r0, r1)
+            self.local = tuple(torch.from_numpy(a).to(dev) for a in (S.rowptr, S.colidx, S.values))
+            self.local_nnz = S.nnz
+            csum = np.concatenate([[0.0], np.cumsum(np.abs(A.values.astype(np.float64)))])
+            a_inf = float((csum[A.rowptr[1:]] - csum[A.rowptr[:-1]]).max()) if A.m else 0.0
+            self.alpha, self.c = (1.0 / a_inf if a_inf > 0 else 1.0), None
+            self.x0 = torch.from_numpy(W.vector(A.n, 2)).to(dev)
+            self.step_desc = "x <- A x / ||A||_inf"
+        self.r0, self.r1 = self.part.range(rank)
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -190,6 +238,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_icpp_cheny24_b200 as sp
+    from paper_conf_icpp_cheny24_b200.dist import IteratedSpMV
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -200,48 +249,31 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
 
     # ---- workload (identical on every rank), this rank's 8-row-aligned slice
-    A = W.make(args.workload)
-    slice_rows = -(-A.m // (8 * world)) * 8
-    r0, r1 = rank * slice_rows, min(A.m, (rank + 1) * slice_rows)
-    S = A.row_slice(r0, r1)
-    csum = np.concatenate([[0.0], np.cumsum(np.abs(A.values.astype(np.float64)))])
-    a_inf = float((csum[A.rowptr[1:]] - csum[A.rowptr[:-1]]).max()) if A.m else 0.0
-    alpha = 1.0 / a_inf if a_inf > 0 else 1.0
+    wl = Workload(args.workload, rank, world, dev)
     sv = 2 if args.dtype == "fp16" else 4
-
-    rp = torch.from_numpy(S.rowptr).to(dev)
-    ci = torch.from_numpy(S.colidx).to(dev)
-    vv = torch.from_numpy(S.values).to(dev)
     stream = torch.cuda.current_stream(dev)
     torch.cuda.synchronize(dev)
     t0 = time.perf_counter()
-    M = sp.convert(rp, ci, vv, A.n, storage=args.dtype)
+    M = sp.convert(*wl.local, wl.n, storage=args.dtype)
     torch.cuda.synchronize(dev)
     convert_s = time.perf_counter() - t0
     info = M.info
-    del rp, ci, vv
+    local_csr = wl.local
+    wl.local = None
 
-    nx = slice_rows * world
-    x0 = np.zeros(nx, np.float32)
-    x0[: A.n] = W.vector(A.n, 2)
-    xa = torch.from_numpy(x0).to(dev)
-    xb = torch.zeros(nx, dtype=torch.float32, device=dev)
-    x_a, x_b = xa, xb
+    ev_pair = [None]
 
-    def step(ev_pair=None):
-        nonlocal x_a, x_b
-        ys = x_b[rank * slice_rows: rank * slice_rows + S.m]
-        if ev_pair is not None:
-            ev_pair[0].record(stream)
-        M.spmv(x_a[: A.n], ys, alpha=alpha, beta=0.0, stream=stream)
-        if ev_pair is not None:
-            ev_pair[1].record(stream)
-        if world > 1:
-            dist.all_gather_into_tensor(x_b, x_b[rank * slice_rows:(rank + 1) * slice_rows])
-        x_a, x_b = x_b, x_a
+    def local_spmv(x, y, alpha, beta):
+        if ev_pair[0] is not None:
+            ev_pair[0][0].record(stream)
+        M.spmv(x, y, alpha=alpha, beta=beta, stream=stream)
+        if ev_pair[0] is not None:
+            ev_pair[0][1].record(stream)
+
+    it = IteratedSpMV(wl.part, wl.n, local_spmv, wl.x0, rank)
 
     for _ in range(max(3, args.warmup)):
-        step()
+        it.step(wl.alpha, wl.c)
     torch.cuda.synchronize(dev)
 
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
@@ -253,7 +285,9 @@ def main():
     with Clocks(local) as clk:
         start.record(stream)
         for i in range(args.steps):
-            step(evs[i])
+            ev_pair[0] = evs[i]
+            it.step(wl.alpha, wl.c)
+        ev_pair[0] = None
         end.record(stream)
         torch.cuda.synchronize(dev)
     if world > 1:
@@ -265,11 +299,11 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     elapsed_ms = float(t.item())
     ms_per_step = elapsed_ms / args.steps
-    gflops = 2.0 * A.nnz * args.steps / (elapsed_ms * 1e-3) / 1e9
+    gflops = 2.0 * wl.nnz * args.steps / (elapsed_ms * 1e-3) / 1e9
 
     # ---- roofline of the dominant kernel (the SpMV) on this rank
     kavg_ms = float(np.mean(kernel_ms))
-    abytes = alg_bytes(S.m, A.n, S.nnz, info.Bnrow, info.Bnnz, sv)
+    abytes = alg_bytes(wl.r1 - wl.r0, wl.n, wl.local_nnz, info.Bnrow, info.Bnnz, sv, beta_nonzero=wl.c is not None)
     peak, peak_kind = peaks()
     achieved = abytes / (kavg_ms * 1e-3) / 1e9
     traffic = None
@@ -285,25 +319,26 @@ def main():
     line = None
     if rank == 0:
         clocks = clk.summary()
-        # ---- e2e through the C ABI with host buffers (N=1 rank-local; H2D x, D2H y per step)
+        beta = 0.0 if wl.c is None else 1.0
+        # ---- e2e through the C ABI with host buffers (H2D x (+y), SpMV, D2H y per step)
         e2e = None
         if world == 1:
-            xh = torch.from_numpy(x0[: A.n].copy()).pin_memory()
-            yh = torch.empty(S.m, dtype=torch.float32).pin_memory()
+            xh = wl.x0.cpu().pin_memory()
+            yh = torch.full((wl.m,), wl.c or 0.0, dtype=torch.float32).pin_memory()
             for _ in range(3):
-                M.spmv_host(xh, yh, alpha=alpha, stream=stream)
+                M.spmv_host(xh, yh, alpha=wl.alpha, beta=beta, stream=stream)
             e2e_steps = max(20, min(args.steps, 200))
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
             torch.cuda.synchronize(dev)
             e0.record(stream)
             for _ in range(e2e_steps):
-                M.spmv_host(xh, yh, alpha=alpha, stream=stream)
+                M.spmv_host(xh, yh, alpha=wl.alpha, beta=beta, stream=stream)
             e1.record(stream)
             torch.cuda.synchronize(dev)
             e2e_ms = e0.elapsed_time(e1) / e2e_steps
-            e2e = {"value": 2.0 * A.nnz / (e2e_ms * 1e-3) / 1e9, "unit": UNIT,
-                   "h2d_bytes_per_step": 4 * A.n, "d2h_bytes_per_step": 4 * S.m,
+            e2e = {"value": 2.0 * wl.nnz / (e2e_ms * 1e-3) / 1e9, "unit": UNIT,
+                   "h2d_bytes_per_step": 4 * wl.n + (4 * wl.m if beta else 0), "d2h_bytes_per_step": 4 * wl.m,
                    "ms_per_step": e2e_ms, "steps": e2e_steps,
                    "api": "spaden_spmv_host (pinned host x/y, stream-synchronous)"}
 
@@ -311,9 +346,8 @@ def main():
         cus = None
         if not args.no_cusparse and world == 1:
             try:
-                Ac = torch.sparse_csr_tensor(torch.from_numpy(A.rowptr).to(dev), torch.from_numpy(A.colidx).to(dev),
-                                             torch.from_numpy(A.values).to(dev), size=(A.m, A.n))
-                xv = xa[: A.n].contiguous()
+                Ac = torch.sparse_csr_tensor(*local_csr, size=(wl.m, wl.n))
+                xv = wl.x0.contiguous()
                 for _ in range(5):
                     yc = torch.mv(Ac, xv)
                 reps = max(20, min(args.steps, 500))
@@ -326,10 +360,10 @@ def main():
                 c1.record(stream)
                 torch.cuda.synchronize(dev)
                 cms = c0.elapsed_time(c1) / reps
-                csr_bytes = 4 * (A.m + 1) + 8 * A.nnz
+                csr_bytes = 4 * (wl.m + 1) + 8 * wl.nnz
                 cus = {"impl": "torch.mv(sparse_csr fp32) -> cuSPARSE SpMV", "ms": cms,
-                       "gflops": 2.0 * A.nnz / (cms * 1e-3) / 1e9,
-                       "footprint_bytes": csr_bytes, "bytes_per_nnz": csr_bytes / A.nnz,
+                       "gflops": 2.0 * wl.nnz / (cms * 1e-3) / 1e9,
+                       "footprint_bytes": csr_bytes, "bytes_per_nnz": csr_bytes / wl.nnz,
                        "speedup_spaden_vs_cusparse": cms / kavg_ms,
                        "footprint_saving": csr_bytes / info.format_bytes}
                 del Ac, yc
@@ -338,30 +372,42 @@ def main():
 
         cpu = None
         if not args.no_cpu_baseline and world == 1:
-            cpu = cpu_oracle_gflops(A, x0[: A.n], args.cpu_seconds)
+            if wl.host is not None:
+                cpu = cpu_oracle_gflops(wl.host, wl.x0.cpu().numpy(), args.cpu_seconds)
+            else:  # bounded row sample of the GPU-generated matrix
+                rp, ci, v = local_csr
+                k = max(8, min(wl.m, wl.m // 64))
+                hi = int(rp[k].item())
+                S = W.CSR(k, wl.n, rp[:k + 1].cpu().numpy(), ci[:hi].cpu().numpy(), v[:hi].cpu().numpy())
+                cpu = cpu_oracle_gflops(S, wl.x0.cpu().numpy(), args.cpu_seconds)
 
+        n_launch = 1 + (2 if info.n_long > 0 else 0)  # tiled kernel [+ long-row chunks and fix-up]
         line = {
             "metric": METRIC, "value": gflops, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": max(3, args.warmup), "ms_per_step": ms_per_step, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32" if args.dtype == "fp32" else "f16xf32->f32",
             "data": "synthetic",
-            "config": {"workload": args.workload, "m": A.m, "n": A.n, "nnz": A.nnz, "Bnrow": int((A.m + 7) // 8),
-                       "Bnnz_rank0": int(info.Bnnz), "fill": A.nnz / max(1, info.Bnnz) if world == 1 else None,
-                       "values": args.dtype, "parallelism": f"row-partition x{world}" + (" + NCCL all-gather" if world > 1 else ""),
-                       "l2": "inputs larger than L2 (A > 126 MB), no flush", "step": "x <- A x / ||A||_inf"},
+            "config": {"workload": args.workload, "m": wl.m, "n": wl.n, "nnz": wl.nnz,
+                       "Bnrow": int((wl.m + 7) // 8), "Bnnz_rank0": int(info.Bnnz),
+                       "fill_rank0": wl.local_nnz / max(1, info.Bnnz),
+                       "values": args.dtype,
+                       "parallelism": f"row-partition x{world}" + (" + NCCL all-gather" if world > 1 else ""),
+                       "l2": "inputs larger than L2 (A > 126 MB), no flush" if info.format_bytes > 126e6
+                             else "matrix fits L2 (no flush): warm-L2 number",
+                       "step": wl.step_desc},
             "hbm_gbs": achieved,
             "bytes_per_nnz": {"stored": info.format_bytes / max(1, info.nnz),
-                              "moved": abytes / max(1, S.nnz)},
+                              "moved": abytes / max(1, wl.local_nnz)},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "peak_kind": f"{peak_kind} copy bandwidth (MEASURED_PEAKS.json hbm_gbs)",
-                         "kernel": "k_spmv (one launch per step)", "kernel_ms": kavg_ms,
-                         "alg_bytes_per_launch": abytes},
-            "convert": {"seconds": convert_s, "ns_per_nnz": convert_s * 1e9 / max(1, S.nnz)},
+                         "kernel": "spaden_spmv (k_spmv_tiled [+ long-row chunks/fix-up])",
+                         "kernel_ms": kavg_ms, "alg_bytes_per_launch": abytes},
+            "convert": {"seconds": convert_s, "ns_per_nnz": convert_s * 1e9 / max(1, wl.local_nnz)},
             "cusparse_csr": cus,
             "cpu_baseline": cpu,
             "e2e": e2e,
-            "gpu_launches": args.steps,
+            "gpu_launches": args.steps * n_launch,
             "clocks": clocks,
         }
         print(json.dumps(line), flush=True)

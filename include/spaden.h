@@ -78,6 +78,7 @@ typedef struct {
                                    bitBSR footprint (2.85 B/nnz with fp16 values) */
     int64_t aux_bytes;          /* extra device bytes (SpMV work schedule, padding)       */
     int64_t n_tiles;            /* SpMV work tiles in the schedule                         */
+    int64_t n_long;             /* block-rows too large for a tile (processed in chunks)  */
 } spaden_info_t;
 
 typedef struct {                /* borrowed device views; valid until spaden_free         */

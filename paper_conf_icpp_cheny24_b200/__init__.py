@@ -40,7 +40,7 @@ class spaden_info_t(ctypes.Structure):
                 ("Bnrow", ctypes.c_int64), ("Bnnz", ctypes.c_int64),
                 ("storage_dtype", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("format_bytes", ctypes.c_int64), ("aux_bytes", ctypes.c_int64),
-                ("n_tiles", ctypes.c_int64)]
+                ("n_tiles", ctypes.c_int64), ("n_long", ctypes.c_int64)]
 
 
 class spaden_arrays_t(ctypes.Structure):

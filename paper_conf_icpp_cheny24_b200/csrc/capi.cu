@@ -197,6 +197,7 @@ spaden_status_t spaden_get_info(spaden_matrix_t A, spaden_info_t *info) {
     info->format_bytes = 4 * (A->Bnrow + 1) + 4 * A->Bnnz + 8 * A->Bnnz + 4 * (A->Bnnz + 1) + sv * A->nnz;
     info->aux_bytes = A->aux_bytes;
     info->n_tiles = A->n_tiles;
+    info->n_long = A->n_long;
     return SPADEN_OK;
 }
 

@@ -385,3 +385,38 @@ def test_fem1p5m_full(sp, torch):
             assert np.array_equal(off - off[0], B.blk_offset)
             assert off[0] == A.rowptr[8 * br]
         M.free()
+
+
+def test_long_rows_deterministic_and_partition_invariant(sp, torch):
+    """Block-rows far larger than a pipeline stage (hub rows) go through the
+    chunked long-row path; y is deterministic, within tolerance, and identical
+    under an 8-row-aligned row split."""
+    A = hub_matrix(m=96, n=400_003, hub_rows=(3, 9, 60, 61), hub_nnz=120_000, seed=11)
+    M = convert(sp, torch, A)
+    assert M.info.n_long >= 2
+    x = W.vector(A.n, 13)
+    y1 = gpu_spmv(torch, M, x)
+    y2 = gpu_spmv(torch, M, x)
+    assert np.array_equal(y1, y2)
+    check_spmv(A, y1, A.values, x)
+    parts = [gpu_spmv(torch, convert(sp, torch, A.row_slice(r0, r1)), x) for r0, r1 in ((0, 56), (56, 96))]
+    assert np.array_equal(np.concatenate(parts), y1)
+
+
+def test_pagerank_iteration_vs_oracle(sp, torch):
+    """rmat-style PageRank (x <- 0.85 A x + 0.15/n) through the CUDA path and the
+    row-partition driver vs the fp64 oracle iteration."""
+    from paper_conf_icpp_cheny24_b200.dist import IteratedSpMV, RowPartition
+    scale, K = 14, 20
+    rp, ci, v, n, nnz = W.pagerank_slice_torch(scale, 16, 0, 1 << scale, seed=3, device="cuda")
+    M = sp.convert(rp, ci, v, n)
+    part = RowPartition(n, 1)
+    it = IteratedSpMV(part, n, lambda xx, yy, a, b: M.spmv(xx, yy, alpha=a, beta=b),
+                      torch.full((n,), 1.0 / n, device="cuda"), 0)
+    for _ in range(K):
+        x = it.step(0.85, 0.15 / n)
+    torch.cuda.synchronize()
+    ref = oracle.pagerank(rp.cpu().numpy(), ci.cpu().numpy(), v.cpu().numpy(), 0.85, K, np.full(n, 1.0 / n))
+    got = x[:n].cpu().numpy().astype(np.float64)
+    rel = np.abs(got - ref) / np.abs(ref)
+    assert rel.max() <= 1e-5, rel.max()

@@ -260,3 +260,63 @@ CONFIGS = {
 
 def make(name: str) -> CSR:
     return CONFIGS[name]()
+
+
+# --------------------------------------------------------------------------
+# R-MAT on the GPU (rmat25: ~1.07B edges; numpy is far too slow at that size)
+# --------------------------------------------------------------------------
+
+def rmat_torch(scale: int, edge_factor: int, seed: int = 0, device="cuda", relabel: bool = True,
+               abcd=(0.57, 0.19, 0.19, 0.05), chunk: int = 1 << 26):
+    """Graph500-style R-MAT edge stream generated with torch on `device` in fixed
+    chunks from one seeded generator, so every rank that calls it with the same
+    arguments gets the same stream.  Returns (src, dst) int64 tensors."""
+    import torch
+    g = torch.Generator(device=device)
+    g.manual_seed(seed)
+    n = 1 << scale
+    ne = edge_factor << scale
+    a, b, c, _ = abcd
+    src = torch.empty(ne, dtype=torch.int64, device=device)
+    dst = torch.empty(ne, dtype=torch.int64, device=device)
+    for s0 in range(0, ne, chunk):
+        k = min(chunk, ne - s0)
+        s = torch.zeros(k, dtype=torch.int64, device=device)
+        d = torch.zeros(k, dtype=torch.int64, device=device)
+        for level in range(scale):
+            u = torch.rand(k, generator=g, device=device)
+            bit_d = ((u >= a) & (u < a + b)) | (u >= a + b + c)
+            bit_s = u >= a + b
+            s |= bit_s.to(torch.int64) << level
+            d |= bit_d.to(torch.int64) << level
+        src[s0:s0 + k] = s
+        dst[s0:s0 + k] = d
+    if relabel:
+        perm = torch.randperm(n, generator=g, device=device)
+        src = perm[src]
+        dst = perm[dst]
+    return src, dst
+
+
+def pagerank_slice_torch(scale: int, edge_factor: int, r0: int, r1: int, seed: int = 0, device="cuda"):
+    """Rows [r0, r1) of the column-stochastic PageRank matrix A[dst][src] =
+    1/outdeg(src) over the unique edges of rmat_torch(...) (global columns).
+    Returns torch CSR pieces (rowptr int32[r1-r0+1], colidx int32, values fp32)
+    on `device`, and the global n and nnz."""
+    import torch
+    n = 1 << scale
+    src, dst = rmat_torch(scale, edge_factor, seed, device)
+    key = torch.unique(dst * n + src)          # sorted by (dst, src), duplicates removed
+    del src, dst
+    s = key % n
+    outdeg = torch.bincount(s, minlength=n)
+    nnz_total = int(key.numel())
+    lo = torch.searchsorted(key, torch.tensor([r0 * n, r1 * n], device=device))
+    ks = key[int(lo[0]):int(lo[1])]
+    rows = (ks // n - r0)
+    cols = (ks % n)
+    vals = (1.0 / outdeg[cols].to(torch.float64)).to(torch.float32)
+    counts = torch.bincount(rows, minlength=r1 - r0)
+    rowptr = torch.zeros(r1 - r0 + 1, dtype=torch.int64, device=device)
+    rowptr[1:] = torch.cumsum(counts, 0)
+    return rowptr.to(torch.int32), cols.to(torch.int32), vals, n, nnz_total
