@@ -72,15 +72,21 @@ enum : uint32_t {
 // stage including the 16-byte alignment slack of its regions.
 struct TileCfg {
     int ctas_per_sm, consumers, stages, stage_bytes;
+    int warp_mode;  // 0: CTA pipeline (producer warp + consumers share stages)
+                    // 1: warp pipelines (each warp streams its own tiles; consumers = warps/CTA)
 };
 constexpr int kMaxStages = 4;
-constexpr int kNumTileCfgs = 4;
+constexpr int kNumTileCfgs = 8;
 __host__ __device__ inline TileCfg tile_cfg(int i) {
     switch (i) {
-    case 1: return TileCfg{2, 16, 3, 36 * 1024};
-    case 2: return TileCfg{3, 8, 3, 24 * 1024};
-    case 3: return TileCfg{4, 8, 2, 27 * 1024};
-    default: return TileCfg{1, 16, 3, 64 * 1024};
+    case 1: return TileCfg{2, 16, 3, 36 * 1024, 0};
+    case 2: return TileCfg{3, 8, 3, 24 * 1024, 0};
+    case 3: return TileCfg{4, 8, 2, 27 * 1024, 0};
+    case 4: return TileCfg{3, 4, 2, 9 * 1024, 1};
+    case 5: return TileCfg{3, 4, 3, 6 * 1024, 1};
+    case 6: return TileCfg{2, 8, 2, 6 * 1024 + 512, 1};
+    case 7: return TileCfg{2, 4, 2, 13 * 1024, 1};
+    default: return TileCfg{1, 16, 3, 64 * 1024, 0};
     }
 }
 int default_tile_cfg();  // SPADEN_TILE_CFG env override, else the measured best

@@ -117,7 +117,9 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     A->tile_cfg = default_tile_cfg();
     const TileCfg cfg = tile_cfg(A->tile_cfg);
     const int64_t cap = cfg.stage_bytes - kStageSlack;
-    const int64_t long_cost = cfg.stage_bytes / 2;
+    // CTA pipelines: rows above half a stage are long (keeps tiles well packed);
+    // warp pipelines: any row that fits a stage alone stays in the tiles
+    const int64_t long_cost = cfg.warp_mode ? cap : cfg.stage_bytes / 2;
     if (Bnrow == 0) return SPADEN_OK;
 
     const size_t n_tmp = scan_tmp_ints(nseg + 1);

@@ -270,6 +270,40 @@ __device__ __forceinline__ void block_bits(uint2 bm, typename VS::P p, const flo
     }
 }
 
+// Phase 2: y for every block-row of a tile from the per-block row partials
+// (9-word stride), 4 block-rows x 8 rows per warp pass, 4 chains per row
+// indexed by block position within the block-row, combined (c0+c1)+(c2+c3).
+__device__ __forceinline__ void reduce_tile(uint32_t a_rp, uint32_t a_part, int nbr, int b0, int br0, int lane,
+                                            int64_t m, float alpha, float beta, float *__restrict__ y) {
+    const int r = lane & 7;
+    for (int base = 0; base < nbr; base += 4) {
+        const int brl = base + (lane >> 3);
+        if (brl < nbr) {
+            const int k0 = lds_i32(a_rp + 4u * brl) - b0;
+            const int k1 = lds_i32(a_rp + 4u * (brl + 1)) - b0;
+            float c0 = 0.f, c1 = 0.f, c2 = 0.f, c3 = 0.f;
+            uint32_t q = a_part + kPartStride * k0 + 4u * r;
+            int k = k0;
+            for (; k + 3 < k1; k += 4, q += 4 * kPartStride) {
+                c0 += lds_f32(q);
+                c1 += lds_f32(q + kPartStride);
+                c2 += lds_f32(q + 2 * kPartStride);
+                c3 += lds_f32(q + 3 * kPartStride);
+            }
+            if (k < k1) c0 += lds_f32(q);
+            if (k + 1 < k1) c1 += lds_f32(q + kPartStride);
+            if (k + 2 < k1) c2 += lds_f32(q + 2 * kPartStride);
+            const float sum = (c0 + c1) + (c2 + c3);
+            const int64_t row = 8 * ((int64_t)br0 + brl) + r;
+            if (row < m) {
+                float o = alpha * sum;
+                if (beta != 0.f) o = fmaf(beta, y[row], o);
+                y[row] = o;
+            }
+        }
+    }
+}
+
 struct alignas(16) StageHdr {
     int br0, nbr, b0, v0;                      // tile
     int nb, units, u_next, done;               // blocks, 32-block units, next unit to grab, units done
@@ -434,39 +468,127 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             }
             if (__shfl_sync(kFull, last, 0)) {  // phase 2: this warp completed the tile
                 __threadfence_block();
-                const int br0 = h0.x, nbr = h0.y, b0 = h0.z;
-                const uint32_t a_rp = h2.w;
-                const int r = lane & 7;
-                for (int base = 0; base < nbr; base += 4) {
-                    const int brl = base + (lane >> 3);
-                    if (brl < nbr) {
-                        const int k0 = lds_i32(a_rp + 4u * brl) - b0;
-                        const int k1 = lds_i32(a_rp + 4u * (brl + 1)) - b0;
-                        float c0 = 0.f, c1 = 0.f, c2 = 0.f, c3 = 0.f;
-                        uint32_t q = a_part + kPartStride * k0 + 4u * r;
-                        int k = k0;
-                        for (; k + 3 < k1; k += 4, q += 4 * kPartStride) {
-                            c0 += lds_f32(q);
-                            c1 += lds_f32(q + kPartStride);
-                            c2 += lds_f32(q + 2 * kPartStride);
-                            c3 += lds_f32(q + 3 * kPartStride);
-                        }
-                        if (k < k1) c0 += lds_f32(q);
-                        if (k + 1 < k1) c1 += lds_f32(q + kPartStride);
-                        if (k + 2 < k1) c2 += lds_f32(q + 2 * kPartStride);
-                        const float sum = (c0 + c1) + (c2 + c3);
-                        const int64_t row = 8 * ((int64_t)br0 + brl) + r;
-                        if (row < m) {
-                            float o = alpha * sum;
-                            if (beta != 0.f) o = fmaf(beta, y[row], o);
-                            y[row] = o;
-                        }
-                    }
-                }
+                reduce_tile((uint32_t)h2.w, a_part, h0.y, h0.z, h0.x, lane, m, alpha, beta, y);
             }
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(smem_u32(&empty_bar[s]));
+    }
+}
+
+// ==========================================================================
+// Warp-pipelined variant (TileCfg::warp_mode): every warp streams its own tiles
+// (tile t -> global warp t % total_warps) through a private S-stage ring of
+// shared memory: lane 0 issues the cp.async.bulk copies of tile k+S-1 into the
+// slot freed by tile k-1 and the warp waits on its own "full" mbarrier; phase 1
+// (lane per block, same decode) and phase 2 (same fixed-order block-row sums)
+// run inside the warp.  No cross-warp synchronisation at all.
+// ==========================================================================
+struct alignas(16) WarpHdr {
+    int br0, nbr, b0, v0, nb, pad0;
+    uint32_t a_bmp, a_col, a_off, a_rp, a_val, a_part;
+};
+
+template <typename V, int DEC, int WARPS, int S>
+__global__ void __launch_bounds__(32 * WARPS)
+k_spmv_warp(int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int ntiles,
+            const int32_t *__restrict__ blk_rowptr, const int32_t *__restrict__ blk_col,
+            const uint64_t *__restrict__ bitmap, const int32_t *__restrict__ blk_offset,
+            const V *__restrict__ vals, const float *__restrict__ x, int nbc_vec, float alpha, float beta,
+            float *__restrict__ y) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t full_bar[WARPS][S];
+    __shared__ WarpHdr hdr[WARPS][S];
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (lane == 0) {
+        for (int s = 0; s < S; ++s) mbar_init(smem_u32(&full_bar[w][s]), 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    const uint32_t wbase = smem_u32(smem) + (uint32_t)(w * S) * (uint32_t)stage_bytes;
+    const int gw = blockIdx.x * WARPS + w, GW = gridDim.x * WARPS;
+    const uint64_t pol = policy_evict_first();
+
+    auto issue = [&](int k) {  // lane 0: tile gw + k*GW into slot k % S
+        const int t = gw + k * GW;
+        const int s = k % S;
+        const int4 d0 = __ldg(reinterpret_cast<const int4 *>(tiles + t));
+        const int4 d1 = __ldg(reinterpret_cast<const int4 *>(tiles + t) + 1);
+        const int br0 = d0.x, br1 = d0.y, b0 = d0.z, b1 = d0.w, v0 = d1.x, v1 = d1.y;
+        uint32_t cur = wbase + (uint32_t)s * (uint32_t)stage_bytes;
+        const uint32_t stage = cur;
+        struct Reg {
+            uintptr_t src;
+            uint32_t sz;
+        };
+        auto region = [&](const void *lo_p, size_t len, uint32_t *addr_out) {
+            const uintptr_t lo = (uintptr_t)lo_p, hi = lo + len;
+            const uintptr_t alo = lo & ~(uintptr_t)15, ahi = (hi + 15) & ~(uintptr_t)15;
+            *addr_out = cur + (uint32_t)(lo - alo);
+            const Reg r{alo, len > 0 ? (uint32_t)(ahi - alo) : 0u};
+            cur += r.sz;
+            return r;
+        };
+        WarpHdr h;
+        h.br0 = br0;
+        h.nbr = br1 - br0;
+        h.b0 = b0;
+        h.v0 = v0;
+        h.nb = b1 - b0;
+        h.pad0 = 0;
+        const Reg rs[5] = {region(bitmap + b0, 8u * (b1 - b0), &h.a_bmp),
+                           region(blk_col + b0, 4u * (b1 - b0), &h.a_col),
+                           region(blk_offset + b0, 4u * (b1 - b0), &h.a_off),
+                           region(blk_rowptr + br0, 4u * (br1 - br0 + 1), &h.a_rp),
+                           region(vals + v0, sizeof(V) * (size_t)(v1 - v0), &h.a_val)};
+        h.a_part = cur;
+        hdr[w][s] = h;
+        const uint32_t fb = smem_u32(&full_bar[w][s]);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // prior generic reads of the slot
+        mbar_arrive_expect_tx(fb, cur - stage);
+        uint32_t dst = stage;
+#pragma unroll
+        for (int q = 0; q < 5; ++q) {
+            if (rs[q].sz) bulk_g2s(dst, (const void *)rs[q].src, rs[q].sz, fb, pol);
+            dst += rs[q].sz;
+        }
+    };
+
+    const int my_tiles = gw < ntiles ? (ntiles - gw + GW - 1) / GW : 0;
+    if (lane == 0)
+        for (int k = 0; k < S - 1 && k < my_tiles; ++k) issue(k);
+    for (int k = 0; k < my_tiles; ++k) {
+        if (lane == 0 && k + S - 1 < my_tiles) issue(k + S - 1);
+        const int s = k % S;
+        mbar_wait(smem_u32(&full_bar[w][s]), (uint32_t)(k / S) & 1u);
+        __syncwarp();
+        const int4 h0 = lds_i4_volatile(smem_u32(&hdr[w][s].br0));
+        const int4 h1 = lds_i4_volatile(smem_u32(&hdr[w][s].nb));
+        const int4 h2 = lds_i4_volatile(smem_u32(&hdr[w][s].a_off));
+        const int br0 = h0.x, nbr = h0.y, b0 = h0.z, v0 = h0.w, nb = h1.x;
+        const uint32_t a_bmp = (uint32_t)h1.z, a_col = (uint32_t)h1.w, a_off = (uint32_t)h2.x;
+        const uint32_t a_rp = (uint32_t)h2.y, a_val = (uint32_t)h2.z, a_part = (uint32_t)h2.w;
+        for (int lb = lane; lb < ((nb + 31) & ~31); lb += 32) {  // phase 1: one block per lane
+            if (lb < nb) {
+                const uint2 bm = lds_u2(a_bmp + 8u * lb);
+                const int bc = lds_i32(a_col + 4u * lb);
+                const uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
+                float acc[8];
+                if constexpr (DEC != 0) {
+                    XSeg xs;
+                    load_x(xs, x, bc, nbc_vec, used_cols(bm));
+                    block_slots<SmemVals<V>>(bm, p, xs, acc);
+                } else {
+                    block_bits<SmemVals<V>>(bm, p, x + 8 * (int64_t)bc, acc);
+                }
+                const uint32_t q = a_part + kPartStride * lb;
+#pragma unroll
+                for (int r = 0; r < 8; ++r) sts_f32(q + 4u * r, acc[r]);
+            }
+        }
+        __syncwarp();
+        reduce_tile(a_rp, a_part, nbr, b0, br0, lane, m, alpha, beta, y);  // phase 2
+        __syncwarp();
     }
 }
 
@@ -561,14 +683,16 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
                              float *y, cudaStream_t st) {
     const int nbc_vec = ((uintptr_t)x & 31u) == 0 ? (int)(A.n / 8) : 0;
     const size_t smem = (size_t)cfg.stages * cfg.stage_bytes;
-    static int occ = 0;  // resident CTAs per SM actually achievable (registers, smem)
-    if (occ == 0) {
+    static size_t occ_smem = 0;  // resident CTAs per SM (registers, smem), cached per smem size
+    static int occ = 0;
+    if (occ_smem != smem) {
         auto kern = k_spmv_tiled<V, DEC, CONSUMERS, MINB>;
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e == cudaSuccess)
             e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * (CONSUMERS + 1), smem);
         if (e != cudaSuccess) return e;
         occ = std::max(1, std::min(occ, MINB));
+        occ_smem = smem;
     }
     if (A.n_tiles > 0) {
         const int grid = (int)std::min<int64_t>(A.n_tiles, (int64_t)sm_count() * occ);
@@ -587,10 +711,47 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
     return cudaGetLastError();
 }
 
+template <typename V, int DEC, int WARPS, int S>
+cudaError_t launch_warp_cfg(const Matrix &A, const TileCfg &cfg, float alpha, const float *x, float beta,
+                            float *y, cudaStream_t st) {
+    const int nbc_vec = ((uintptr_t)x & 31u) == 0 ? (int)(A.n / 8) : 0;
+    const size_t smem = (size_t)WARPS * S * cfg.stage_bytes;
+    static size_t occ_smem = 0;  // occupancy cached per dynamic-smem size
+    static int occ = 0;
+    if (occ_smem != smem) {
+        auto kern = k_spmv_warp<V, DEC, WARPS, S>;
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * WARPS, smem);
+        if (e != cudaSuccess) return e;
+        occ = std::max(1, std::min(occ, cfg.ctas_per_sm));
+        occ_smem = smem;
+    }
+    if (A.n_tiles > 0) {
+        const int64_t need = (A.n_tiles + WARPS - 1) / WARPS;
+        const int grid = (int)std::min<int64_t>(need, (int64_t)sm_count() * occ);
+        k_spmv_warp<V, DEC, WARPS, S><<<grid, 32 * WARPS, smem, st>>>(
+            cfg.stage_bytes, A.m, A.tiles, (int)A.n_tiles, A.blk_rowptr, A.blk_col, A.bitmap, A.blk_offset,
+            (const V *)A.values, x, nbc_vec, alpha, beta, y);
+    }
+    if (A.n_long > 0) {
+        const int64_t threads = 32 * A.n_chunks;
+        k_spmv_long_chunks<V, (DEC != 0)><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+            (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
+            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry);
+        k_spmv_long_fixup<<<(unsigned)((8 * A.n_long + 255) / 256), 256, 0, st>>>(
+            A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y);
+    }
+    return cudaGetLastError();
+}
+
 template <typename V, int DEC>
 cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st) {
     const TileCfg cfg = tile_cfg(A.tile_cfg);
     switch (A.tile_cfg) {
+    case 4: return launch_warp_cfg<V, DEC, 4, 2>(A, cfg, alpha, x, beta, y, st);
+    case 5: return launch_warp_cfg<V, DEC, 4, 3>(A, cfg, alpha, x, beta, y, st);
+    case 6: return launch_warp_cfg<V, DEC, 8, 2>(A, cfg, alpha, x, beta, y, st);
+    case 7: return launch_warp_cfg<V, DEC, 4, 2>(A, cfg, alpha, x, beta, y, st);
     case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st);
     case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st);
     case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);

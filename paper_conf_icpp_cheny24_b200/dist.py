@@ -42,7 +42,7 @@ def gather_slices(full, local, group=None):
     """full[world*slice] <- concat over ranks of local[slice] (in rank order)."""
     import torch.distributed as dist
 
-    if dist.get_world_size(group) == 1:
+    if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
         if full.data_ptr() != local.data_ptr():
             full[: local.numel()].copy_(local)
         return full

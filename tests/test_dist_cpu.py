@@ -92,3 +92,14 @@ def test_partition_shapes():
             rs = [p.range(r) for r in range(P)]
             assert rs[0][0] == 0 and rs[-1][1] == m
             assert all(a[1] == b[0] for a, b in zip(rs[:-1], rs[1:]))
+
+
+def test_single_process_without_process_group():
+    """N=1 (no torch.distributed init): the driver degenerates to a local copy."""
+    from paper_conf_icpp_cheny24_b200.dist import IteratedSpMV, RowPartition
+    A = W.fem(4, 4, 5, seed=1)
+    x0 = torch.from_numpy(W.vector(A.n, 3))
+    it = IteratedSpMV(RowPartition(A.m, 1), A.n, oracle_local_spmv(A), x0, 0)
+    x = it.step(0.01)
+    ys, _ = oracle.spmv(A.rowptr, A.colidx, A.values, x0.numpy())
+    assert np.array_equal(x[: A.n].numpy(), (0.01 * ys).astype(np.float32))

@@ -420,3 +420,24 @@ def test_pagerank_iteration_vs_oracle(sp, torch):
     got = x[:n].cpu().numpy().astype(np.float64)
     rel = np.abs(got - ref) / np.abs(ref)
     assert rel.max() <= 1e-5, rel.max()
+
+
+@pytest.mark.parametrize("cfg", list(range(8)))
+def test_every_tile_config_same_result(sp, torch, cfg, monkeypatch):
+    """All launch shapes (CTA or warp pipelines, SPADEN_TILE_CFG) give the oracle's
+    y within tolerance, and block-rows classified alike give bitwise equal y."""
+    A = W.make("fem62k")
+    x = W.vector(A.n, 17)
+    monkeypatch.setenv("SPADEN_TILE_CFG", str(cfg))
+    for storage, stored in (("fp32", A.values), ("fp16", oracle.f32_to_f16(A.values))):
+        M = convert(sp, torch, A, storage=storage)
+        y = gpu_spmv(torch, M, x)
+        check_spmv(A, y, stored, x)
+        if M.info.n_long == 0:   # no long rows: identical arithmetic for every config
+            monkeypatch.setenv("SPADEN_TILE_CFG", "3")
+            y3 = gpu_spmv(torch, convert(sp, torch, A, storage=storage), x)
+            monkeypatch.setenv("SPADEN_TILE_CFG", str(cfg))
+            assert np.array_equal(y, y3)
+    H = hub_matrix()
+    M = convert(sp, torch, H)
+    check_spmv(H, gpu_spmv(torch, M, W.vector(H.n, 3)), H.values, W.vector(H.n, 3))
