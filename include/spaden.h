@@ -144,6 +144,23 @@ SPADEN_API spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const flo
 SPADEN_API spaden_status_t spaden_spmv_host(spaden_matrix_t A, float alpha, const float *h_x, float beta,
                                  float *h_y, void *stream);
 
+/*
+ * spaden_spmv_host_batched -- nvec independent products y_k = alpha*A*x_k + beta*y_k
+ * with HOST vectors, pipelined: the host->device copy of x_{k+1} and the
+ * device->host copy of y_{k-1} overlap the SpMV of vector k (two internal copy
+ * streams owned by the handle, double-buffered device staging).
+ *
+ *   h_x     host float32, vector k at h_x + k*ldx (ldx >= n); pinned memory
+ *           is required for the copies to overlap.
+ *   h_y     host float32, vector k at h_y + k*ldy (ldy >= m); read when beta != 0.
+ *   nvec    number of vectors (>= 0).
+ *   stream  cudaStream_t (void*) on which the SpMVs run; the call returns after
+ *           every y_k is back on the host.  Not thread-safe per handle.
+ */
+SPADEN_API spaden_status_t spaden_spmv_host_batched(spaden_matrix_t A, float alpha, const float *h_x,
+                                                    int64_t ldx, float beta, float *h_y, int64_t ldy,
+                                                    int64_t nvec, void *stream);
+
 /* spaden_free -- synchronises the handle's device, then releases all device
  * arrays owned by A.  spaden_free(NULL) returns SPADEN_OK. */
 SPADEN_API spaden_status_t spaden_free(spaden_matrix_t A);

@@ -64,6 +64,9 @@ spaden_spmv.restype = _ST
 spaden_spmv_host = _lib.spaden_spmv_host
 spaden_spmv_host.argtypes = [_P, _F, _P, _F, _P, _P]
 spaden_spmv_host.restype = _ST
+spaden_spmv_host_batched = _lib.spaden_spmv_host_batched
+spaden_spmv_host_batched.argtypes = [_P, _F, _P, _I64, _F, _P, _I64, _I64, _P]
+spaden_spmv_host_batched.restype = _ST
 spaden_free = _lib.spaden_free
 spaden_free.argtypes = [_P]
 spaden_free.restype = _ST
@@ -83,7 +86,8 @@ spaden_version = _lib.spaden_version
 spaden_version.argtypes = []
 spaden_version.restype = ctypes.c_char_p
 
-EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_spmv", "spaden_spmv_host", "spaden_free",
+EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_spmv", "spaden_spmv_host", "spaden_spmv_host_batched",
+            "spaden_free",
             "spaden_get_info", "spaden_get_arrays", "spaden_status_string",
             "spaden_last_error_message", "spaden_version"]
 
@@ -195,6 +199,15 @@ class Matrix:
         _check(spaden_spmv_host(self._h, alpha, ctypes.c_void_p(x_host.data_ptr()), beta,
                                 ctypes.c_void_p(y_host.data_ptr()), _stream_ptr(stream)), "spaden_spmv_host")
         return y_host
+
+    def spmv_host_batched(self, X_host, Y_host, alpha: float = 1.0, beta: float = 0.0, stream=None):
+        """Rows of X_host (k x n, pinned) -> rows of Y_host (k x m); copies overlap the SpMVs."""
+        k = X_host.shape[0]
+        assert Y_host.shape[0] == k and X_host.stride(1) == 1 and Y_host.stride(1) == 1
+        _check(spaden_spmv_host_batched(self._h, alpha, ctypes.c_void_p(X_host.data_ptr()), X_host.stride(0), beta,
+                                        ctypes.c_void_p(Y_host.data_ptr()), Y_host.stride(0), k,
+                                        _stream_ptr(stream)), "spaden_spmv_host_batched")
+        return Y_host
 
     def free(self):
         if self._h:

@@ -40,9 +40,13 @@ struct spaden_matrix_s {
     int32_t *chunk_row = nullptr;              // [n_chunks] index into long_rows
     float *carry = nullptr;                    // [n_chunks*8] per-chunk row partials
 
-    // host-API staging buffers (lazily allocated)
+    // host-API staging buffers (lazily allocated): [2] slots for the batched pipeline
     float *stage_x = nullptr;
     float *stage_y = nullptr;
+    float *stage_x2 = nullptr;
+    float *stage_y2 = nullptr;
+    cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+    cudaEvent_t ev[8] = {};
 };
 
 namespace spaden {
@@ -75,7 +79,7 @@ struct TileCfg {
     int warp_mode;  // 0: CTA pipeline (producer warp + consumers share stages)
                     // 1: warp pipelines (each warp streams its own tiles; consumers = warps/CTA)
 };
-constexpr int kMaxStages = 4;
+constexpr int kMaxStages = 8;
 constexpr int kNumTileCfgs = 8;
 __host__ __device__ inline TileCfg tile_cfg(int i) {
     switch (i) {
@@ -83,9 +87,9 @@ __host__ __device__ inline TileCfg tile_cfg(int i) {
     case 2: return TileCfg{3, 8, 3, 24 * 1024, 0};
     case 3: return TileCfg{4, 8, 2, 27 * 1024, 0};
     case 4: return TileCfg{3, 4, 2, 9 * 1024, 1};
-    case 5: return TileCfg{3, 4, 3, 6 * 1024, 1};
-    case 6: return TileCfg{2, 8, 2, 6 * 1024 + 512, 1};
-    case 7: return TileCfg{2, 4, 2, 13 * 1024, 1};
+    case 5: return TileCfg{3, 8, 4, 18 * 1024, 0};
+    case 6: return TileCfg{2, 16, 6, 18 * 1024, 0};
+    case 7: return TileCfg{4, 8, 3, 18 * 1024, 0};
     default: return TileCfg{1, 16, 3, 64 * 1024, 0};
     }
 }

@@ -121,12 +121,15 @@ __device__ __forceinline__ void mbar_arrive(uint32_t bar) {
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
 }
+// try_wait suspends the warp (up to the hint) instead of spinning: waiting
+// warps then cost no issue slots
+constexpr uint32_t kSuspendHintNs = 0x989680;
 __device__ __forceinline__ bool mbar_try_wait(uint32_t bar, uint32_t parity) {
     uint32_t ok;
     asm volatile(
-        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n selp.u32 %0, 1, 0, p;\n}\n"
         : "=r"(ok)
-        : "r"(bar), "r"(parity)
+        : "r"(bar), "r"(parity), "r"(kSuspendHintNs)
         : "memory");
     return ok != 0;
 }
@@ -337,10 +340,9 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
     if (warp == 0) {  // ---------------------------------------------- producer
         if (lane == 0) {
             const uint64_t pol = policy_evict_first();
-            int i = 0;
-            for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
-                const int s = i % stages;
-                const uint32_t ph = (uint32_t)(i / stages) & 1u;
+            int i = 0, s = 0;
+            uint32_t ph = 0;
+            for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i, s = (s + 1 == stages) ? (ph ^= 1u, 0) : s + 1) {
                 const int4 d0 = __ldg(reinterpret_cast<const int4 *>(tiles + t));
                 const int4 d1 = __ldg(reinterpret_cast<const int4 *>(tiles + t) + 1);
                 const int br0 = d0.x, br1 = d0.y, b0 = d0.z, b1 = d0.w, v0 = d1.x, v1 = d1.y;
@@ -391,10 +393,9 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
     }
 
     // ------------------------------------------------------------ consumers
-    int i = 0;
-    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
-        const int s = i % stages;
-        const uint32_t ph = (uint32_t)(i / stages) & 1u;
+    int s = 0;
+    uint32_t ph = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, s = (s + 1 == stages) ? (ph ^= 1u, 0) : s + 1) {
         mbar_wait(smem_u32(&full_bar[s]), ph);
         const int4 h0 = lds_i4_volatile(smem_u32(&hdr[s].br0));
         const int4 h1 = lds_i4_volatile(smem_u32(&hdr[s].nb));
@@ -749,9 +750,9 @@ cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float bet
     const TileCfg cfg = tile_cfg(A.tile_cfg);
     switch (A.tile_cfg) {
     case 4: return launch_warp_cfg<V, DEC, 4, 2>(A, cfg, alpha, x, beta, y, st);
-    case 5: return launch_warp_cfg<V, DEC, 4, 3>(A, cfg, alpha, x, beta, y, st);
-    case 6: return launch_warp_cfg<V, DEC, 8, 2>(A, cfg, alpha, x, beta, y, st);
-    case 7: return launch_warp_cfg<V, DEC, 4, 2>(A, cfg, alpha, x, beta, y, st);
+    case 5: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st);
+    case 6: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st);
+    case 7: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
     case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st);
     case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st);
     case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);

@@ -441,3 +441,17 @@ def test_every_tile_config_same_result(sp, torch, cfg, monkeypatch):
     H = hub_matrix()
     M = convert(sp, torch, H)
     check_spmv(H, gpu_spmv(torch, M, W.vector(H.n, 3)), H.values, W.vector(H.n, 3))
+
+
+@pytest.mark.parametrize("beta", [0.0, 0.5])
+def test_spmv_host_batched(sp, torch, beta):
+    A = W.make("fem62k")
+    M = convert(sp, torch, A)
+    K = 5
+    X = torch.from_numpy(np.stack([W.vector(A.n, 40 + k) for k in range(K)])).pin_memory()
+    Y0 = np.stack([W.vector(A.m, 60 + k) for k in range(K)])
+    Y = torch.from_numpy(Y0.copy()).pin_memory()
+    M.spmv_host_batched(X, Y, alpha=1.5, beta=beta)
+    for k in range(K):
+        yd = gpu_spmv(torch, M, X[k].numpy(), alpha=1.5, beta=beta, y0=Y0[k])
+        assert np.array_equal(Y[k].numpy(), yd)
