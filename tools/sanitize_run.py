@@ -1,0 +1,41 @@
+"""Small end-to-end exercise of every kernel for compute-sanitizer
+(memcheck / racecheck / synccheck): conversions in all dtype modes, the tiled
+SpMV, the long-row chunk path, alpha/beta, the batched host pipeline."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tests"))
+
+import paper_conf_icpp_cheny24_b200 as sp  # noqa: E402
+import workloads as W  # noqa: E402
+from test_gpu_parity import hub_matrix  # noqa: E402
+
+
+def run(A, storage):
+    rp = torch.from_numpy(A.rowptr).cuda()
+    ci = torch.from_numpy(A.colidx).cuda()
+    v = torch.from_numpy(A.values).cuda()
+    M = sp.convert(rp, ci, v, A.n, storage=storage)
+    x = torch.from_numpy(W.vector(A.n, 1)).cuda()
+    y = torch.from_numpy(W.vector(A.m, 2)).cuda()
+    M.spmv(x, y, alpha=1.0, beta=0.5)
+    M.spmv(x, y)
+    torch.cuda.synchronize()
+    M.free()
+
+
+for A in (W.h2(), W.tiny(0), W.fem(6, 7, 8, seed=2), hub_matrix(m=40, n=70_001, hub_rows=(3, 30), hub_nnz=40_000)):
+    for st in ("fp32", "fp16"):
+        run(A, st)
+A = W.fem(5, 5, 6, seed=1)
+M = sp.convert(torch.from_numpy(A.rowptr).cuda(), torch.from_numpy(A.colidx).cuda(),
+               torch.from_numpy(A.values).cuda(), A.n)
+X = torch.from_numpy(np.stack([W.vector(A.n, k) for k in range(3)])).pin_memory()
+Y = torch.zeros((3, A.m)).pin_memory()
+M.spmv_host_batched(X, Y)
+print("sanitize run ok")
