@@ -50,6 +50,7 @@ def parse():
     p.add_argument("--impl", default="spaden", choices=["spaden", "reference"])
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-cusparse", action="store_true")
+    p.add_argument("--no-variants", action="store_true", help="skip the other-precision kernel timing")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     return p.parse_args()
 
@@ -383,6 +384,34 @@ def main():
                 S = W.CSR(k, wl.n, rp[:k + 1].cpu().numpy(), ci[:hi].cpu().numpy(), v[:hi].cpu().numpy())
                 cpu = cpu_oracle_gflops(S, wl.x0.cpu().numpy(), args.cpu_seconds)
 
+        # ---- the other value precision on the same matrix (kernel time only)
+        variants = {}
+        if world == 1 and not args.no_variants:
+            other = "fp16" if args.dtype == "fp32" else "fp32"
+            M2 = sp.convert(*local_csr, wl.n, storage=other)
+            i2 = M2.info
+            ys = torch.empty(wl.m, dtype=torch.float32, device=dev)
+            for _ in range(5):
+                M2.spmv(wl.x0, ys, alpha=wl.alpha, stream=stream)
+            reps = max(20, min(args.steps, 500))
+            v0e = torch.cuda.Event(enable_timing=True)
+            v1e = torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize(dev)
+            v0e.record(stream)
+            for _ in range(reps):
+                M2.spmv(wl.x0, ys, alpha=wl.alpha, stream=stream)
+            v1e.record(stream)
+            torch.cuda.synchronize(dev)
+            vms = v0e.elapsed_time(v1e) / reps
+            vb = alg_bytes(wl.m, wl.n, wl.local_nnz, i2.Bnrow, i2.Bnnz, 2 if other == "fp16" else 4)
+            variants[other] = {"kernel_ms": vms, "gflops": 2.0 * wl.nnz / (vms * 1e-3) / 1e9,
+                               "hbm_gbs": vb / (vms * 1e-3) / 1e9, "frac": vb / (vms * 1e-3) / 1e9 / peak,
+                               "bytes_per_nnz_stored": i2.format_bytes / max(1, i2.nnz),
+                               "note": "back-to-back launches, no L2 flush" + (" (matrix > L2)" if i2.format_bytes > 126e6
+                                                                                 else " (matrix fits L2)")}
+            M2.free()
+            del ys
+
         n_launch = 1 + (2 if info.n_long > 0 else 0)  # tiled kernel [+ long-row chunks and fix-up]
         line = {
             "metric": METRIC, "value": gflops, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -407,6 +436,7 @@ def main():
                          "kernel_ms": kavg_ms, "alg_bytes_per_launch": abytes},
             "convert": {"seconds": convert_s, "ns_per_nnz": convert_s * 1e9 / max(1, wl.local_nnz)},
             "cusparse_csr": cus,
+            "variants": variants,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": args.steps * n_launch,

@@ -80,7 +80,7 @@ struct TileCfg {
                     // 1: warp pipelines (each warp streams its own tiles; consumers = warps/CTA)
 };
 constexpr int kMaxStages = 8;
-constexpr int kNumTileCfgs = 8;
+constexpr int kNumTileCfgs = 10;
 __host__ __device__ inline TileCfg tile_cfg(int i) {
     switch (i) {
     case 1: return TileCfg{2, 16, 3, 36 * 1024, 0};
@@ -90,11 +90,15 @@ __host__ __device__ inline TileCfg tile_cfg(int i) {
     case 5: return TileCfg{3, 8, 4, 18 * 1024, 0};
     case 6: return TileCfg{2, 16, 6, 18 * 1024, 0};
     case 7: return TileCfg{4, 8, 3, 18 * 1024, 0};
+    case 8: return TileCfg{4, 8, 3, 9 * 1024, 0};
+    case 9: return TileCfg{4, 8, 4, 6 * 1024, 0};
     default: return TileCfg{1, 16, 3, 64 * 1024, 0};
     }
 }
-int default_tile_cfg();  // SPADEN_TILE_CFG env override, else the measured best
+int default_tile_cfg(int64_t format_bytes);  // SPADEN_TILE_CFG override, else by matrix size
 constexpr int kStageSlack = 384;
+constexpr int64_t kSmallMatrixBytes = 64ll << 20;  // below: kSmallTileCfg
+constexpr int kSmallTileCfg = 3;  // measured: smaller stages do not help fem62k
 // shared-memory bytes a block occupies in a stage: bitmap 8 + blk_col 4 +
 // blk_offset 4 (copied) + 8 fp32 row partials at a 9-word stride (scratch)
 constexpr int kBlockStageBytes = 16 + 36;

@@ -753,6 +753,8 @@ cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float bet
     case 5: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st);
     case 6: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st);
     case 7: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
+    case 8: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
+    case 9: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
     case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st);
     case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st);
     case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
