@@ -79,6 +79,8 @@ typedef struct {
     int64_t aux_bytes;          /* extra device bytes (SpMV work schedule, padding)       */
     int64_t n_tiles;            /* SpMV work tiles in the schedule                         */
     int64_t n_long;             /* block-rows too large for a tile (processed in chunks)  */
+    int64_t residual_nnz;       /* entries held in the CSR residual (hybrid mode, else 0);
+                                   format_bytes then also counts 4(m+1) + (4+s_v)*residual_nnz */
 } spaden_info_t;
 
 typedef struct {                /* borrowed device views; valid until spaden_free         */
@@ -86,8 +88,20 @@ typedef struct {                /* borrowed device views; valid until spaden_fre
     const int32_t  *blk_col;    /* [Bnnz]    */
     const uint64_t *bitmap;     /* [Bnnz]    */
     const int32_t  *blk_offset; /* [Bnnz+1]  */
-    const void     *values;     /* [nnz] of storage_dtype */
+    const void     *values;     /* [nnz - residual_nnz] of storage_dtype */
+    const int32_t  *res_rowptr; /* [m+1] hybrid residual CSR (NULL when residual_nnz == 0) */
+    const int32_t  *res_colidx; /* [residual_nnz] */
+    const void     *res_values; /* [residual_nnz] of storage_dtype */
 } spaden_arrays_t;
+
+/* Conversion options (spaden_convert_csr_to_bitmap_ex).  Zero-initialise. */
+typedef struct {
+    int32_t struct_size;        /* sizeof(spaden_convert_opts_t)                          */
+    int32_t residual_max_popc;  /* hybrid format: blocks holding at
+                                   most this many entries are stored as a CSR residual
+                                   instead of bitBSR blocks (0 = pure bitBSR, max 64)     */
+    int32_t reserved[6];
+} spaden_convert_opts_t;
 
 /*
  * spaden_convert_csr_to_bitmap -- CSR -> bitBSR on the GPU (§4.2).
@@ -113,6 +127,22 @@ SPADEN_API spaden_status_t spaden_convert_csr_to_bitmap(int64_t m, int64_t n, in
                                              const int32_t *d_rowptr, const int32_t *d_colidx,
                                              const void *d_values, spaden_dtype_t values_dtype,
                                              spaden_dtype_t storage_dtype, void *stream,
+                                             spaden_matrix_t *out);
+
+/*
+ * spaden_convert_csr_to_bitmap_ex -- as spaden_convert_csr_to_bitmap, with options
+ * (opts may be NULL = defaults).  With residual_max_popc = t > 0 the matrix is
+ * split by block: 8x8 blocks with <= t entries go to a CSR residual (row-sorted,
+ * global columns), the others stay bitBSR; spaden_spmv then computes
+ * y = alpha*(A_bit + A_res) x + beta*y.  Useful for low-degree matrices whose
+ * blocks hold ~1 entry (bitmaps are a burden there).  One more
+ * host synchronisation than the pure conversion.
+ */
+SPADEN_API spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n, int64_t nnz,
+                                             const int32_t *d_rowptr, const int32_t *d_colidx,
+                                             const void *d_values, spaden_dtype_t values_dtype,
+                                             spaden_dtype_t storage_dtype,
+                                             const spaden_convert_opts_t *opts, void *stream,
                                              spaden_matrix_t *out);
 
 /*

@@ -186,3 +186,29 @@ def csr_inf_norm(rowptr, values) -> float:
         return 0.0
     c = np.concatenate([[0.0], np.cumsum(v)])
     return float((c[rp[1:]] - c[rp[:-1]]).max())
+
+
+def hybrid_split(m, n, rowptr, colidx, values, t: int):
+    """Hybrid format reference: an entry goes
+    to the CSR residual iff its 8x8 block (row//8, col//8) holds at most t
+    entries; all other entries stay in bitBSR.  Returns (kept CSR, residual CSR)
+    as (rowptr int64[m+1], colidx int32, values) tuples, both row-sorted."""
+    rowptr = np.asarray(rowptr, np.int64)
+    colidx = np.asarray(colidx, np.int32)
+    values = np.asarray(values)
+    rows = np.repeat(np.arange(m, dtype=np.int64), np.diff(rowptr))
+    nbc = (n + 7) // 8
+    key = (rows // 8) * max(nbc, 1) + colidx.astype(np.int64) // 8
+    if key.size:
+        _, inv, cnt = np.unique(key, return_inverse=True, return_counts=True)
+        res = cnt[inv] <= t
+    else:
+        res = np.zeros(0, bool)
+
+    def sub(mask):
+        counts = np.bincount(rows[mask], minlength=m) if m else np.zeros(0, np.int64)
+        rp = np.zeros(m + 1, np.int64)
+        np.cumsum(counts, out=rp[1:])
+        return rp, colidx[mask], values[mask]
+
+    return sub(~res), sub(res)

@@ -40,13 +40,19 @@ class spaden_info_t(ctypes.Structure):
                 ("Bnrow", ctypes.c_int64), ("Bnnz", ctypes.c_int64),
                 ("storage_dtype", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("format_bytes", ctypes.c_int64), ("aux_bytes", ctypes.c_int64),
-                ("n_tiles", ctypes.c_int64), ("n_long", ctypes.c_int64)]
+                ("n_tiles", ctypes.c_int64), ("n_long", ctypes.c_int64), ("residual_nnz", ctypes.c_int64)]
 
 
 class spaden_arrays_t(ctypes.Structure):
     _fields_ = [("blk_rowptr", ctypes.c_void_p), ("blk_col", ctypes.c_void_p),
                 ("bitmap", ctypes.c_void_p), ("blk_offset", ctypes.c_void_p),
-                ("values", ctypes.c_void_p)]
+                ("values", ctypes.c_void_p), ("res_rowptr", ctypes.c_void_p),
+                ("res_colidx", ctypes.c_void_p), ("res_values", ctypes.c_void_p)]
+
+
+class spaden_convert_opts_t(ctypes.Structure):
+    _fields_ = [("struct_size", ctypes.c_int32), ("residual_max_popc", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 6)]
 
 
 _P = ctypes.c_void_p
@@ -58,6 +64,10 @@ spaden_convert_csr_to_bitmap = _lib.spaden_convert_csr_to_bitmap
 spaden_convert_csr_to_bitmap.argtypes = [_I64, _I64, _I64, _P, _P, _P, ctypes.c_int, ctypes.c_int, _P,
                                          ctypes.POINTER(_P)]
 spaden_convert_csr_to_bitmap.restype = _ST
+spaden_convert_csr_to_bitmap_ex = _lib.spaden_convert_csr_to_bitmap_ex
+spaden_convert_csr_to_bitmap_ex.argtypes = [_I64, _I64, _I64, _P, _P, _P, ctypes.c_int, ctypes.c_int,
+                                            ctypes.POINTER(spaden_convert_opts_t), _P, ctypes.POINTER(_P)]
+spaden_convert_csr_to_bitmap_ex.restype = _ST
 spaden_spmv = _lib.spaden_spmv
 spaden_spmv.argtypes = [_P, _F, _P, _F, _P, _P]
 spaden_spmv.restype = _ST
@@ -86,7 +96,7 @@ spaden_version = _lib.spaden_version
 spaden_version.argtypes = []
 spaden_version.restype = ctypes.c_char_p
 
-EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_spmv", "spaden_spmv_host", "spaden_spmv_host_batched",
+EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_spmv", "spaden_spmv_host", "spaden_spmv_host_batched",
             "spaden_free",
             "spaden_get_info", "spaden_get_arrays", "spaden_status_string",
             "spaden_last_error_message", "spaden_version"]
@@ -176,11 +186,16 @@ class Matrix:
             if n == 0 or not p:
                 return torch.empty(0, dtype=tdt[t], device=self.device)
             return torch.as_tensor(_CudaArray(p, (n,), t, self), device=self.device)
-        return {"blk_rowptr": mk(a.blk_rowptr, i.Bnrow + 1, "<i4"),
-                "blk_col": mk(a.blk_col, i.Bnnz, "<i4"),
-                "bitmap": mk(a.bitmap, i.Bnnz, "<i8"),       # uint64 bits viewed as int64
-                "blk_offset": mk(a.blk_offset, i.Bnnz + 1, "<i4"),
-                "values": mk(a.values, i.nnz, vt)}
+        out = {"blk_rowptr": mk(a.blk_rowptr, i.Bnrow + 1, "<i4"),
+               "blk_col": mk(a.blk_col, i.Bnnz, "<i4"),
+               "bitmap": mk(a.bitmap, i.Bnnz, "<i8"),       # uint64 bits viewed as int64
+               "blk_offset": mk(a.blk_offset, i.Bnnz + 1, "<i4"),
+               "values": mk(a.values, i.nnz - i.residual_nnz, vt)}
+        if a.res_rowptr:
+            out["res_rowptr"] = mk(a.res_rowptr, i.m + 1, "<i4")
+            out["res_colidx"] = mk(a.res_colidx, i.residual_nnz, "<i4")
+            out["res_values"] = mk(a.res_values, i.residual_nnz, vt)
+        return out
 
     def spmv(self, x, y=None, alpha: float = 1.0, beta: float = 0.0, stream=None):
         """y = alpha * A x + beta * y on the device (x, y float32 CUDA tensors)."""
@@ -223,8 +238,9 @@ class Matrix:
             pass
 
 
-def convert(rowptr, colidx, values, n: int, storage=None, stream=None) -> Matrix:
-    """CSR (int32 CUDA tensors + fp32/fp16 values) -> bitBSR Matrix."""
+def convert(rowptr, colidx, values, n: int, storage=None, stream=None, residual_max_popc: int = 0) -> Matrix:
+    """CSR (int32 CUDA tensors + fp32/fp16 values) -> bitBSR Matrix (hybrid with a CSR
+    residual for blocks of <= residual_max_popc entries when that is > 0)."""
     torch = _torch()
     assert rowptr.dtype == torch.int32 and colidx.dtype == torch.int32
     assert rowptr.is_cuda and colidx.is_cuda and values.is_cuda
@@ -232,9 +248,10 @@ def convert(rowptr, colidx, values, n: int, storage=None, stream=None) -> Matrix
     sdt = vdt if storage is None else _dtype_code(storage)
     m = rowptr.numel() - 1
     h = ctypes.c_void_p()
-    st = spaden_convert_csr_to_bitmap(m, n, colidx.numel(), ctypes.c_void_p(rowptr.data_ptr()),
-                                      ctypes.c_void_p(colidx.data_ptr()),
-                                      ctypes.c_void_p(values.data_ptr()), vdt, sdt,
-                                      _stream_ptr(stream), ctypes.byref(h))
+    opts = spaden_convert_opts_t(ctypes.sizeof(spaden_convert_opts_t), int(residual_max_popc))
+    st = spaden_convert_csr_to_bitmap_ex(m, n, colidx.numel(), ctypes.c_void_p(rowptr.data_ptr()),
+                                         ctypes.c_void_p(colidx.data_ptr()),
+                                         ctypes.c_void_p(values.data_ptr()), vdt, sdt, ctypes.byref(opts),
+                                         _stream_ptr(stream), ctypes.byref(h))
     _check(st, "spaden_convert_csr_to_bitmap")
     return Matrix(h, rowptr.device)

@@ -45,7 +45,8 @@ static void release(Matrix *A) {
     if (!A) return;
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap,   A->blk_offset, A->values,
                     A->stage_x,     A->stage_y,  A->stage_x2, A->stage_y2,   A->tiles,
-                    A->long_rows,   A->chunk_start, A->chunk_row, A->carry};
+                    A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->res_rowptr,
+                    A->res_colidx,  A->res_values};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (cudaEvent_t e : A->ev)
@@ -95,7 +96,26 @@ spaden_status_t spaden_convert_csr_to_bitmap(int64_t m, int64_t n, int64_t nnz, 
                                              const int32_t *d_colidx, const void *d_values,
                                              spaden_dtype_t values_dtype, spaden_dtype_t storage_dtype,
                                              void *stream, spaden_matrix_t *out) {
+    return spaden_convert_csr_to_bitmap_ex(m, n, nnz, d_rowptr, d_colidx, d_values, values_dtype, storage_dtype,
+                                           nullptr, stream, out);
+}
+
+spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n, int64_t nnz, const int32_t *d_rowptr,
+                                                const int32_t *d_colidx, const void *d_values,
+                                                spaden_dtype_t values_dtype, spaden_dtype_t storage_dtype,
+                                                const spaden_convert_opts_t *opts, void *stream,
+                                                spaden_matrix_t *out) {
     g_last_error.clear();
+    int res_t = 0;
+    if (opts) {
+        if (opts->struct_size != (int32_t)sizeof(spaden_convert_opts_t) || opts->residual_max_popc < 0 ||
+            opts->residual_max_popc > 64) {
+            if (out) *out = nullptr;
+            set_error("bad spaden_convert_opts_t (struct_size or residual_max_popc not in [0, 64])");
+            return SPADEN_ERR_INVALID_ARGUMENT;
+        }
+        res_t = opts->residual_max_popc;
+    }
     if (!out) {
         set_error("out must not be NULL");
         return SPADEN_ERR_INVALID_ARGUMENT;
@@ -132,7 +152,7 @@ spaden_status_t spaden_convert_csr_to_bitmap(int64_t m, int64_t n, int64_t nnz, 
         return SPADEN_ERR_OUT_OF_MEMORY;
     }
     A->device = dev;
-    s = convert_csr(m, n, nnz, d_rowptr, d_colidx, d_values, values_dtype, storage_dtype,
+    s = convert_csr(m, n, nnz, d_rowptr, d_colidx, d_values, values_dtype, storage_dtype, res_t,
                     (cudaStream_t)stream, A);
     if (s != SPADEN_OK) {
         cudaStreamSynchronize((cudaStream_t)stream);
@@ -254,7 +274,10 @@ spaden_status_t spaden_get_info(spaden_matrix_t A, spaden_info_t *info) {
     info->Bnnz = A->Bnnz;
     info->storage_dtype = (int32_t)A->storage;
     info->device = A->device;
-    info->format_bytes = 4 * (A->Bnrow + 1) + 4 * A->Bnnz + 8 * A->Bnnz + 4 * (A->Bnnz + 1) + sv * A->nnz;
+    info->format_bytes = 4 * (A->Bnrow + 1) + 4 * A->Bnnz + 8 * A->Bnnz + 4 * (A->Bnnz + 1) +
+                         sv * (A->nnz - A->res_nnz);
+    if (A->res_max_popc > 0) info->format_bytes += 4 * (A->m + 1) + (4 + sv) * A->res_nnz;
+    info->residual_nnz = A->res_nnz;
     info->aux_bytes = A->aux_bytes;
     info->n_tiles = A->n_tiles;
     info->n_long = A->n_long;
@@ -271,6 +294,9 @@ spaden_status_t spaden_get_arrays(spaden_matrix_t A, spaden_arrays_t *v) {
     v->bitmap = A->bitmap;
     v->blk_offset = A->blk_offset;
     v->values = A->values;
+    v->res_rowptr = A->res_rowptr;
+    v->res_colidx = A->res_colidx;
+    v->res_values = A->res_values;
     return SPADEN_OK;
 }
 

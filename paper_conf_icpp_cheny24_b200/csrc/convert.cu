@@ -303,7 +303,7 @@ void launch_fill(int64_t m, int64_t n, int64_t NBC, const int32_t *rowptr, const
 
 spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *rowptr,
                             const int32_t *colidx, const void *values, spaden_dtype_t vdt,
-                            spaden_dtype_t sdt, cudaStream_t st, Matrix *A) {
+                            spaden_dtype_t sdt, int residual_max_popc, cudaStream_t st, Matrix *A) {
     const int64_t Bnrow = (m + 7) / 8;
     const int64_t NBC = (n + 7) / 8;
     const int64_t max_chunks = Bnrow + nnz / kChunkNnz + 1;
@@ -402,7 +402,12 @@ spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *ro
     k_finalize<<<grid_for(Bnrow + 1, 256), 256, 0, st>>>(Bnrow, Bnnz, nnz, chunk_start, cnt_blk,
                                                          A->blk_rowptr, A->blk_offset);
     SPADEN_CUDA_TRY(cudaGetLastError());
-    // SpMV tile schedule (second and last host sync: tile / long-row counts)
+    // hybrid mode: move low-fill blocks into the CSR residual (one more sync)
+    if (residual_max_popc > 0) {
+        spaden_status_t hs = split_residual(A, residual_max_popc, st);
+        if (hs != SPADEN_OK) return hs;
+    }
+    // SpMV tile schedule (second host sync: tile / long-row counts)
     return build_schedule(A, st);
 }
 

@@ -1,0 +1,233 @@
+// hybrid.cu -- fill-adaptive hybrid format.
+//
+// "bitBSR is expected to be effective for high-degree
+// matrices.  As for low-degree matrices, the utilization of bitmaps may become
+// burdensome, e.g., if one block only contains a single nonzero element."  In
+// hybrid mode the converted bitBSR is split: blocks holding at most t entries
+// become a row-sorted CSR residual (global columns), the rest stay bitBSR.
+// spaden_spmv then runs the bitBSR kernels (y = alpha*A_bit*x + beta*y) followed
+// by a residual pass (y += alpha*A_res*x, one warp per row, fixed lane order and
+// xor tree: deterministic and independent of the row partition).
+//
+// Split = count kernel (per block-row: kept blocks / values, residual entries
+// per row) -> exclusive scans -> one host sync (sizes) -> fill kernel (compacts
+// the kept blocks, appends residual entries row by row in ascending column).
+#include "internal.cuh"
+
+namespace spaden {
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+__device__ __forceinline__ int warp_sum(int v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+    return v;
+}
+
+// one warp per block-row
+__global__ void k_split_count(int64_t m, int64_t Bnrow, int t, const int32_t *__restrict__ brp,
+                              const uint64_t *__restrict__ bitmap, int32_t *__restrict__ res_rowcnt,
+                              int32_t *__restrict__ kept_blk, int32_t *__restrict__ kept_val) {
+    const int64_t br = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (br >= Bnrow) return;
+    const int b0 = brp[br], b1 = brp[br + 1];
+    int cnt[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    int kb = 0, kv = 0;
+    for (int base = b0; base < b1; base += 32) {
+        const int b = base + lane;
+        const uint64_t bm = b < b1 ? bitmap[b] : 0ull;
+        const int pc = __popcll(bm);
+        const bool res = b < b1 && pc <= t;
+        const bool keep = b < b1 && !res;
+        kb += __popc(__ballot_sync(kFull, keep));
+        kv += warp_sum(keep ? pc : 0);
+#pragma unroll
+        for (int r = 0; r < 8; ++r) cnt[r] += warp_sum(res ? __popc((uint32_t)(bm >> (8 * r)) & 0xffu) : 0);
+    }
+#pragma unroll
+    for (int r = 0; r < 8; ++r)
+        if (lane == r && 8 * br + r < m) res_rowcnt[8 * br + r] = cnt[r];
+    if (lane == 0) {
+        kept_blk[br] = kb;
+        kept_val[br] = kv;
+    }
+}
+
+template <typename V>
+__global__ void k_split_fill(int64_t m, int64_t Bnrow, int t, const int32_t *__restrict__ brp,
+                             const int32_t *__restrict__ bcol, const uint64_t *__restrict__ bitmap,
+                             const int32_t *__restrict__ boff, const V *__restrict__ vals,
+                             const int32_t *__restrict__ new_brp, const int32_t *__restrict__ new_vstart,
+                             int32_t *__restrict__ n_col, uint64_t *__restrict__ n_bmp, int32_t *__restrict__ n_off,
+                             V *__restrict__ n_vals, const int32_t *__restrict__ res_rowptr,
+                             int32_t *__restrict__ res_col, V *__restrict__ res_val) {
+    const int64_t br = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (br >= Bnrow) return;
+    const int b0 = brp[br], b1 = brp[br + 1];
+    int nb = new_brp[br], nv = new_vstart[br];
+    int rpos = (lane < 8 && 8 * br + lane < m) ? res_rowptr[8 * br + lane] : 0;  // lane r: next slot of row r
+    for (int base = b0; base < b1; base += 32) {
+        const int b = base + lane;
+        const uint64_t bm = b < b1 ? bitmap[b] : 0ull;
+        const int pc = __popcll(bm);
+        const bool res = b < b1 && pc <= t;
+        const bool keep = b < b1 && !res;
+        const int col = b < b1 ? bcol[b] : 0;
+        const int off = b < b1 ? boff[b] : 0;
+        // kept blocks, compacted in order
+        const unsigned km = __ballot_sync(kFull, keep);
+        int vtot;
+        const int vex = warp_excl_scan_i32(keep ? pc : 0, lane, &vtot);
+        if (keep) {
+            const int idx = nb + __popc(km & ((1u << lane) - 1u));
+            n_col[idx] = col;
+            n_bmp[idx] = bm;
+            n_off[idx] = nv + vex;
+            for (int j = 0; j < pc; ++j) n_vals[nv + vex + j] = vals[off + j];
+        }
+        nb += __popc(km);
+        nv += vtot;
+        // residual entries, row by row: lanes (blocks) in ascending column order
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+            uint32_t byte = res ? ((uint32_t)(bm >> (8 * r)) & 0xffu) : 0u;
+            int rtot;
+            const int rex = warp_excl_scan_i32(__popc(byte), lane, &rtot);
+            const int start = __shfl_sync(kFull, rpos, r) + rex;
+            int q = off + __popcll(bm & ((1ull << (8 * r)) - 1ull));
+            int j = 0;
+            while (byte) {
+                const int c = __ffs(byte) - 1;
+                byte &= byte - 1;
+                res_col[start + j] = 8 * col + c;
+                res_val[start + j] = vals[q + j];
+                ++j;
+            }
+            if (lane == r) rpos += rtot;
+        }
+    }
+    if (br == Bnrow - 1 && lane == 0) n_off[nb] = nv;  // blk_offset[Bnnz'] = kept nnz
+}
+
+__global__ void k_split_summary(const int32_t *a, const int32_t *b, const int32_t *c, int32_t *out) {
+    out[0] = *a;
+    out[1] = *b;
+    out[2] = *c;
+}
+
+// residual CSR: one warp per row, lanes over entries, fixed xor tree
+template <typename V>
+__global__ void __launch_bounds__(256)
+k_residual(int64_t m, const int32_t *__restrict__ rp, const int32_t *__restrict__ col, const V *__restrict__ val,
+           const float *__restrict__ x, float alpha, float *__restrict__ y) {
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    for (int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; row < m; row += nw) {
+        const int k0 = rp[row], k1 = rp[row + 1];
+        if (k0 == k1) continue;
+        float a = 0.f;
+        for (int k = k0 + lane; k < k1; k += 32) {
+            float v;
+            if constexpr (sizeof(V) == 2) v = __half2float(val[k]);
+            else v = val[k];
+            a = fmaf(v, __ldg(x + col[k]), a);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(kFull, a, o);
+        if (lane == 0) y[row] = fmaf(alpha, a, y[row]);
+    }
+}
+
+}  // namespace
+
+spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
+    A->res_max_popc = t;
+    const int64_t m = A->m, Bnrow = A->Bnrow;
+    if (t <= 0 || m == 0) return SPADEN_OK;
+    const size_t sv = A->storage == SPADEN_R_16F ? 2 : 4;
+    const size_t nt = scan_tmp_ints(std::max<int64_t>(m, Bnrow) + 1);
+    int32_t *tmp = nullptr;
+    const size_t ints = (size_t)(m + 1) + 2 * (size_t)(Bnrow + 1) + nt + 4;
+    SPADEN_CUDA_TRY(cudaMallocAsync(&tmp, ints * sizeof(int32_t), st));
+    int32_t *res_cnt = tmp, *kept_blk = tmp + (m + 1), *kept_val = kept_blk + (Bnrow + 1);
+    int32_t *scan_tmp = kept_val + (Bnrow + 1), *summary = scan_tmp + nt;
+    auto fail = [&](cudaError_t e, const char *what) {
+        cudaFreeAsync(tmp, st);
+        return cuda_status(e, what);
+    };
+    const unsigned grid = (unsigned)((32 * Bnrow + 255) / 256);
+    k_split_count<<<grid, 256, 0, st>>>(m, Bnrow, t, A->blk_rowptr, A->bitmap, res_cnt, kept_blk, kept_val);
+    cudaError_t e = exclusive_scan_i32(res_cnt, res_cnt, m, scan_tmp, st);
+    if (e == cudaSuccess) e = exclusive_scan_i32(kept_blk, kept_blk, Bnrow, scan_tmp, st);
+    if (e == cudaSuccess) e = exclusive_scan_i32(kept_val, kept_val, Bnrow, scan_tmp, st);
+    int32_t h[3] = {0, 0, 0};
+    if (e == cudaSuccess) {
+        k_split_summary<<<1, 1, 0, st>>>(res_cnt + m, kept_blk + Bnrow, kept_val + Bnrow, summary);
+        e = cudaMemcpyAsync(h, summary, sizeof(h), cudaMemcpyDeviceToHost, st);
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return fail(e, "hybrid split (count)");
+    const int64_t res_nnz = h[0], nB = h[1], nV = h[2];
+    int32_t *n_col = nullptr, *n_off = nullptr, *r_col = nullptr;
+    uint64_t *n_bmp = nullptr;
+    void *n_vals = nullptr, *r_vals = nullptr;
+    e = cudaMalloc(&n_col, pad16(4 * nB));
+    if (e == cudaSuccess) e = cudaMalloc(&n_bmp, pad16(8 * nB));
+    if (e == cudaSuccess) e = cudaMalloc(&n_off, pad16(4 * (nB + 1)));
+    if (e == cudaSuccess) e = cudaMalloc(&n_vals, pad16(sv * nV));
+    if (e == cudaSuccess) e = cudaMalloc(&A->res_rowptr, pad16(4 * (m + 1)));
+    if (e == cudaSuccess) e = cudaMalloc(&r_col, pad16(4 * res_nnz));
+    if (e == cudaSuccess) e = cudaMalloc(&r_vals, pad16(sv * res_nnz));
+    if (e != cudaSuccess) {
+        for (void *p : {(void *)n_col, (void *)n_bmp, (void *)n_off, n_vals, (void *)r_col, r_vals})
+            if (p) cudaFree(p);
+        return fail(e, "hybrid split (allocation)");
+    }
+    cudaMemsetAsync(n_off, 0, pad16(4 * (nB + 1)), st);
+    e = cudaMemcpyAsync(A->res_rowptr, res_cnt, 4 * (m + 1), cudaMemcpyDeviceToDevice, st);
+    if (A->storage == SPADEN_R_16F)
+        k_split_fill<__half><<<grid, 256, 0, st>>>(m, Bnrow, t, A->blk_rowptr, A->blk_col, A->bitmap, A->blk_offset,
+                                                   (const __half *)A->values, kept_blk, kept_val, n_col, n_bmp, n_off,
+                                                   (__half *)n_vals, A->res_rowptr, r_col, (__half *)r_vals);
+    else
+        k_split_fill<float><<<grid, 256, 0, st>>>(m, Bnrow, t, A->blk_rowptr, A->blk_col, A->bitmap, A->blk_offset,
+                                                  (const float *)A->values, kept_blk, kept_val, n_col, n_bmp, n_off,
+                                                  (float *)n_vals, A->res_rowptr, r_col, (float *)r_vals);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(A->blk_rowptr, kept_blk, 4 * (Bnrow + 1), cudaMemcpyDeviceToDevice, st);
+    if (e == cudaSuccess) e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    cudaFreeAsync(tmp, st);
+    // install the compacted bitBSR (free the old arrays) and the residual
+    cudaFree(A->blk_col);
+    cudaFree(A->bitmap);
+    cudaFree(A->blk_offset);
+    cudaFree(A->values);
+    A->blk_col = n_col;
+    A->bitmap = n_bmp;
+    A->blk_offset = n_off;
+    A->values = n_vals;
+    A->res_colidx = r_col;
+    A->res_values = r_vals;
+    A->Bnnz = nB;
+    A->res_nnz = res_nnz;
+    if (e != cudaSuccess) return cuda_status(e, "hybrid split (fill)");
+    return SPADEN_OK;
+}
+
+cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y, cudaStream_t st) {
+    if (A.res_nnz == 0) return cudaSuccess;
+    const int64_t warps = std::min<int64_t>(A.m, 148LL * 64 * 8);
+    const unsigned grid = (unsigned)((32 * warps + 255) / 256);
+    if (A.storage == SPADEN_R_16F)
+        k_residual<__half><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx, (const __half *)A.res_values, x,
+                                                 alpha, y);
+    else
+        k_residual<float><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx, (const float *)A.res_values, x,
+                                                alpha, y);
+    return cudaGetLastError();
+}
+
+}  // namespace spaden

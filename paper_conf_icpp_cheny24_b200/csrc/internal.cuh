@@ -40,6 +40,13 @@ struct spaden_matrix_s {
     int32_t *chunk_row = nullptr;              // [n_chunks] index into long_rows
     float *carry = nullptr;                    // [n_chunks*8] per-chunk row partials
 
+    // hybrid residual CSR (csrc/hybrid.cu), empty in pure bitBSR mode
+    int64_t res_nnz = 0;
+    int res_max_popc = 0;
+    int32_t *res_rowptr = nullptr;   // [m+1]
+    int32_t *res_colidx = nullptr;   // [res_nnz]
+    void *res_values = nullptr;      // [res_nnz]
+
     // host-API staging buffers (lazily allocated): [2] slots for the batched pipeline
     float *stage_x = nullptr;
     float *stage_y = nullptr;
@@ -118,7 +125,11 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t stream);
 // converter (convert.cu)
 spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *rowptr,
                             const int32_t *colidx, const void *values, spaden_dtype_t vdt,
-                            spaden_dtype_t sdt, cudaStream_t stream, Matrix *A);
+                            spaden_dtype_t sdt, int residual_max_popc, cudaStream_t stream, Matrix *A);
+
+// hybrid split (hybrid.cu): move blocks with popc <= t into a CSR residual
+spaden_status_t split_residual(Matrix *A, int t, cudaStream_t stream);
+cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y, cudaStream_t stream);
 
 // SpMV (spmv.cu)
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,

@@ -781,6 +781,7 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
                                                       A.blk_offset, (const float *)A.values, x, x_vec, alpha,
                                                       beta, y);
         SPADEN_CUDA_TRY(cudaGetLastError());
+        SPADEN_CUDA_TRY(residual_spmv(A, alpha, x, y, st));
         return SPADEN_OK;
     }
     // decode style from the mean block fill (predicated slots for dense-ish blocks)
@@ -802,6 +803,7 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
         e = dec == 0 ? launch_tiled<float, 0>(A, alpha, x, beta, y, st)
                      : (dec == 1 ? launch_tiled<float, 1>(A, alpha, x, beta, y, st)
                                  : launch_tiled<float, 2>(A, alpha, x, beta, y, st));
+    if (e == cudaSuccess) e = residual_spmv(A, alpha, x, y, st);  // hybrid residual (if any)
     if (e != cudaSuccess) return cuda_status(e, "launching k_spmv_tiled");
     return SPADEN_OK;
 }

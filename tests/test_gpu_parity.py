@@ -455,3 +455,59 @@ def test_spmv_host_batched(sp, torch, beta):
     for k in range(K):
         yd = gpu_spmv(torch, M, X[k].numpy(), alpha=1.5, beta=beta, y0=Y0[k])
         assert np.array_equal(Y[k].numpy(), yd)
+
+
+# ------------------------------------------------------------ hybrid (NEXT-1)
+HYB_CASES = {"h1": W.h1, "tiny": lambda: W.tiny(0), "hub": lambda: hub_matrix(),
+             "pl14": lambda: W.powerlaw(14, 5, seed=1), "fem": lambda: W.fem(6, 7, 8, seed=2)}
+
+
+@pytest.mark.parametrize("name", sorted(HYB_CASES))
+@pytest.mark.parametrize("t", [1, 2, 4])
+@pytest.mark.parametrize("storage", ["fp32", "fp16"])
+def test_hybrid_conversion_bit_exact(sp, torch, name, t, storage):
+    A = HYB_CASES[name]()
+    stored = A.values if storage == "fp32" else oracle.f32_to_f16(A.values)
+    rp, ci, v = dev(torch, A)
+    M = sp.convert(rp, ci, v, A.n, storage=storage, residual_max_popc=t)
+    torch.cuda.synchronize()
+    (krp, kci, kv), (rrp, rci, rv) = oracle.hybrid_split(A.m, A.n, A.rowptr, A.colidx, stored, t)
+    st, B = oracle.csr_to_bitbsr(A.m, A.n, krp, kci, kv)
+    h = host_arrays(torch, M)
+    i = M.info
+    ub = np.uint16 if storage == "fp16" else np.uint32
+    assert i.residual_nnz == rci.size and i.Bnnz == B.Bnnz
+    assert np.array_equal(h["blk_rowptr"].astype(np.int64), B.blk_rowptr)
+    assert np.array_equal(h["blk_offset"].astype(np.int64), B.blk_offset)
+    if B.Bnnz:
+        assert np.array_equal(h["blk_col"], B.blk_col)
+        assert np.array_equal(h["bitmap"].view(np.uint64), B.bitmap)
+        assert np.array_equal(h["values"].view(ub), np.ascontiguousarray(B.values).view(ub))
+    assert np.array_equal(h["res_rowptr"].astype(np.int64), rrp)
+    assert np.array_equal(h["res_colidx"], rci)
+    assert np.array_equal(h["res_values"].view(ub), np.ascontiguousarray(rv).view(ub))
+    sv = 2 if storage == "fp16" else 4
+    assert i.format_bytes == oracle.bitbsr_bytes(A.m, B.Bnnz, kci.size, sv) + 4 * (A.m + 1) + (4 + sv) * rci.size
+
+
+@pytest.mark.parametrize("name", sorted(HYB_CASES))
+def test_hybrid_spmv(sp, torch, name):
+    A = HYB_CASES[name]()
+    x = W.vector(A.n, 23)
+    rp, ci, v = dev(torch, A)
+    M = sp.convert(rp, ci, v, A.n, residual_max_popc=2)
+    y1 = gpu_spmv(torch, M, x)
+    assert np.array_equal(y1, gpu_spmv(torch, M, x))
+    check_spmv(A, y1, A.values, x)
+    y0 = W.vector(A.m, 24)
+    y2 = gpu_spmv(torch, M, x, alpha=0.5, beta=2.0, y0=y0)
+    ys, s = oracle.spmv(A.rowptr, A.colidx, A.values, x)
+    assert oracle.componentwise_error(y2, 0.5 * ys + 2.0 * y0, 0.5 * s + 2.0 * np.abs(y0)) <= TOL32
+    if A.m >= 16:   # 8-row-aligned split gives identical y
+        cut = (A.m // 16) * 8
+        parts = []
+        for r0, r1 in ((0, cut), (cut, A.m)):
+            S = A.row_slice(r0, r1)
+            r, c, vv = dev(torch, S)
+            parts.append(gpu_spmv(torch, sp.convert(r, c, vv, S.n, residual_max_popc=2), x))
+        assert np.array_equal(np.concatenate(parts), y1)

@@ -340,3 +340,38 @@ def test_fem62k_invariants():
     assert (d[~starts[1:]] > 0).all()
     fill = A.nnz / B.Bnnz
     assert 18 < fill < 26   # cant: 22.25 (Table 1)
+
+
+# ------------------------------------------------------------ hybrid (NEXT-1)
+def test_hybrid_split_hand_worked():
+    """H1 with t = 2: only block (0,0) (4 entries) stays bitBSR (worked by hand)."""
+    A = W.h1()
+    (krp, kci, kv), (rrp, rci, rv) = oracle.hybrid_split(A.m, A.n, A.rowptr, A.colidx, A.values, 2)
+    st, B = oracle.csr_to_bitbsr(A.m, A.n, krp, kci, kv)
+    assert B.blk_rowptr.tolist() == [0, 1, 1] and B.blk_col.tolist() == [0]
+    assert [int(w) for w in B.bitmap] == [0x8000000080000201]
+    assert B.values.tolist() == [1, 3, 4, 5]
+    assert rrp.tolist() == [0, 1, 1, 1, 1, 1, 1, 1, 2, 2, 3, 3, 3, 4, 4, 4, 5]
+    assert rci.tolist() == [9, 8, 2, 3, 15] and rv.tolist() == [2, 6, 7, -1, 8]
+    # t = 1: only the single-entry block (1,1) -> residual
+    (krp, kci, kv), (rrp, rci, rv) = oracle.hybrid_split(A.m, A.n, A.rowptr, A.colidx, A.values, 1)
+    assert rci.tolist() == [15] and rv.tolist() == [8] and rrp[-1] == 1
+
+
+@pytest.mark.parametrize("t", [1, 2, 5, 64])
+def test_hybrid_split_partitions_entries(t):
+    A = W.random_sparse(300, 250, 0.03, 4)
+    (krp, kci, kv), (rrp, rci, rv) = oracle.hybrid_split(A.m, A.n, A.rowptr, A.colidx, A.values, t)
+    D = dense_of(A)
+    K = dense_of(W.CSR(A.m, A.n, krp.astype(np.int32), kci, kv))
+    R = dense_of(W.CSR(A.m, A.n, rrp.astype(np.int32), rci, rv))
+    assert np.array_equal(K + R, D)
+    assert not ((K != 0) & (R != 0)).any()
+    st, B = oracle.csr_to_bitbsr(A.m, A.n, krp, kci, kv)
+    pc = np.array([bin(int(w)).count("1") for w in B.bitmap])
+    assert (pc > t).all()
+    x = W.vector(A.n, 1)
+    y, _ = oracle.spmv(A.rowptr, A.colidx, A.values, x)
+    yk, _ = oracle.spmv(krp, kci, kv, x)
+    yr, _ = oracle.spmv(rrp, rci, rv, x)
+    np.testing.assert_allclose(yk + yr, y, rtol=1e-12, atol=1e-12)
