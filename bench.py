@@ -51,6 +51,8 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-cusparse", action="store_true")
     p.add_argument("--no-variants", action="store_true", help="skip the other-precision kernel timing")
+    p.add_argument("--hybrid", type=int, default=0,
+                   help="hybrid format: blocks with <= HYBRID entries go to a CSR residual (0 = pure bitBSR)")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     return p.parse_args()
 
@@ -64,10 +66,15 @@ def peaks():
         return 6650.0, "fallback"
 
 
-def alg_bytes(m, n, nnz, Bnrow, Bnnz, sv, beta_nonzero=False):
+def alg_bytes(m, n, nnz, Bnrow, Bnnz, sv, beta_nonzero=False, res_nnz=0):
     """Algorithmic bytes of one SpMV: the bitBSR arrays once
-    (blk_rowptr, blk_col, bitmap, blk_offset, values), x once, y written once."""
-    return 4 * (Bnrow + 1) + (4 + 8 + 4) * Bnnz + sv * nnz + 4 * n + 4 * m + (4 * m if beta_nonzero else 0)
+    (blk_rowptr, blk_col, bitmap, blk_offset, values), x once, y written once;
+    in hybrid mode also the residual CSR (rowptr, colidx, values) and y re-read
+    and re-written by the residual pass."""
+    b = 4 * (Bnrow + 1) + (4 + 8 + 4) * Bnnz + sv * (nnz - res_nnz) + 4 * n + 4 * m + (4 * m if beta_nonzero else 0)
+    if res_nnz:
+        b += 4 * (m + 1) + (4 + sv) * res_nnz + 8 * m
+    return b
 
 
 class Clocks:
@@ -255,7 +262,7 @@ def main():
     stream = torch.cuda.current_stream(dev)
     torch.cuda.synchronize(dev)
     t0 = time.perf_counter()
-    M = sp.convert(*wl.local, wl.n, storage=args.dtype)
+    M = sp.convert(*wl.local, wl.n, storage=args.dtype, residual_max_popc=args.hybrid)
     torch.cuda.synchronize(dev)
     convert_s = time.perf_counter() - t0
     info = M.info
@@ -304,7 +311,8 @@ def main():
 
     # ---- roofline of the dominant kernel (the SpMV) on this rank
     kavg_ms = float(np.mean(kernel_ms))
-    abytes = alg_bytes(wl.r1 - wl.r0, wl.n, wl.local_nnz, info.Bnrow, info.Bnnz, sv, beta_nonzero=wl.c is not None)
+    abytes = alg_bytes(wl.r1 - wl.r0, wl.n, wl.local_nnz, info.Bnrow, info.Bnnz, sv, beta_nonzero=wl.c is not None,
+                       res_nnz=info.residual_nnz)
     peak, peak_kind = peaks()
     achieved = abytes / (kavg_ms * 1e-3) / 1e9
     traffic = None
@@ -388,7 +396,7 @@ def main():
         variants = {}
         if world == 1 and not args.no_variants:
             other = "fp16" if args.dtype == "fp32" else "fp32"
-            M2 = sp.convert(*local_csr, wl.n, storage=other)
+            M2 = sp.convert(*local_csr, wl.n, storage=other, residual_max_popc=args.hybrid)
             i2 = M2.info
             ys = torch.empty(wl.m, dtype=torch.float32, device=dev)
             for _ in range(5):
@@ -403,7 +411,8 @@ def main():
             v1e.record(stream)
             torch.cuda.synchronize(dev)
             vms = v0e.elapsed_time(v1e) / reps
-            vb = alg_bytes(wl.m, wl.n, wl.local_nnz, i2.Bnrow, i2.Bnnz, 2 if other == "fp16" else 4)
+            vb = alg_bytes(wl.m, wl.n, wl.local_nnz, i2.Bnrow, i2.Bnnz, 2 if other == "fp16" else 4,
+                           res_nnz=i2.residual_nnz)
             variants[other] = {"kernel_ms": vms, "gflops": 2.0 * wl.nnz / (vms * 1e-3) / 1e9,
                                "hbm_gbs": vb / (vms * 1e-3) / 1e9, "frac": vb / (vms * 1e-3) / 1e9 / peak,
                                "bytes_per_nnz_stored": i2.format_bytes / max(1, i2.nnz),
@@ -412,7 +421,8 @@ def main():
             M2.free()
             del ys
 
-        n_launch = 1 + (2 if info.n_long > 0 else 0)  # tiled kernel [+ long-row chunks and fix-up]
+        # tiled kernel [+ long-row chunks and fix-up] [+ hybrid residual pass]
+        n_launch = 1 + (2 if info.n_long > 0 else 0) + (1 if info.residual_nnz > 0 else 0)
         line = {
             "metric": METRIC, "value": gflops, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": max(3, args.warmup), "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -421,7 +431,8 @@ def main():
             "config": {"workload": args.workload, "m": wl.m, "n": wl.n, "nnz": wl.nnz,
                        "Bnrow": int((wl.m + 7) // 8), "Bnnz_rank0": int(info.Bnnz),
                        "fill_rank0": wl.local_nnz / max(1, info.Bnnz),
-                       "values": args.dtype,
+                       "values": args.dtype, "hybrid_residual_max_popc": args.hybrid,
+                       "residual_nnz_rank0": int(info.residual_nnz),
                        "parallelism": f"row-partition x{world}" + (" + NCCL all-gather" if world > 1 else ""),
                        "l2": "inputs larger than L2 (A > 126 MB), no flush" if info.format_bytes > 126e6
                              else "matrix fits L2 (no flush): warm-L2 number",

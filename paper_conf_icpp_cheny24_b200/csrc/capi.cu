@@ -46,7 +46,8 @@ static void release(Matrix *A) {
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap,   A->blk_offset, A->values,
                     A->stage_x,     A->stage_y,  A->stage_x2, A->stage_y2,   A->tiles,
                     A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->res_rowptr,
-                    A->res_colidx,  A->res_values};
+                    A->res_colidx,  A->res_values, A->res_long_rows, A->res_chunk_start,
+                    A->res_chunk_row, A->res_carry};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (cudaEvent_t e : A->ev)

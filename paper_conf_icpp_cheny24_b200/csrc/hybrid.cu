@@ -6,8 +6,8 @@
 // hybrid mode the converted bitBSR is split: blocks holding at most t entries
 // become a row-sorted CSR residual (global columns), the rest stay bitBSR.
 // spaden_spmv then runs the bitBSR kernels (y = alpha*A_bit*x + beta*y) followed
-// by a residual pass (y += alpha*A_res*x, one warp per row, fixed lane order and
-// xor tree: deterministic and independent of the row partition).
+// by a residual pass (y += alpha*A_res*x, 8 lanes per row, fixed chunked order
+// and xor tree: deterministic and independent of the row partition).
 //
 // Split = count kernel (per block-row: kept blocks / values, residual entries
 // per row) -> exclusive scans -> one host sync (sizes) -> fill kernel (compacts
@@ -118,27 +118,128 @@ __global__ void k_split_summary(const int32_t *a, const int32_t *b, const int32_
     out[2] = *c;
 }
 
-// residual CSR: one warp per row, lanes over entries, fixed xor tree
+// residual CSR: 8 lanes per row (4 rows per warp).  Fixed per-row order: the
+// row is cut into kResChunk-entry chunks; in a chunk lane l sums entries l,
+// l+8, ... sequentially, a 3-level xor tree combines the 8 lanes, and chunk sums
+// are added in order -- a function of the row alone (partition invariant).
+// Rows longer than kResLongRow are skipped here: their chunks run in parallel
+// (k_res_chunks) and k_res_fixup adds the chunk sums in the same order.
+template <typename V>
+__device__ __forceinline__ float res_chunk_sum(int c0, int c1, int sub, unsigned gmask,
+                                               const int32_t *__restrict__ col, const V *__restrict__ val,
+                                               const float *__restrict__ x) {
+    float a = 0.f;
+#pragma unroll 4
+    for (int k = c0 + sub; k < c1; k += 8) {
+        float v;
+        if constexpr (sizeof(V) == 2) v = __half2float(val[k]);
+        else v = __ldg(val + k);
+        a = fmaf(v, __ldg(x + __ldg(col + k)), a);
+    }
+#pragma unroll
+    for (int o = 4; o > 0; o >>= 1) a += __shfl_xor_sync(gmask, a, o);
+    return a;
+}
+
 template <typename V>
 __global__ void __launch_bounds__(256)
 k_residual(int64_t m, const int32_t *__restrict__ rp, const int32_t *__restrict__ col, const V *__restrict__ val,
            const float *__restrict__ x, float alpha, float *__restrict__ y) {
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int lane = threadIdx.x & 31;
-    for (int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; row < m; row += nw) {
-        const int k0 = rp[row], k1 = rp[row + 1];
-        if (k0 == k1) continue;
-        float a = 0.f;
-        for (int k = k0 + lane; k < k1; k += 32) {
-            float v;
-            if constexpr (sizeof(V) == 2) v = __half2float(val[k]);
-            else v = val[k];
-            a = fmaf(v, __ldg(x + col[k]), a);
-        }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(kFull, a, o);
-        if (lane == 0) y[row] = fmaf(alpha, a, y[row]);
+    const int64_t ngroups = ((int64_t)gridDim.x * blockDim.x) / 8;
+    const int sub = threadIdx.x & 7;
+    const unsigned gmask = 0xffu << (threadIdx.x & 24);  // this row's 8 lanes
+    for (int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 8; row < m; row += ngroups) {
+        const int k0 = __ldg(rp + row), k1 = __ldg(rp + row + 1);
+        if (k0 == k1 || k1 - k0 > kResLongRow) continue;  // uniform within the 8-lane group
+        float sum = 0.f;
+        for (int c0 = k0; c0 < k1; c0 += kResChunk) sum += res_chunk_sum<V>(c0, min(k1, c0 + kResChunk), sub, gmask, col, val, x);
+        if (sub == 0) y[row] = fmaf(alpha, sum, y[row]);
     }
+}
+
+template <typename V>
+__global__ void __launch_bounds__(256)
+k_res_chunks(int64_t nchunks, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
+             const int32_t *__restrict__ chunk_row, const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
+             const V *__restrict__ val, const float *__restrict__ x, float *__restrict__ carry) {
+    const int64_t g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 8;
+    const int sub = threadIdx.x & 7;
+    const unsigned gmask = 0xffu << (threadIdx.x & 24);
+    if (g >= nchunks) return;  // uniform within the group
+    const int j = chunk_row[g];
+    const int row = long_rows[j];
+    const int k1 = rp[row + 1];
+    const int c0 = rp[row] + (int)(g - chunk_start[j]) * kResChunk;
+    const float a = res_chunk_sum<V>(c0, min(k1, c0 + kResChunk), sub, gmask, col, val, x);
+    if (sub == 0) carry[g] = a;
+}
+
+__global__ void k_res_fixup(int64_t nlong, const int32_t *__restrict__ long_rows,
+                            const int32_t *__restrict__ chunk_start, const float *__restrict__ carry, float alpha,
+                            float *__restrict__ y) {
+    const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (j >= nlong) return;
+    float sum = 0.f;
+    for (int c = chunk_start[j]; c < chunk_start[j + 1]; ++c) sum += carry[c];
+    const int row = long_rows[j];
+    y[row] = fmaf(alpha, sum, y[row]);
+}
+
+// long residual rows: flag -> scan -> list; chunk counts -> scan -> chunk owners
+__global__ void k_res_long_flag(int64_t m, const int32_t *__restrict__ rp, int32_t *__restrict__ flag) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < m) flag[i] = (rp[i + 1] - rp[i]) > kResLongRow ? 1 : 0;
+}
+__global__ void k_res_long_list(int64_t m, const int32_t *__restrict__ rp, const int32_t *__restrict__ pos,
+                                int32_t *__restrict__ long_rows, int32_t *__restrict__ nch) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < m && pos[i + 1] != pos[i]) {
+        long_rows[pos[i]] = (int32_t)i;
+        nch[pos[i]] = (rp[i + 1] - rp[i] + kResChunk - 1) / kResChunk;
+    }
+}
+__global__ void k_res_chunk_rows(int64_t nlong, const int32_t *__restrict__ cs, int32_t *__restrict__ crow) {
+    const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (j < nlong)
+        for (int c = cs[j]; c < cs[j + 1]; ++c) crow[c] = (int32_t)j;
+}
+
+spaden_status_t residual_long_rows(Matrix *A, cudaStream_t st) {
+    const int64_t m = A->m;
+    const size_t nt = scan_tmp_ints(m + 1);
+    int32_t *tmp = nullptr;
+    SPADEN_CUDA_TRY(cudaMallocAsync(&tmp, ((size_t)m + 1 + nt + 4) * sizeof(int32_t), st));
+    int32_t *flag = tmp, *scan_tmp = tmp + (m + 1);
+    const unsigned g = (unsigned)((m + 255) / 256);
+    k_res_long_flag<<<g, 256, 0, st>>>(m, A->res_rowptr, flag);
+    cudaError_t e = exclusive_scan_i32(flag, flag, m, scan_tmp, st);
+    int32_t nl = 0;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&nl, flag + m, 4, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e == cudaSuccess && nl > 0) {
+        A->res_n_long = nl;
+        e = cudaMalloc(&A->res_long_rows, 4 * (size_t)nl);
+        if (e == cudaSuccess) e = cudaMalloc(&A->res_chunk_start, 4 * ((size_t)nl + 1));
+        if (e == cudaSuccess) {
+            k_res_long_list<<<g, 256, 0, st>>>(m, A->res_rowptr, flag, A->res_long_rows, A->res_chunk_start);
+            e = exclusive_scan_i32(A->res_chunk_start, A->res_chunk_start, nl, scan_tmp, st);
+        }
+        int32_t nc = 0;
+        if (e == cudaSuccess) e = cudaMemcpyAsync(&nc, A->res_chunk_start + nl, 4, cudaMemcpyDeviceToHost, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        if (e == cudaSuccess) {
+            A->res_n_chunks = nc;
+            e = cudaMalloc(&A->res_chunk_row, 4 * (size_t)std::max(1, nc));
+        }
+        if (e == cudaSuccess) e = cudaMalloc(&A->res_carry, 4 * (size_t)std::max(1, nc));
+        if (e == cudaSuccess) {
+            k_res_chunk_rows<<<(unsigned)((nl + 255) / 256), 256, 0, st>>>(nl, A->res_chunk_start, A->res_chunk_row);
+            e = cudaGetLastError();
+        }
+    }
+    cudaFreeAsync(tmp, st);
+    if (e != cudaSuccess) return cuda_status(e, "hybrid residual long rows");
+    return SPADEN_OK;
 }
 
 }  // namespace
@@ -214,19 +315,32 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
     A->Bnnz = nB;
     A->res_nnz = res_nnz;
     if (e != cudaSuccess) return cuda_status(e, "hybrid split (fill)");
-    return SPADEN_OK;
+    return residual_long_rows(A, st);
 }
 
 cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y, cudaStream_t st) {
     if (A.res_nnz == 0) return cudaSuccess;
-    const int64_t warps = std::min<int64_t>(A.m, 148LL * 64 * 8);
-    const unsigned grid = (unsigned)((32 * warps + 255) / 256);
+    const int64_t groups = std::min<int64_t>(A.m, 148LL * 64 * 32);  // 8 lanes per row
+    const unsigned grid = (unsigned)((8 * groups + 255) / 256);
     if (A.storage == SPADEN_R_16F)
         k_residual<__half><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx, (const __half *)A.res_values, x,
                                                  alpha, y);
     else
         k_residual<float><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx, (const float *)A.res_values, x,
                                                 alpha, y);
+    if (A.res_n_long > 0) {
+        const unsigned gc = (unsigned)((8 * A.res_n_chunks + 255) / 256);
+        if (A.storage == SPADEN_R_16F)
+            k_res_chunks<__half><<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start,
+                                                     A.res_chunk_row, A.res_rowptr, A.res_colidx,
+                                                     (const __half *)A.res_values, x, A.res_carry);
+        else
+            k_res_chunks<float><<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start,
+                                                    A.res_chunk_row, A.res_rowptr, A.res_colidx,
+                                                    (const float *)A.res_values, x, A.res_carry);
+        k_res_fixup<<<(unsigned)((A.res_n_long + 255) / 256), 256, 0, st>>>(A.res_n_long, A.res_long_rows,
+                                                                            A.res_chunk_start, A.res_carry, alpha, y);
+    }
     return cudaGetLastError();
 }
 

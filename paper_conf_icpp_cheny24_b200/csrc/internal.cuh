@@ -46,6 +46,12 @@ struct spaden_matrix_s {
     int32_t *res_rowptr = nullptr;   // [m+1]
     int32_t *res_colidx = nullptr;   // [res_nnz]
     void *res_values = nullptr;      // [res_nnz]
+    int64_t res_n_long = 0;          // residual rows longer than kResLongRow (chunked)
+    int64_t res_n_chunks = 0;
+    int32_t *res_long_rows = nullptr;    // [res_n_long]
+    int32_t *res_chunk_start = nullptr;  // [res_n_long+1]
+    int32_t *res_chunk_row = nullptr;    // [res_n_chunks] index into res_long_rows
+    float *res_carry = nullptr;          // [res_n_chunks]
 
     // host-API staging buffers (lazily allocated): [2] slots for the batched pipeline
     float *stage_x = nullptr;
@@ -112,6 +118,10 @@ constexpr int kBlockStageBytes = 16 + 36;
 // long block-rows are split into chunks of this many blocks (relative to the
 // block-row start, so the split depends only on the row itself)
 constexpr int kLongChunk = 1024;
+// hybrid residual rows: fixed 1024-entry chunks; rows above kResLongRow entries
+// have their chunks processed in parallel (carry + ordered fix-up)
+constexpr int kResChunk = 1024;
+constexpr int kResLongRow = 4096;
 // mean nonzeros per block from which the predicated-slot decode is used
 constexpr int kSlotsMinFill = 8;
 // decode used above that fill (1 = lane per block, 2 = lane per block row)
