@@ -307,6 +307,101 @@ __device__ __forceinline__ void reduce_tile(uint32_t a_rp, uint32_t a_part, int 
     }
 }
 
+__device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
+    unsigned short h;
+    asm("ld.shared.u16 %0, [%1];" : "=h"(h) : "r"(a));
+    return h;
+}
+
+__device__ __forceinline__ uint32_t pack_f16x2(float lo, float hi) {
+    uint32_t r;
+    asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+    return r;
+}
+
+__device__ __forceinline__ float2 unpack_f16x2(uint32_t v) {
+    return __half22float2(*reinterpret_cast<__half2 *>(&v));
+}
+
+__device__ __forceinline__ void mma16816(float d[4], const uint32_t a[4], uint32_t b0, uint32_t b1) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+
+// One 32-block unit through tensor cores (fp16 values): 8 MMAs of 4 blocks.
+__device__ __forceinline__ void mma_unit(int lb0, int nb, int lane, uint32_t a_bmp, uint32_t a_col, uint32_t a_off,
+                                         uint32_t a_val, int v0, uint32_t a_part, const float *__restrict__ x,
+                                         int nbc_vec) {
+    const int g = lane >> 2, t = lane & 3;
+    const uint32_t mlo = lane < 16 ? (1u << (2 * lane)) - 1u : 0xffffffffu;
+    const uint32_t mhi = lane < 16 ? 0u : (1u << (2 * lane - 32)) - 1u;
+    const int sh = (2 * lane) & 31;
+#pragma unroll 1
+    for (int q = 0; q < 8; ++q) {
+        uint32_t a[4];
+        // fragment register order: {TL, BL, TR, BR} = blocks {P, R, Q, S} = {4q, 4q+2, 4q+1, 4q+3}
+        const int order[4] = {0, 2, 1, 3};
+#pragma unroll
+        for (int f = 0; f < 4; ++f) {
+            const int lb = lb0 + 4 * q + order[f];
+            uint32_t reg = 0u;
+            if (lb < nb) {
+                const uint2 bm = lds_u2(a_bmp + 8u * lb);
+                const uint32_t two = ((lane < 16 ? bm.x : bm.y) >> sh) & 3u;
+                if (two) {
+                    const int rank = __popc(bm.x & mlo) + __popc(bm.y & mhi);
+                    const uint32_t p = a_val + 2u * (uint32_t)(lds_i32(a_off + 4u * lb) - v0 + rank);
+                    const uint32_t h0 = (two & 1u) ? lds_u16(p) : 0u;
+                    const uint32_t h1 = (two & 2u) ? lds_u16(p + 2u * (two & 1u)) : 0u;
+                    reg = h0 | (h1 << 16);
+                }
+            }
+            a[f] = reg;
+        }
+        // B: column g (< 4) holds block (4q+g)'s x segment in its k-half
+        uint32_t bh0 = 0u, bh1 = 0u, bl0 = 0u, bl1 = 0u;
+        const int lbx = lb0 + 4 * q + g;
+        if (g < 4 && lbx < nb) {
+            const int bc = lds_i32(a_col + 4u * lbx);
+            const float *xp = x + 8 * (int64_t)bc + 2 * t;
+            const uint2 bm = lds_u2(a_bmp + 8u * lbx);
+            const uint32_t cols = used_cols(bm);
+            float x0 = 0.f, x1 = 0.f;
+            if (bc < nbc_vec) {
+                const float2 v = __ldg(reinterpret_cast<const float2 *>(xp));
+                x0 = v.x;
+                x1 = v.y;
+            } else {
+                if ((cols >> (2 * t)) & 1u) x0 = __ldg(xp);
+                if ((cols >> (2 * t + 1)) & 1u) x1 = __ldg(xp + 1);
+            }
+            const uint32_t hi = pack_f16x2(x0, x1);
+            const float2 hf = unpack_f16x2(hi);
+            const uint32_t lo = pack_f16x2(x0 - hf.x, x1 - hf.y);
+            if (g & 1) {
+                bh1 = hi;
+                bl1 = lo;
+            } else {
+                bh0 = hi;
+                bl0 = lo;
+            }
+        }
+        float d[4] = {0.f, 0.f, 0.f, 0.f};
+        mma16816(d, a, bh0, bh1);
+        mma16816(d, a, bl0, bl1);
+        // P row g = C[g][0], Q row g = C[g][1] (t = 0); R row g = C[g+8][2], S = C[g+8][3] (t = 1)
+        if (t < 2) {
+            const int lbA = lb0 + 4 * q + 2 * t, lbB = lbA + 1;
+            const float vA = t == 0 ? d[0] : d[2], vB = t == 0 ? d[1] : d[3];
+            if (lbA < nb) sts_f32(a_part + kPartStride * lbA + 4u * g, vA);
+            if (lbB < nb) sts_f32(a_part + kPartStride * lbB + 4u * g, vB);
+        }
+    }
+}
+
 struct alignas(16) StageHdr {
     int br0, nbr, b0, v0;                      // tile
     int nb, units, u_next, done;               // blocks, 32-block units, next unit to grab, units done
@@ -412,7 +507,14 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             ul = __shfl_sync(kFull, ul, 0);
             if (ul >= units) break;
             ++mine;
-            if constexpr (DEC == 2) {
+            if constexpr (DEC == 4) {
+                // tensor-core ablation (SURVEY.md §8(f) NEXT-3, fp16 values): the
+                // paper's fragment trick on mma.sync.m16n8k16 -- four
+                // blocks per MMA, block P/Q/R/S in the TL/TR/BL/BR quadrants, lane l
+                // owns bits 2l, 2l+1 of each (Alg. 2 mapping); x split
+                // into fp16 hi + lo parts (two MMAs) to keep ~22 bits of x.
+                mma_unit(ul * 32, nb, lane, a_bmp, a_col, a_off, a_val, v0, a_part, x, nbc_vec);
+            } else if constexpr (DEC == 2) {
                 const int g = lane >> 3, r = lane & 7;
                 const uint32_t mlo = r == 0 ? 0u : (r < 4 ? (1u << (8 * r)) - 1u : 0xffffffffu);
                 const uint32_t mhi = r <= 4 ? 0u : (1u << (8 * (r - 4))) - 1u;
@@ -785,11 +887,12 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
         return SPADEN_OK;
     }
     // decode style from the mean block fill (predicated slots for dense-ish blocks)
-    static const int decode_env = [] {  // SPADEN_DECODE=bits|slots|rows overrides (ablation)
+    const int decode_env = [] {  // SPADEN_DECODE=bits|slots|rows|mma overrides (ablation), read per call
         const char *e = getenv("SPADEN_DECODE");
         if (e && e[0] == 'b') return 0;
         if (e && e[0] == 's') return 1;
         if (e && e[0] == 'r') return 2;
+        if (e && e[0] == 'm') return 4;
         return -1;
     }();
     const int dec = decode_env >= 0 ? decode_env
@@ -797,12 +900,13 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
     cudaError_t e;
     if (A.storage == SPADEN_R_16F)
         e = dec == 0 ? launch_tiled<__half, 0>(A, alpha, x, beta, y, st)
-                     : (dec == 1 ? launch_tiled<__half, 1>(A, alpha, x, beta, y, st)
-                                 : launch_tiled<__half, 2>(A, alpha, x, beta, y, st));
-    else
+                     : dec == 2 ? launch_tiled<__half, 2>(A, alpha, x, beta, y, st)
+                                : dec == 4 ? launch_tiled<__half, 4>(A, alpha, x, beta, y, st)
+                                           : launch_tiled<__half, 1>(A, alpha, x, beta, y, st);
+    else  // (the tensor-core ablation exists for fp16 values only)
         e = dec == 0 ? launch_tiled<float, 0>(A, alpha, x, beta, y, st)
-                     : (dec == 1 ? launch_tiled<float, 1>(A, alpha, x, beta, y, st)
-                                 : launch_tiled<float, 2>(A, alpha, x, beta, y, st));
+                     : (dec == 2 ? launch_tiled<float, 2>(A, alpha, x, beta, y, st)
+                                 : launch_tiled<float, 1>(A, alpha, x, beta, y, st));
     if (e == cudaSuccess) e = residual_spmv(A, alpha, x, y, st);  // hybrid residual (if any)
     if (e != cudaSuccess) return cuda_status(e, "launching k_spmv_tiled");
     return SPADEN_OK;

@@ -511,3 +511,16 @@ def test_hybrid_spmv(sp, torch, name):
             r, c, vv = dev(torch, S)
             parts.append(gpu_spmv(torch, sp.convert(r, c, vv, S.n, residual_max_popc=2), x))
         assert np.array_equal(np.concatenate(parts), y1)
+
+
+@pytest.mark.parametrize("decode", ["slots", "bits", "rows", "mma"])
+@pytest.mark.parametrize("name", ["fem62k_small", "hub", "tiny", "h2"])
+def test_decode_ablations_fp16(sp, torch, decode, name, monkeypatch):
+    """Every decode variant (SPADEN_DECODE) on fp16 storage, including the
+    tensor-core ablation (mma.sync m16n8k16, x split into fp16 hi+lo)."""
+    A = W.fem(9, 9, 10, seed=4) if name == "fem62k_small" else CASES[name]()
+    monkeypatch.setenv("SPADEN_DECODE", decode)
+    M = convert(sp, torch, A, storage="fp16")
+    x = W.vector(A.n, 29)
+    y = gpu_spmv(torch, M, x)
+    check_spmv(A, y, oracle.f32_to_f16(A.values), x)
