@@ -44,7 +44,8 @@ static spaden_status_t check_device_ptr(const void *p, const char *name, int dev
 static void release(Matrix *A) {
     if (!A) return;
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap,   A->blk_offset, A->values,
-                    A->stage_x,     A->stage_y,  A->stage_x2, A->stage_y2,   A->tiles,
+                    A->stage_x,     A->stage_y,  A->pipe_x[0], A->pipe_x[1], A->pipe_x[2],
+                    A->pipe_y[0],   A->pipe_y[1], A->pipe_y[2], A->tiles,
                     A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->res_rowptr,
                     A->res_colidx,  A->res_values, A->res_long_rows, A->res_chunk_start,
                     A->res_chunk_row, A->res_carry};
@@ -60,10 +61,10 @@ static void release(Matrix *A) {
 // lazily create the batched host pipeline resources
 static spaden_status_t ensure_pipeline(Matrix *A) {
     if (A->s_h2d) return SPADEN_OK;
-    if (!A->stage_x && A->n > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->stage_x, pad16(4 * A->n)));
-    if (!A->stage_y && A->m > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->stage_y, pad16(4 * A->m)));
-    if (A->n > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->stage_x2, pad16(4 * A->n)));
-    if (A->m > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->stage_y2, pad16(4 * A->m)));
+    for (int j = 0; j < 3; ++j) {
+        if (A->n > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->pipe_x[j], pad16(4 * A->n)));
+        if (A->m > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->pipe_y[j], pad16(4 * A->m)));
+    }
     for (cudaEvent_t &e : A->ev) SPADEN_CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     SPADEN_CUDA_TRY(cudaStreamCreateWithFlags(&A->s_d2h, cudaStreamNonBlocking));
     SPADEN_CUDA_TRY(cudaStreamCreateWithFlags(&A->s_h2d, cudaStreamNonBlocking));
@@ -217,34 +218,34 @@ spaden_status_t spaden_spmv_host_batched(spaden_matrix_t A, float alpha, const f
     spaden_status_t s = ensure_pipeline(A);
     if (s != SPADEN_OK) return s;
     cudaStream_t cs = (cudaStream_t)stream;
-    float *dx[2] = {A->stage_x, A->stage_x2}, *dy[2] = {A->stage_y, A->stage_y2};
-    cudaEvent_t *in_ready = A->ev, *computed = A->ev + 2, *drained = A->ev + 4;
-    // slot k&1: H2D(x_k[, y_k]) on s_h2d -> SpMV on cs -> D2H(y_k) on s_d2h.  The
-    // H2D into a slot waits until the SpMV of vector k-2 consumed x and its y
-    // left the device.
-    SPADEN_CUDA_TRY(cudaEventRecord(A->ev[6], cs));
-    SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_h2d, A->ev[6], 0));
-    SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_d2h, A->ev[6], 0));
+    cudaEvent_t *in_ready = A->ev, *computed = A->ev + 3, *drained = A->ev + 6;
+    // slot k%3: H2D(x_k[, y_k]) on s_h2d -> SpMV on cs -> D2H(y_k) on s_d2h.  A
+    // slot is refilled only after the SpMV of vector k-3 consumed it and its y
+    // left the device, so H2D(k+1), SpMV(k) and D2H(k-1) run concurrently.
+    SPADEN_CUDA_TRY(cudaEventRecord(A->ev[9], cs));
+    SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_h2d, A->ev[9], 0));
+    SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_d2h, A->ev[9], 0));
     for (int64_t k = 0; k < nvec; ++k) {
-        const int j = (int)(k & 1);
-        if (k >= 2) SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_h2d, drained[j], 0));
+        const int j = (int)(k % 3);
+        float *dx = A->pipe_x[j], *dy = A->pipe_y[j];
+        if (k >= 3) SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_h2d, drained[j], 0));
         if (A->n > 0)
-            SPADEN_CUDA_TRY(cudaMemcpyAsync(dx[j], h_x + k * ldx, 4 * A->n, cudaMemcpyHostToDevice, A->s_h2d));
+            SPADEN_CUDA_TRY(cudaMemcpyAsync(dx, h_x + k * ldx, 4 * A->n, cudaMemcpyHostToDevice, A->s_h2d));
         if (beta != 0.f && A->m > 0)
-            SPADEN_CUDA_TRY(cudaMemcpyAsync(dy[j], h_y + k * ldy, 4 * A->m, cudaMemcpyHostToDevice, A->s_h2d));
+            SPADEN_CUDA_TRY(cudaMemcpyAsync(dy, h_y + k * ldy, 4 * A->m, cudaMemcpyHostToDevice, A->s_h2d));
         SPADEN_CUDA_TRY(cudaEventRecord(in_ready[j], A->s_h2d));
         SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, in_ready[j], 0));
-        if (k >= 2 && beta == 0.f) SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, drained[j], 0));
-        s = spmv_launch(*A, alpha, dx[j], beta, dy[j], cs);
+        if (k >= 3 && beta == 0.f) SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, drained[j], 0));
+        s = spmv_launch(*A, alpha, dx, beta, dy, cs);
         if (s != SPADEN_OK) return s;
         SPADEN_CUDA_TRY(cudaEventRecord(computed[j], cs));
         SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_d2h, computed[j], 0));
         if (A->m > 0)
-            SPADEN_CUDA_TRY(cudaMemcpyAsync(h_y + k * ldy, dy[j], 4 * A->m, cudaMemcpyDeviceToHost, A->s_d2h));
+            SPADEN_CUDA_TRY(cudaMemcpyAsync(h_y + k * ldy, dy, 4 * A->m, cudaMemcpyDeviceToHost, A->s_d2h));
         SPADEN_CUDA_TRY(cudaEventRecord(drained[j], A->s_d2h));
     }
-    SPADEN_CUDA_TRY(cudaEventRecord(A->ev[7], A->s_d2h));
-    SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, A->ev[7], 0));
+    SPADEN_CUDA_TRY(cudaEventRecord(A->ev[10], A->s_d2h));
+    SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, A->ev[10], 0));
     SPADEN_CUDA_TRY(cudaStreamSynchronize(cs));
     return SPADEN_OK;
 }

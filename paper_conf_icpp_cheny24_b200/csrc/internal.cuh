@@ -54,12 +54,12 @@ struct spaden_matrix_s {
     float *res_carry = nullptr;          // [res_n_chunks]
 
     // host-API staging buffers (lazily allocated): [2] slots for the batched pipeline
-    float *stage_x = nullptr;
+    float *stage_x = nullptr;          // spaden_spmv_host
     float *stage_y = nullptr;
-    float *stage_x2 = nullptr;
-    float *stage_y2 = nullptr;
+    float *pipe_x[3] = {};             // spaden_spmv_host_batched: triple-buffered slots
+    float *pipe_y[3] = {};
     cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
-    cudaEvent_t ev[8] = {};
+    cudaEvent_t ev[11] = {};
 };
 
 namespace spaden {
