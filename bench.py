@@ -441,7 +441,7 @@ def main():
             "bytes_per_nnz": {"stored": info.format_bytes / max(1, info.nnz),
                               "moved": abytes / max(1, wl.local_nnz)},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic,
+                         "frac": achieved / peak, "traffic": traffic, "frac_of_8tbps_spec": achieved / 8000.0,
                          "peak_kind": f"{peak_kind} copy bandwidth (MEASURED_PEAKS.json hbm_gbs)",
                          "kernel": "spaden_spmv (k_spmv_tiled [+ long-row chunks/fix-up])",
                          "kernel_ms": kavg_ms, "alg_bytes_per_launch": abytes},
