@@ -507,7 +507,44 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             ul = __shfl_sync(kFull, ul, 0);
             if (ul >= units) break;
             ++mine;
-            if constexpr (DEC == 4) {
+            if constexpr (DEC == 5 || DEC == 6) {
+                // LPB lanes per block (5: 4 lanes x 2 rows, 6: 2 lanes x 4 rows), 32/LPB
+                // consecutive blocks per step: a step's value loads stay inside fewer,
+                // contiguous runs (fewer bank conflicts, esp. for fp16)
+                constexpr int LPB = DEC == 5 ? 4 : 2, RPL = 8 / LPB, BPS = 32 / LPB;
+                const int g = lane / LPB, q = lane % LPB;
+                const int r0 = q * RPL;  // first row of this lane
+#pragma unroll 1
+                for (int st = 0; st < LPB; ++st) {
+                    const int lb = ul * 32 + st * BPS + g;
+                    if (lb < nb) {
+                        const uint2 bm = lds_u2(a_bmp + 8u * lb);
+                        const int bc = lds_i32(a_col + 4u * lb);
+                        const uint32_t p0 = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
+                        XSeg xs;
+                        load_x(xs, x, bc, nbc_vec, used_cols(bm));
+                        const int plo = __popc(bm.x);
+#pragma unroll
+                        for (int rr = 0; rr < RPL; ++rr) {
+                            const int r = r0 + rr;  // not a compile-time constant: select by q
+                            const uint32_t w = r < 4 ? bm.x : bm.y;
+                            const int sh = 8 * (r & 3);
+                            const uint32_t byte = (w >> sh) & 0xffu;
+                            const int below = ((r & 3) == 0 ? 0 : __popc(w & ((1u << sh) - 1u))) + (r < 4 ? 0 : plo);
+                            uint32_t p = p0 + (uint32_t)below * (uint32_t)sizeof(V);
+                            float a = 0.f;
+#pragma unroll
+                            for (int c = 0; c < 8; ++c) {
+                                if ((byte >> c) & 1u) {
+                                    a = fmaf(SmemVals<V>::get(p), xs.v[c], a);
+                                    p += SmemVals<V>::step;
+                                }
+                            }
+                            sts_f32(a_part + kPartStride * lb + 4u * r, a);
+                        }
+                    }
+                }
+            } else if constexpr (DEC == 4) {
                 // tensor-core ablation (SURVEY.md §8(f) NEXT-3, fp16 values): the
                 // paper's fragment trick on mma.sync.m16n8k16 -- four
                 // blocks per MMA, block P/Q/R/S in the TL/TR/BL/BR quadrants, lane l
@@ -893,20 +930,31 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
         if (e && e[0] == 's') return 1;
         if (e && e[0] == 'r') return 2;
         if (e && e[0] == 'm') return 4;
+        if (e && e[0] == 'q') return 5;  // "quad": 4 lanes per block
+        if (e && e[0] == 'p') return 6;  // "pair": 2 lanes per block
         return -1;
     }();
     const int dec = decode_env >= 0 ? decode_env
                                     : ((A.Bnnz == 0 || A.nnz >= (int64_t)kSlotsMinFill * A.Bnnz) ? kDenseDecode : 0);
     cudaError_t e;
-    if (A.storage == SPADEN_R_16F)
-        e = dec == 0 ? launch_tiled<__half, 0>(A, alpha, x, beta, y, st)
-                     : dec == 2 ? launch_tiled<__half, 2>(A, alpha, x, beta, y, st)
-                                : dec == 4 ? launch_tiled<__half, 4>(A, alpha, x, beta, y, st)
-                                           : launch_tiled<__half, 1>(A, alpha, x, beta, y, st);
-    else  // (the tensor-core ablation exists for fp16 values only)
-        e = dec == 0 ? launch_tiled<float, 0>(A, alpha, x, beta, y, st)
-                     : (dec == 2 ? launch_tiled<float, 2>(A, alpha, x, beta, y, st)
-                                 : launch_tiled<float, 1>(A, alpha, x, beta, y, st));
+    if (A.storage == SPADEN_R_16F) {
+        switch (dec) {
+        case 0: e = launch_tiled<__half, 0>(A, alpha, x, beta, y, st); break;
+        case 2: e = launch_tiled<__half, 2>(A, alpha, x, beta, y, st); break;
+        case 4: e = launch_tiled<__half, 4>(A, alpha, x, beta, y, st); break;
+        case 5: e = launch_tiled<__half, 5>(A, alpha, x, beta, y, st); break;
+        case 6: e = launch_tiled<__half, 6>(A, alpha, x, beta, y, st); break;
+        default: e = launch_tiled<__half, 1>(A, alpha, x, beta, y, st);
+        }
+    } else {  // (the tensor-core ablation exists for fp16 values only)
+        switch (dec) {
+        case 0: e = launch_tiled<float, 0>(A, alpha, x, beta, y, st); break;
+        case 2: e = launch_tiled<float, 2>(A, alpha, x, beta, y, st); break;
+        case 5: e = launch_tiled<float, 5>(A, alpha, x, beta, y, st); break;
+        case 6: e = launch_tiled<float, 6>(A, alpha, x, beta, y, st); break;
+        default: e = launch_tiled<float, 1>(A, alpha, x, beta, y, st);
+        }
+    }
     if (e == cudaSuccess) e = residual_spmv(A, alpha, x, y, st);  // hybrid residual (if any)
     if (e != cudaSuccess) return cuda_status(e, "launching k_spmv_tiled");
     return SPADEN_OK;

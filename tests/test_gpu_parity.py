@@ -513,7 +513,7 @@ def test_hybrid_spmv(sp, torch, name):
         assert np.array_equal(np.concatenate(parts), y1)
 
 
-@pytest.mark.parametrize("decode", ["slots", "bits", "rows", "mma"])
+@pytest.mark.parametrize("decode", ["slots", "bits", "rows", "mma", "quad", "pair"])
 @pytest.mark.parametrize("name", ["fem62k_small", "hub", "tiny", "h2"])
 def test_decode_ablations_fp16(sp, torch, decode, name, monkeypatch):
     """Every decode variant (SPADEN_DECODE) on fp16 storage, including the
@@ -524,3 +524,44 @@ def test_decode_ablations_fp16(sp, torch, decode, name, monkeypatch):
     x = W.vector(A.n, 29)
     y = gpu_spmv(torch, M, x)
     check_spmv(A, y, oracle.f32_to_f16(A.values), x)
+
+
+@pytest.mark.parametrize("decode", ["bits", "rows", "quad", "pair"])
+@pytest.mark.parametrize("storage", ["fp32", "fp16"])
+def test_decodes_bitwise_equal_to_slots(sp, torch, decode, storage, monkeypatch):
+    """Every CUDA-core decode computes the same per-block row partials in the same
+    order, so y is bitwise identical to the default decode."""
+    A = W.fem(9, 9, 10, seed=5)
+    x = W.vector(A.n, 31)
+    monkeypatch.setenv("SPADEN_DECODE", "slots")
+    M = convert(sp, torch, A, storage=storage)
+    ref = gpu_spmv(torch, M, x)
+    monkeypatch.setenv("SPADEN_DECODE", decode)
+    assert np.array_equal(gpu_spmv(torch, M, x), ref)
+
+
+def random_cases(count=24, seed=123):
+    rng = np.random.default_rng(seed)
+    for i in range(count):
+        m = int(rng.choice([1, 2, 7, 8, 9, 63, 64, 65, 300, 1000, 4099]))
+        n = int(rng.choice([1, 3, 8, 15, 64, 129, 1000, 5000, 70_001]))
+        dens = float(rng.choice([0.001, 0.01, 0.05, 0.3, 1.0]))
+        dens = min(dens, 200_000 / max(1, m * n))
+        yield i, m, n, dens
+
+
+@pytest.mark.parametrize("case", list(random_cases()), ids=lambda c: f"r{c[0]}_{c[1]}x{c[2]}")
+def test_random_shapes_all_modes(sp, torch, case):
+    """Randomised shapes (1xN, Nx1, ragged, dense, very sparse) through every
+    storage mode and the hybrid split: conversion exact, SpMV within tolerance."""
+    i, m, n, dens = case
+    A = W.random_sparse(m, n, dens, seed=1000 + i)
+    x = W.vector(n, 2000 + i)
+    for storage in ("fp32", "fp16"):
+        stored = A.values if storage == "fp32" else oracle.f32_to_f16(A.values)
+        M = convert(sp, torch, A, storage=storage)
+        assert_format_parity(torch, M, W.CSR(A.m, A.n, A.rowptr, A.colidx, stored), stored)
+        check_spmv(A, gpu_spmv(torch, M, x), stored, x)
+        rp, ci, v = dev(torch, A)
+        H = sp.convert(rp, ci, v, n, storage=storage, residual_max_popc=int(1 + i % 4))
+        check_spmv(A, gpu_spmv(torch, H, x), stored, x)
