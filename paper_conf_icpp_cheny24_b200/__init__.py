@@ -16,7 +16,7 @@ import ctypes
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libspaden.so")
+LIB_PATH = os.environ.get("SPADEN_LIB") or os.path.join(_PKG, "libspaden.so")  # override: A/B experiments
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_icpp_cheny24_b200.build` "
