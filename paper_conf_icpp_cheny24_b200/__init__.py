@@ -71,6 +71,9 @@ spaden_convert_csr_to_bitmap_ex.restype = _ST
 spaden_spmv = _lib.spaden_spmv
 spaden_spmv.argtypes = [_P, _F, _P, _F, _P, _P]
 spaden_spmv.restype = _ST
+spaden_spmm = _lib.spaden_spmm
+spaden_spmm.argtypes = [_P, _F, _P, _I64, ctypes.c_int32, _F, _P, _I64, _P]
+spaden_spmm.restype = _ST
 spaden_spmv_host = _lib.spaden_spmv_host
 spaden_spmv_host.argtypes = [_P, _F, _P, _F, _P, _P]
 spaden_spmv_host.restype = _ST
@@ -96,7 +99,7 @@ spaden_version = _lib.spaden_version
 spaden_version.argtypes = []
 spaden_version.restype = ctypes.c_char_p
 
-EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_spmv", "spaden_spmv_host", "spaden_spmv_host_batched",
+EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_spmv", "spaden_spmm", "spaden_spmv_host", "spaden_spmv_host_batched",
             "spaden_free",
             "spaden_get_info", "spaden_get_arrays", "spaden_status_string",
             "spaden_last_error_message", "spaden_version"]
@@ -208,6 +211,19 @@ class Matrix:
         _check(spaden_spmv(self._h, alpha, ctypes.c_void_p(x.data_ptr()), beta,
                            ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream)), "spaden_spmv")
         return y
+
+    def spmm(self, X, Y=None, alpha: float = 1.0, beta: float = 0.0, stream=None):
+        """Y[j] = alpha * A X[j] + beta * Y[j] for the rows j of X (k x n, CUDA float32,
+        rows contiguous) -> Y (k x m)."""
+        torch = _torch()
+        k = X.shape[0]
+        if Y is None:
+            Y = torch.empty((k, self.m), dtype=torch.float32, device=X.device)
+        assert X.dtype == torch.float32 and Y.dtype == torch.float32 and X.is_cuda and Y.is_cuda
+        assert X.shape[1] == self.n and Y.shape == (k, self.m) and X.stride(1) == 1 and Y.stride(1) == 1
+        _check(spaden_spmm(self._h, alpha, ctypes.c_void_p(X.data_ptr()), X.stride(0), k, beta,
+                           ctypes.c_void_p(Y.data_ptr()), Y.stride(0), _stream_ptr(stream)), "spaden_spmm")
+        return Y
 
     def spmv_host(self, x_host, y_host, alpha: float = 1.0, beta: float = 0.0, stream=None):
         """Host-buffer variant (H2D x, SpMV, D2H y, stream sync) through the C ABI."""

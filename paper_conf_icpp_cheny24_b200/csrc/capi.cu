@@ -48,7 +48,7 @@ static void release(Matrix *A) {
                     A->pipe_y[0],   A->pipe_y[1], A->pipe_y[2], A->tiles,
                     A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->res_rowptr,
                     A->res_colidx,  A->res_values, A->res_long_rows, A->res_chunk_start,
-                    A->res_chunk_row, A->res_carry};
+                    A->res_chunk_row, A->res_carry, A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (cudaEvent_t e : A->ev)
@@ -184,6 +184,24 @@ spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const float *d_x, fl
         }
     }
     return spmv_launch(*A, alpha, d_x, beta, d_y, (cudaStream_t)stream);
+}
+
+spaden_status_t spaden_spmm(spaden_matrix_t A, float alpha, const float *d_X, int64_t ldx, int32_t k, float beta,
+                            float *d_Y, int64_t ldy, void *stream) {
+    if (!A || k < 0 || ldx < A->n || ldy < A->m || (k > 0 && ((A->m > 0 && !d_Y) || (A->Bnnz > 0 && !d_X)))) {
+        set_error("NULL handle/matrices, k < 0, or ldx < n / ldy < m");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (k > 0 && d_X && d_Y && A->m > 0 && A->n > 0) {
+        const char *xb = (const char *)d_X, *xe = (const char *)(d_X + (int64_t)(k - 1) * ldx + A->n);
+        const char *yb = (const char *)d_Y, *ye = (const char *)(d_Y + (int64_t)(k - 1) * ldy + A->m);
+        if (xb < ye && yb < xe) {
+            set_error("X and Y must not overlap");
+            return SPADEN_ERR_INVALID_ARGUMENT;
+        }
+    }
+    if (k == 0) return SPADEN_OK;
+    return spmm_launch(*A, alpha, d_X, ldx, k, beta, d_Y, ldy, (cudaStream_t)stream);
 }
 
 spaden_status_t spaden_spmv_host(spaden_matrix_t A, float alpha, const float *h_x, float beta, float *h_y,

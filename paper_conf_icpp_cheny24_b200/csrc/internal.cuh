@@ -40,6 +40,11 @@ struct spaden_matrix_s {
     int32_t *chunk_row = nullptr;              // [n_chunks] index into long_rows
     float *carry = nullptr;                    // [n_chunks*8] per-chunk row partials
 
+    // SpMM schedules for K = 2, 4, 8 right-hand sides (built lazily by spaden_spmm)
+    struct spaden_tile_desc_s *spmm_tiles[3] = {};
+    int64_t spmm_ntiles[3] = {};
+    int spmm_state[3] = {};                    // 0 not built, 1 built, -1 unsupported
+
     // hybrid residual CSR (csrc/hybrid.cu), empty in pure bitBSR mode
     int64_t res_nnz = 0;
     int res_max_popc = 0;
@@ -130,6 +135,7 @@ constexpr int kDenseDecode = 1;
 using TileDesc = ::spaden_tile_desc_s;
 
 spaden_status_t build_schedule(Matrix *A, cudaStream_t stream);
+spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t stream);
 
 
 // converter (convert.cu)
@@ -144,6 +150,9 @@ cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y
 // SpMV (spmv.cu)
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,
                             cudaStream_t stream);
+// SpMM: k column-major vectors (spmv.cu)
+spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx, int k, float beta, float *Y,
+                            int64_t ldy, cudaStream_t stream);
 
 // exclusive scan of int32 (scan.cu): out[i] = sum_{j<i} in[j], out[count] = total.
 // `in` and `out` may alias.  tmp must hold scan_tmp_ints(count) int32.

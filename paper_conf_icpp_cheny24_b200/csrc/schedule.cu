@@ -21,18 +21,24 @@ namespace {
 
 constexpr int kSeg = 256;
 
+// stage bytes of a block-row: `blk_bytes` per block (copied metadata + partial
+// scratch), its values, its blk_rowptr entry
 __device__ __forceinline__ int64_t br_cost(const int32_t *brp, const int32_t *boff, int64_t br, int sv,
-                                           int32_t *nb_out, int32_t *nv_out) {
+                                           int blk_bytes, int32_t *nb_out, int32_t *nv_out) {
     const int b0 = brp[br], b1 = brp[br + 1];
     const int nv = boff[b1] - boff[b0];
     *nb_out = b1 - b0;
     *nv_out = nv;
-    return (int64_t)kBlockStageBytes * (b1 - b0) + (int64_t)sv * nv + 4;
+    return (int64_t)blk_bytes * (b1 - b0) + (int64_t)sv * nv + 4;
 }
 
+// Long rows are classified with the SpMV cost (kBlockStageBytes per block) so
+// SpMV and SpMM schedules (pack_blk_bytes = 16 + 4(8K+1)) share one long-row set;
+// a normal row that does not fit a stage under the pack cost sets *too_big.
 template <bool WRITE>
 __global__ void k_pack(int64_t Bnrow, const int32_t *__restrict__ brp, const int32_t *__restrict__ boff,
-                       int sv, int64_t cap, int64_t long_cost, int32_t *__restrict__ seg_tiles,
+                       int sv, int64_t cap, int64_t long_cost, int pack_blk_bytes, uint32_t *too_big,
+                       int32_t *__restrict__ seg_tiles,
                        int32_t *__restrict__ seg_long, const int32_t *__restrict__ tile_start,
                        const int32_t *__restrict__ long_start, TileDesc *__restrict__ tiles,
                        int32_t *__restrict__ long_rows) {
@@ -64,13 +70,14 @@ __global__ void k_pack(int64_t Bnrow, const int32_t *__restrict__ brp, const int
     };
     for (int64_t br = s0; br < s1; ++br) {
         int32_t nb, nv;
-        const int64_t c = br_cost(brp, boff, br, sv, &nb, &nv);
-        if (c > long_cost) {
+        if (br_cost(brp, boff, br, sv, kBlockStageBytes, &nb, &nv) > long_cost) {
             close(br);
-            if (WRITE) long_rows[lbase + nl] = (int32_t)br;
+            if (WRITE && long_rows) long_rows[lbase + nl] = (int32_t)br;
             ++nl;
             continue;
         }
+        const int64_t c = br_cost(brp, boff, br, sv, pack_blk_bytes, &nb, &nv);
+        if (c > cap && too_big) atomicOr(too_big, 1u);
         if (open_br >= 0 && open_cost + c > cap) close(br);
         if (open_br < 0) open_br = br;
         open_cost += c;
@@ -132,8 +139,8 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     int32_t *seg_tiles = tmp, *seg_long = tmp + (nseg + 1), *scan_tmp = tmp + 2 * (nseg + 1);
     int32_t *summary = scan_tmp + n_tmp;
     const unsigned grid = (unsigned)((nseg + 127) / 128);
-    k_pack<false><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, seg_tiles,
-                                        seg_long, nullptr, nullptr, nullptr, nullptr);
+    k_pack<false><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, kBlockStageBytes,
+                                        nullptr, seg_tiles, seg_long, nullptr, nullptr, nullptr, nullptr);
     cudaError_t e = exclusive_scan_i32(seg_tiles, seg_tiles, nseg, scan_tmp, st);
     if (e == cudaSuccess) e = exclusive_scan_i32(seg_long, seg_long, nseg, scan_tmp, st);
     int32_t h[2] = {0, 0};
@@ -157,8 +164,8 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
         return cuda_status(e, "allocating SpMV schedule");
     }
     A->aux_bytes = (int64_t)(tile_bytes + long_bytes);
-    k_pack<true><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, nullptr,
-                                       nullptr, seg_tiles, seg_long, A->tiles, A->long_rows);
+    k_pack<true><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, kBlockStageBytes,
+                                       nullptr, nullptr, nullptr, seg_tiles, seg_long, A->tiles, A->long_rows);
     e = cudaGetLastError();
     cudaFreeAsync(tmp, st);
     if (e != cudaSuccess) return cuda_status(e, "packing SpMV schedule");
@@ -189,6 +196,59 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     }
     if (e != cudaSuccess) return cuda_status(e, "long-row chunk schedule");
     A->aux_bytes += (int64_t)sizeof(int32_t) * (nl + 1 + nch) + (int64_t)sizeof(float) * 8 * nch;
+    return SPADEN_OK;
+}
+
+// SpMM schedule for K right-hand sides (built lazily by spaden_spmm): same
+// stage size and long-row set as the SpMV schedule, tiles packed with the
+// larger per-block partial scratch.  Returns UNSUPPORTED when some normal
+// block-row cannot fit a stage with K vectors (the caller then runs K SpMVs).
+spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t st) {
+    const int64_t Bnrow = A->Bnrow;
+    const int sv = A->storage == SPADEN_R_16F ? 2 : 4;
+    const TileCfg cfg = tile_cfg(A->tile_cfg);
+    const int64_t cap = cfg.stage_bytes - kStageSlack;
+    const int64_t long_cost = cfg.warp_mode ? cap : cfg.stage_bytes / 2;
+    const int pack_bytes = 16 + 4 * (8 * K + 1);
+    const int64_t nseg = (Bnrow + kSeg - 1) / kSeg;
+    A->spmm_state[kidx] = -1;
+    if (Bnrow == 0 || cfg.warp_mode) return SPADEN_ERR_UNSUPPORTED;
+    const size_t n_tmp = scan_tmp_ints(nseg + 1);
+    int32_t *tmp = nullptr;
+    SPADEN_CUDA_TRY(cudaMallocAsync(&tmp, (2 * (size_t)(nseg + 1) + n_tmp + 8) * sizeof(int32_t), st));
+    int32_t *seg_tiles = tmp, *seg_long = tmp + (nseg + 1), *scan_tmp = tmp + 2 * (nseg + 1);
+    int32_t *summary = scan_tmp + n_tmp;
+    uint32_t *too_big = (uint32_t *)(summary + 4);
+    cudaMemsetAsync(too_big, 0, 4, st);
+    const unsigned grid = (unsigned)((nseg + 127) / 128);
+    k_pack<false><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, pack_bytes, too_big,
+                                        seg_tiles, seg_long, nullptr, nullptr, nullptr, nullptr);
+    cudaError_t e = exclusive_scan_i32(seg_tiles, seg_tiles, nseg, scan_tmp, st);
+    int32_t h[2] = {0, 0};
+    if (e == cudaSuccess) {
+        k_sched_summary<<<1, 1, 0, st>>>(seg_tiles + nseg, (const int32_t *)too_big, summary);
+        e = cudaMemcpyAsync(h, summary, sizeof(h), cudaMemcpyDeviceToHost, st);
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess || h[1] != 0) {
+        cudaFreeAsync(tmp, st);
+        if (e != cudaSuccess) return cuda_status(e, "building SpMM schedule");
+        set_error("a block-row does not fit a pipeline stage with this many right-hand sides");
+        return SPADEN_ERR_UNSUPPORTED;
+    }
+    const size_t tile_bytes = sizeof(TileDesc) * (size_t)std::max(1, h[0] + 1);
+    e = cudaMalloc(&A->spmm_tiles[kidx], tile_bytes);
+    if (e == cudaSuccess) {
+        k_pack<true><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, pack_bytes,
+                                           nullptr, nullptr, nullptr, seg_tiles, seg_long, A->spmm_tiles[kidx],
+                                           nullptr);
+        e = cudaGetLastError();
+    }
+    cudaFreeAsync(tmp, st);
+    if (e != cudaSuccess) return cuda_status(e, "packing SpMM schedule");
+    A->spmm_ntiles[kidx] = h[0];
+    A->spmm_state[kidx] = 1;
+    A->aux_bytes += (int64_t)tile_bytes;
     return SPADEN_OK;
 }
 

@@ -307,6 +307,71 @@ __device__ __forceinline__ void reduce_tile(uint32_t a_rp, uint32_t a_part, int 
     }
 }
 
+// Phase 2 for K right-hand sides: partials of a block are [r][j] at a
+// 4(8K+1)-byte stride; entry idx = (block-row, r, j); same chain order as
+// reduce_tile, so column j equals the SpMV of vector j bitwise.
+template <int K>
+__device__ __forceinline__ void reduce_tile_k(uint32_t a_rp, uint32_t a_part, int nbr, int b0, int br0, int lane,
+                                              int64_t m, float alpha, float beta, float *__restrict__ y,
+                                              int64_t ldy) {
+    constexpr uint32_t PS = 4u * (8 * K + 1);
+    for (int idx = lane; idx < nbr * 8 * K; idx += 32) {
+        const int brl = idx / (8 * K), rj = idx % (8 * K);
+        const int r = rj / K, j = rj % K;
+        const int k0 = lds_i32(a_rp + 4u * brl) - b0;
+        const int k1 = lds_i32(a_rp + 4u * (brl + 1)) - b0;
+        float c0 = 0.f, c1 = 0.f, c2 = 0.f, c3 = 0.f;
+        uint32_t q = a_part + PS * k0 + 4u * rj;
+        int k = k0;
+        for (; k + 3 < k1; k += 4, q += 4 * PS) {
+            c0 += lds_f32(q);
+            c1 += lds_f32(q + PS);
+            c2 += lds_f32(q + 2 * PS);
+            c3 += lds_f32(q + 3 * PS);
+        }
+        if (k < k1) c0 += lds_f32(q);
+        if (k + 1 < k1) c1 += lds_f32(q + PS);
+        if (k + 2 < k1) c2 += lds_f32(q + 2 * PS);
+        const float sum = (c0 + c1) + (c2 + c3);
+        const int64_t row = 8 * ((int64_t)br0 + brl) + r;
+        if (row < m) {
+            float *yp = y + (int64_t)j * ldy + row;
+            float o = alpha * sum;
+            if (beta != 0.f) o = fmaf(beta, *yp, o);
+            *yp = o;
+        }
+    }
+}
+
+// Phase 1 for K right-hand sides: one lane per block, 64 predicated slots, each
+// loaded value multiplied into K accumulators (per-row, same fma order as
+// block_slots for every vector); partials stored [r][j].
+template <class VS, int K>
+__device__ __forceinline__ void block_slots_k(uint2 bm, typename VS::P p0, const XSeg (&xs)[K], uint32_t q) {
+    const int plo = __popc(bm.x);
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+        const uint32_t w = r < 4 ? bm.x : bm.y;
+        const uint32_t byte = (w >> (8 * (r & 3))) & 0xffu;
+        const int below = ((r & 3) == 0 ? 0 : __popc(w & ((1u << (8 * (r & 3))) - 1u))) + (r < 4 ? 0 : plo);
+        typename VS::P p = p0 + below * VS::step;
+        float a[K];
+#pragma unroll
+        for (int j = 0; j < K; ++j) a[j] = 0.f;
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+            if ((byte >> c) & 1u) {
+                const float v = VS::get(p);
+#pragma unroll
+                for (int j = 0; j < K; ++j) a[j] = fmaf(v, xs[j].v[c], a[j]);
+                p += VS::step;
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < K; ++j) sts_f32(q + 4u * (r * K + j), a[j]);
+    }
+}
+
 __device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
     unsigned short h;
     asm("ld.shared.u16 %0, [%1];" : "=h"(h) : "r"(a));
@@ -412,12 +477,12 @@ struct alignas(16) StageHdr {
 // DEC: 0 = set-bit loop, 1 = 64 predicated slots per lane (lane = block),
 //      2 = 8 predicated slots per lane (lane = one row of a block, 4 blocks per
 //          warp step: value loads of a step stay inside 4 consecutive runs).
-template <typename V, int DEC, int CONSUMERS, int MINB>
+template <typename V, int DEC, int CONSUMERS, int MINB, int K = 1>
 __global__ void __launch_bounds__(32 * (CONSUMERS + 1), MINB)
 k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int ntiles, const int32_t *__restrict__ blk_rowptr,
              const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
              const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
-             int nbc_vec, float alpha, float beta, float *__restrict__ y) {
+             int nbc_vec, float alpha, float beta, float *__restrict__ y, int64_t ldx = 0, int64_t ldy = 0) {
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t full_bar[kMaxStages], empty_bar[kMaxStages];
     __shared__ StageHdr hdr[kMaxStages];
@@ -507,7 +572,19 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             ul = __shfl_sync(kFull, ul, 0);
             if (ul >= units) break;
             ++mine;
-            if constexpr (DEC == 5 || DEC == 6) {
+            if constexpr (K > 1) {  // SpMM: K right-hand sides
+                const int lb = ul * 32 + lane;
+                if (lb < nb) {
+                    const uint2 bm = lds_u2(a_bmp + 8u * lb);
+                    const int bc = lds_i32(a_col + 4u * lb);
+                    const uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
+                    const uint32_t cols = used_cols(bm);
+                    XSeg xs[K];
+#pragma unroll
+                    for (int j = 0; j < K; ++j) load_x(xs[j], x + j * ldx, bc, nbc_vec, cols);
+                    block_slots_k<SmemVals<V>, K>(bm, p, xs, a_part + 4u * (8 * K + 1) * lb);
+                }
+            } else if constexpr (DEC == 5 || DEC == 6) {
                 // LPB lanes per block (5: 4 lanes x 2 rows, 6: 2 lanes x 4 rows), 32/LPB
                 // consecutive blocks per step: a step's value loads stay inside fewer,
                 // contiguous runs (fewer bank conflicts, esp. for fp16)
@@ -608,7 +685,10 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             }
             if (__shfl_sync(kFull, last, 0)) {  // phase 2: this warp completed the tile
                 __threadfence_block();
-                reduce_tile((uint32_t)h2.w, a_part, h0.y, h0.z, h0.x, lane, m, alpha, beta, y);
+                if constexpr (K > 1)
+                    reduce_tile_k<K>((uint32_t)h2.w, a_part, h0.y, h0.z, h0.x, lane, m, alpha, beta, y, ldy);
+                else
+                    reduce_tile((uint32_t)h2.w, a_part, h0.y, h0.z, h0.x, lane, m, alpha, beta, y);
             }
         }
         __syncwarp();
@@ -901,7 +981,93 @@ cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float bet
     }
 }
 
+template <typename V, int K, int CONSUMERS, int MINB>
+cudaError_t launch_spmm_cfg(const Matrix &A, const TileCfg &cfg, const TileDesc *tiles, int64_t ntiles, float alpha,
+                            const float *X, int64_t ldx, float beta, float *Y, int64_t ldy, cudaStream_t st) {
+    const bool aligned = ((uintptr_t)X & 31u) == 0 && ((ldx * 4) % 32) == 0;
+    const int nbc_vec = aligned ? (int)(A.n / 8) : 0;
+    const size_t smem = (size_t)cfg.stages * cfg.stage_bytes;
+    static size_t occ_smem = 0;
+    static int occ = 0;
+    if (occ_smem != smem) {
+        auto kern = k_spmv_tiled<V, 1, CONSUMERS, MINB, K>;
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e == cudaSuccess)
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * (CONSUMERS + 1), smem);
+        if (e != cudaSuccess) return e;
+        occ = std::max(1, std::min(occ, MINB));
+        occ_smem = smem;
+    }
+    if (ntiles > 0) {
+        const int grid = (int)std::min<int64_t>(ntiles, (int64_t)sm_count() * occ);
+        k_spmv_tiled<V, 1, CONSUMERS, MINB, K><<<grid, 32 * (CONSUMERS + 1), smem, st>>>(
+            cfg.stages, cfg.stage_bytes, A.m, tiles, (int)ntiles, A.blk_rowptr, A.blk_col, A.bitmap,
+            A.blk_offset, (const V *)A.values, X, nbc_vec, alpha, beta, Y, ldx, ldy);
+    }
+    if (A.n_long > 0) {  // long block-rows: the SpMV chunk path, once per vector (same arithmetic)
+        const int nbc1 = ((uintptr_t)X & 31u) == 0 && ((ldx * 4) % 32) == 0 ? (int)(A.n / 8) : 0;
+        for (int j = 0; j < K; ++j) {
+            const int64_t threads = 32 * A.n_chunks;
+            k_spmv_long_chunks<V, true><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+                (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
+                A.blk_offset, (const V *)A.values, X + j * ldx, nbc1, A.carry);
+            k_spmv_long_fixup<<<(unsigned)((8 * A.n_long + 255) / 256), 256, 0, st>>>(
+                A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, Y + j * ldy);
+        }
+    }
+    return cudaGetLastError();
+}
+
+template <typename V, int K>
+cudaError_t launch_spmm(const Matrix &A, const TileDesc *tiles, int64_t ntiles, float alpha, const float *X,
+                        int64_t ldx, float beta, float *Y, int64_t ldy, cudaStream_t st) {
+    const TileCfg cfg = tile_cfg(A.tile_cfg);
+    // same stage geometry as the SpMV schedule; fewer CTAs per SM so the K
+    // accumulators and x segments fit in registers without spilling
+    switch (A.tile_cfg) {
+    case 0: case 1: case 6:
+        return launch_spmm_cfg<V, K, 16, 1>(A, cfg, tiles, ntiles, alpha, X, ldx, beta, Y, ldy, st);
+    default: return launch_spmm_cfg<V, K, 8, 2>(A, cfg, tiles, ntiles, alpha, X, ldx, beta, Y, ldy, st);
+    }
+}
+
 }  // namespace
+
+spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx, int k, float beta, float *Y,
+                            int64_t ldy, cudaStream_t st) {
+    int j = 0;
+    while (j < k) {
+        const int left = k - j;
+        const int K = left >= 8 ? 8 : left >= 4 ? 4 : left >= 2 ? 2 : 1;
+        const int kidx = K == 8 ? 2 : K == 4 ? 1 : 0;
+        if (K > 1 && A.m > 0 && A.spmm_state[kidx] == 0) build_spmm_schedule(&A, kidx, K, st);
+        if (K == 1 || A.spmm_state[kidx] != 1 || A.m == 0) {  // one SpMV per vector
+            for (int q = 0; q < K; ++q) {
+                spaden_status_t s = spmv_launch(A, alpha, X + (j + q) * ldx, beta, Y + (j + q) * ldy, st);
+                if (s != SPADEN_OK) return s;
+            }
+        } else {
+            const TileDesc *tiles = A.spmm_tiles[kidx];
+            const int64_t nt = A.spmm_ntiles[kidx];
+            const float *Xj = X + j * ldx;
+            float *Yj = Y + j * ldy;
+            cudaError_t e;
+            if (A.storage == SPADEN_R_16F)
+                e = K == 8 ? launch_spmm<__half, 8>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
+                    : K == 4 ? launch_spmm<__half, 4>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
+                             : launch_spmm<__half, 2>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st);
+            else
+                e = K == 8 ? launch_spmm<float, 8>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
+                    : K == 4 ? launch_spmm<float, 4>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
+                             : launch_spmm<float, 2>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st);
+            for (int q = 0; q < K && e == cudaSuccess; ++q)
+                e = residual_spmv(A, alpha, Xj + q * ldx, Yj + q * ldy, st);
+            if (e != cudaSuccess) return cuda_status(e, "launching SpMM");
+        }
+        j += K;
+    }
+    return SPADEN_OK;
+}
 
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,
                             cudaStream_t st) {

@@ -565,3 +565,36 @@ def test_random_shapes_all_modes(sp, torch, case):
         rp, ci, v = dev(torch, A)
         H = sp.convert(rp, ci, v, n, storage=storage, residual_max_popc=int(1 + i % 4))
         check_spmv(A, gpu_spmv(torch, H, x), stored, x)
+
+
+# ------------------------------------------------------------ SpMM (NEXT-4)
+@pytest.mark.parametrize("k", [1, 2, 3, 4, 7, 8, 13])
+@pytest.mark.parametrize("name", ["fem", "hub", "tiny", "h2"])
+@pytest.mark.parametrize("storage", ["fp32", "fp16"])
+def test_spmm_columns_equal_spmv(sp, torch, k, name, storage):
+    """spaden_spmm: column j equals spaden_spmv on vector j bitwise, and the
+    oracle within tolerance (fp32/fp16 values, long rows, ragged shapes)."""
+    A = {"fem": lambda: W.fem(7, 8, 9, seed=6), "hub": hub_matrix, "tiny": lambda: W.tiny(2), "h2": W.h2}[name]()
+    M = convert(sp, torch, A, storage=storage)
+    X = torch.from_numpy(np.stack([W.vector(A.n, 300 + j) for j in range(k)])).cuda()
+    Y0 = torch.from_numpy(np.stack([W.vector(A.m, 400 + j) for j in range(k)])).cuda()
+    Y = M.spmm(X, Y0.clone(), alpha=0.75, beta=0.5)
+    torch.cuda.synchronize()
+    stored = A.values if storage == "fp32" else oracle.f32_to_f16(A.values)
+    for j in range(k):
+        yj = M.spmv(X[j].contiguous(), Y0[j].clone(), alpha=0.75, beta=0.5)
+        torch.cuda.synchronize()
+        assert torch.equal(Y[j], yj), j
+        ys, s = oracle.spmv(A.rowptr, A.colidx, stored, X[j].cpu().numpy())
+        y0 = Y0[j].cpu().numpy().astype(np.float64)
+        assert oracle.componentwise_error(Y[j].cpu().numpy(), 0.75 * ys + 0.5 * y0, 0.75 * s + 0.5 * np.abs(y0)) <= TOL32
+
+
+def test_spmm_hybrid(sp, torch):
+    A = hub_matrix()
+    rp, ci, v = dev(torch, A)
+    M = sp.convert(rp, ci, v, A.n, residual_max_popc=2)
+    X = torch.from_numpy(np.stack([W.vector(A.n, 500 + j) for j in range(4)])).cuda()
+    Y = M.spmm(X)
+    for j in range(4):
+        assert torch.equal(Y[j], M.spmv(X[j].contiguous()))
