@@ -51,6 +51,7 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-cusparse", action="store_true")
     p.add_argument("--no-variants", action="store_true", help="skip the other-precision kernel timing")
+    p.add_argument("--spmm", default="4", help="comma list of right-hand-side counts for the SpMM extra ('' = skip)")
     p.add_argument("--hybrid", type=int, default=0,
                    help="hybrid format: blocks with <= HYBRID entries go to a CSR residual (0 = pure bitBSR)")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -422,6 +423,28 @@ def main():
             del ys
 
         # tiled kernel [+ long-row chunks and fix-up] [+ hybrid residual pass]
+        # ---- SpMM (NEXT-4): K right-hand sides per decoded block
+        spmm = {}
+        if world == 1 and args.spmm:
+            for K in [int(v) for v in args.spmm.split(",") if v]:
+                X = wl.x0.expand(K, wl.n).contiguous()
+                Yk = torch.empty((K, wl.m), dtype=torch.float32, device=dev)
+                for _ in range(3):
+                    M.spmm(X, Yk, alpha=wl.alpha, stream=stream)
+                reps = max(10, min(args.steps, 200))
+                s0e = torch.cuda.Event(enable_timing=True)
+                s1e = torch.cuda.Event(enable_timing=True)
+                torch.cuda.synchronize(dev)
+                s0e.record(stream)
+                for _ in range(reps):
+                    M.spmm(X, Yk, alpha=wl.alpha, stream=stream)
+                s1e.record(stream)
+                torch.cuda.synchronize(dev)
+                sms = s0e.elapsed_time(s1e) / reps
+                spmm[str(K)] = {"ms": sms, "gflops": 2.0 * wl.nnz * K / (sms * 1e-3) / 1e9,
+                                "per_vector_speedup_vs_spmv": kavg_ms * K / sms}
+                del X, Yk
+
         n_launch = 1 + (2 if info.n_long > 0 else 0) + (1 if info.residual_nnz > 0 else 0)
         line = {
             "metric": METRIC, "value": gflops, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -448,6 +471,7 @@ def main():
             "convert": {"seconds": convert_s, "ns_per_nnz": convert_s * 1e9 / max(1, wl.local_nnz)},
             "cusparse_csr": cus,
             "variants": variants,
+            "spmm": spmm,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": args.steps * n_launch,

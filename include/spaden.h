@@ -170,10 +170,10 @@ SPADEN_API spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const flo
  * spaden_spmm -- k products at once (SURVEY.md §8(f) NEXT-4, P:L336 future work):
  * Y[:, j] = alpha * A X[:, j] + beta * Y[:, j] for j < k, with column-major device
  * matrices: vector j of X at d_X + j*ldx (ldx >= n), of Y at d_Y + j*ldy (ldy >= m).
- * Each block is decoded once for up to 8 vectors (its values are loaded once
+ * Each block is decoded once for up to 4 vectors (its values are loaded once
  * from shared memory and multiplied into every vector), so throughput per
  * vector rises with k.  Column j is bitwise identical to spaden_spmv on
- * vector j.  The first call for a given group size (2, 4 or 8) builds a small
+ * vector j.  The first call for a given group size (2 or 4) builds a small
  * schedule and synchronises `stream` once; if a block-row cannot fit a
  * pipeline stage with that many vectors the call falls back to k SpMVs.
  * X and Y must not overlap.  Calls on one handle must be ordered.

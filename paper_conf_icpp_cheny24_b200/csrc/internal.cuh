@@ -40,7 +40,7 @@ struct spaden_matrix_s {
     int32_t *chunk_row = nullptr;              // [n_chunks] index into long_rows
     float *carry = nullptr;                    // [n_chunks*8] per-chunk row partials
 
-    // SpMM schedules for K = 2, 4, 8 right-hand sides (built lazily by spaden_spmm)
+    // SpMM schedules for K = 2, 4 right-hand sides (index 0, 1; built lazily by spaden_spmm)
     struct spaden_tile_desc_s *spmm_tiles[3] = {};
     int64_t spmm_ntiles[3] = {};
     int spmm_state[3] = {};                    // 0 not built, 1 built, -1 unsupported

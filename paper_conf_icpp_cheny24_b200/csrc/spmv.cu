@@ -1038,8 +1038,10 @@ spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx,
     int j = 0;
     while (j < k) {
         const int left = k - j;
-        const int K = left >= 8 ? 8 : left >= 4 ? 4 : left >= 2 ? 2 : 1;
-        const int kidx = K == 8 ? 2 : K == 4 ? 1 : 0;
+        // groups of 4 (measured best: 8 needs more registers than 2 CTAs/SM allow
+        // and smaller tiles)
+        const int K = left >= 4 ? 4 : left >= 2 ? 2 : 1;
+        const int kidx = K == 4 ? 1 : 0;
         if (K > 1 && A.m > 0 && A.spmm_state[kidx] == 0) build_spmm_schedule(&A, kidx, K, st);
         if (K == 1 || A.spmm_state[kidx] != 1 || A.m == 0) {  // one SpMV per vector
             for (int q = 0; q < K; ++q) {
@@ -1053,13 +1055,11 @@ spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx,
             float *Yj = Y + j * ldy;
             cudaError_t e;
             if (A.storage == SPADEN_R_16F)
-                e = K == 8 ? launch_spmm<__half, 8>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
-                    : K == 4 ? launch_spmm<__half, 4>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
-                             : launch_spmm<__half, 2>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st);
+                e = K == 4 ? launch_spmm<__half, 4>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
+                           : launch_spmm<__half, 2>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st);
             else
-                e = K == 8 ? launch_spmm<float, 8>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
-                    : K == 4 ? launch_spmm<float, 4>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
-                             : launch_spmm<float, 2>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st);
+                e = K == 4 ? launch_spmm<float, 4>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
+                           : launch_spmm<float, 2>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st);
             for (int q = 0; q < K && e == cudaSuccess; ++q)
                 e = residual_spmv(A, alpha, Xj + q * ldx, Yj + q * ldy, st);
             if (e != cudaSuccess) return cuda_status(e, "launching SpMM");
