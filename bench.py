@@ -55,6 +55,9 @@ def parse():
     p.add_argument("--hybrid", type=int, default=0,
                    help="hybrid format: blocks with <= HYBRID entries go to a CSR residual (0 = pure bitBSR)")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
+    p.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
+                   help="x rebuild for N>1: NCCL all-gather after the SpMV, or peer stores fused into the "
+                        "SpMV epilogue (spaden_spmv_scatter over symmetric memory, NEXT-2)")
     return p.parse_args()
 
 
@@ -247,7 +250,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_icpp_cheny24_b200 as sp
-    from paper_conf_icpp_cheny24_b200.dist import IteratedSpMV
+    from paper_conf_icpp_cheny24_b200.dist import FusedIteratedSpMV, IteratedSpMV
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -279,7 +282,20 @@ def main():
         if ev_pair[0] is not None:
             ev_pair[0][1].record(stream)
 
-    it = IteratedSpMV(wl.part, wl.n, local_spmv, wl.x0, rank)
+    class _Timed:  # spmv_scatter with the per-launch events of the roofline
+        def spmv_scatter(self, x, ptrs, off, y=None, alpha=1.0, beta=0.0):
+            if ev_pair[0] is not None:
+                ev_pair[0][0].record(stream)
+            M.spmv_scatter(x, ptrs, off, y=y, alpha=alpha, beta=beta, stream=stream)
+            if ev_pair[0] is not None:
+                ev_pair[0][1].record(stream)
+
+    if args.exchange == "fused":
+        if args.hybrid:
+            raise SystemExit("--exchange fused needs pure bitBSR (no --hybrid)")
+        it = FusedIteratedSpMV(wl.part, wl.n, _Timed(), wl.x0, rank)
+    else:
+        it = IteratedSpMV(wl.part, wl.n, local_spmv, wl.x0, rank)
 
     for _ in range(max(3, args.warmup)):
         it.step(wl.alpha, wl.c)
@@ -456,7 +472,10 @@ def main():
                        "fill_rank0": wl.local_nnz / max(1, info.Bnnz),
                        "values": args.dtype, "hybrid_residual_max_popc": args.hybrid,
                        "residual_nnz_rank0": int(info.residual_nnz),
-                       "parallelism": f"row-partition x{world}" + (" + NCCL all-gather" if world > 1 else ""),
+                       "parallelism": f"row-partition x{world}" + (
+                           (" + NCCL all-gather" if args.exchange == "nccl" else " + fused peer-store all-gather")
+                           if world > 1 else ""),
+                       "exchange": args.exchange,
                        "l2": "inputs larger than L2 (A > 126 MB), no flush" if info.format_bytes > 126e6
                              else "matrix fits L2 (no flush): warm-L2 number",
                        "step": wl.step_desc},

@@ -167,6 +167,26 @@ SPADEN_API spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const flo
                             float *d_y, void *stream);
 
 /*
+ * spaden_spmv_scatter -- fused SpMV + all-gather epilogue
+ * for row-partitioned iterated SpMV: computes this rank's slice
+ * y = alpha * A x + beta * y (A = the rank's row slice, global columns) and stores
+ * every y value straight into each destination buffer:
+ *   h_out_ptrs[p][out_offset + i] = y_i   for p < npeers, i < m
+ * from the SpMV epilogue (plain stores; on a multi-GPU node the pointers are the
+ * NVLink-mapped next-x buffers of every rank, e.g. torch symmetric memory peer
+ * pointers, including this rank's own), so the exchange overlaps the compute
+ * tile by tile instead of following it as a separate collective.  The caller
+ * adds the cross-GPU barrier before the buffers are read.  Values are bitwise
+ * identical to spaden_spmv.
+ *   h_out_ptrs  HOST array of npeers device pointers (1 <= npeers <= 8).
+ *   d_y         local y (read if beta != 0, also written if non-NULL; may be NULL).
+ * Requires a pure bitBSR handle (no hybrid residual).
+ */
+SPADEN_API spaden_status_t spaden_spmv_scatter(spaden_matrix_t A, float alpha, const float *d_x, float beta,
+                                               float *d_y, float *const *h_out_ptrs, int32_t npeers,
+                                               int64_t out_offset, void *stream);
+
+/*
  * spaden_spmm -- k products at once (SURVEY.md §8(f) NEXT-4, P:L336 future work):
  * Y[:, j] = alpha * A X[:, j] + beta * Y[:, j] for j < k, with column-major device
  * matrices: vector j of X at d_X + j*ldx (ldx >= n), of Y at d_Y + j*ldy (ldy >= m).

@@ -71,6 +71,9 @@ spaden_convert_csr_to_bitmap_ex.restype = _ST
 spaden_spmv = _lib.spaden_spmv
 spaden_spmv.argtypes = [_P, _F, _P, _F, _P, _P]
 spaden_spmv.restype = _ST
+spaden_spmv_scatter = _lib.spaden_spmv_scatter
+spaden_spmv_scatter.argtypes = [_P, _F, _P, _F, _P, ctypes.POINTER(_P), ctypes.c_int32, _I64, _P]
+spaden_spmv_scatter.restype = _ST
 spaden_spmm = _lib.spaden_spmm
 spaden_spmm.argtypes = [_P, _F, _P, _I64, ctypes.c_int32, _F, _P, _I64, _P]
 spaden_spmm.restype = _ST
@@ -99,7 +102,8 @@ spaden_version = _lib.spaden_version
 spaden_version.argtypes = []
 spaden_version.restype = ctypes.c_char_p
 
-EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_spmv", "spaden_spmm", "spaden_spmv_host", "spaden_spmv_host_batched",
+EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_spmv", "spaden_spmm",
+            "spaden_spmv_scatter", "spaden_spmv_host", "spaden_spmv_host_batched",
             "spaden_free",
             "spaden_get_info", "spaden_get_arrays", "spaden_status_string",
             "spaden_last_error_message", "spaden_version"]
@@ -211,6 +215,20 @@ class Matrix:
         _check(spaden_spmv(self._h, alpha, ctypes.c_void_p(x.data_ptr()), beta,
                            ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream)), "spaden_spmv")
         return y
+
+    def spmv_scatter(self, x, out_ptrs, out_offset: int, y=None, alpha: float = 1.0, beta: float = 0.0,
+                     stream=None):
+        """Fused SpMV + all-gather store: y values written to every out_ptrs[p] + out_offset
+        (device addresses as ints, e.g. symmetric-memory peer buffers)."""
+        torch = _torch()
+        assert x.dtype == torch.float32 and x.is_cuda and x.is_contiguous() and x.numel() == self.n
+        if y is not None:
+            assert y.dtype == torch.float32 and y.is_cuda and y.is_contiguous() and y.numel() == self.m
+        arr = (ctypes.c_void_p * len(out_ptrs))(*[ctypes.c_void_p(int(p)) for p in out_ptrs])
+        _check(spaden_spmv_scatter(self._h, alpha, ctypes.c_void_p(x.data_ptr()), beta,
+                                   ctypes.c_void_p(y.data_ptr()) if y is not None else None,
+                                   ctypes.cast(arr, ctypes.POINTER(ctypes.c_void_p)), len(out_ptrs),
+                                   int(out_offset), _stream_ptr(stream)), "spaden_spmv_scatter")
 
     def spmm(self, X, Y=None, alpha: float = 1.0, beta: float = 0.0, stream=None):
         """Y[j] = alpha * A X[j] + beta * Y[j] for the rows j of X (k x n, CUDA float32,

@@ -186,6 +186,26 @@ spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const float *d_x, fl
     return spmv_launch(*A, alpha, d_x, beta, d_y, (cudaStream_t)stream);
 }
 
+spaden_status_t spaden_spmv_scatter(spaden_matrix_t A, float alpha, const float *d_x, float beta, float *d_y,
+                                    float *const *h_out_ptrs, int32_t npeers, int64_t out_offset, void *stream) {
+    if (!A || npeers < 1 || npeers > kMaxPeers || !h_out_ptrs || out_offset < 0 ||
+        (A->Bnnz > 0 && !d_x) || (beta != 0.f && A->m > 0 && !d_y)) {
+        set_error("bad arguments (handle, 1 <= npeers <= 8, out pointers, x, y with beta != 0)");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    PeerOut po{};
+    for (int p = 0; p < npeers; ++p) {
+        if (!h_out_ptrs[p]) {
+            set_error("NULL destination pointer");
+            return SPADEN_ERR_INVALID_ARGUMENT;
+        }
+        po.ptr[p] = h_out_ptrs[p];
+    }
+    po.n = npeers;
+    po.offset = out_offset;
+    return spmv_launch(*A, alpha, d_x, beta, d_y, (cudaStream_t)stream, &po);
+}
+
 spaden_status_t spaden_spmm(spaden_matrix_t A, float alpha, const float *d_X, int64_t ldx, int32_t k, float beta,
                             float *d_Y, int64_t ldy, void *stream) {
     if (!A || k < 0 || ldx < A->n || ldy < A->m || (k > 0 && ((A->m > 0 && !d_Y) || (A->Bnnz > 0 && !d_X)))) {

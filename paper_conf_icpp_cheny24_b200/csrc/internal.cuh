@@ -138,6 +138,17 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t stream);
 spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t stream);
 
 
+// Fused SpMV + all-gather: besides (or instead of) y,
+// every y value is stored at ptr[p][offset + row] for each of the n peer
+// buffers (NVLink-mapped x_next slices of the other GPUs, plus the local one).
+constexpr int kMaxPeers = 8;
+struct PeerOut {
+    float *ptr[kMaxPeers];
+    int32_t n;
+    int32_t pad;
+    int64_t offset;
+};
+
 // converter (convert.cu)
 spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *rowptr,
                             const int32_t *colidx, const void *values, spaden_dtype_t vdt,
@@ -149,7 +160,7 @@ cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y
 
 // SpMV (spmv.cu)
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,
-                            cudaStream_t stream);
+                            cudaStream_t stream, const PeerOut *peers = nullptr);
 // SpMM: k column-major vectors (spmv.cu)
 spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx, int k, float beta, float *Y,
                             int64_t ldy, cudaStream_t stream);

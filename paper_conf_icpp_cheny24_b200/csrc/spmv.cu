@@ -273,11 +273,25 @@ __device__ __forceinline__ void block_bits(uint2 bm, typename VS::P p, const flo
     }
 }
 
+// Final store of y[row]: local y, and/or the peer buffers of the fused
+// all-gather (plain st.global through NVLink-mapped addresses).
+__device__ __forceinline__ void store_y(float *__restrict__ y, int64_t row, float o, const PeerOut &po) {
+    if (po.n == 0) {
+        y[row] = o;
+        return;
+    }
+    if (y) y[row] = o;
+#pragma unroll
+    for (int p = 0; p < kMaxPeers; ++p)
+        if (p < po.n) po.ptr[p][po.offset + row] = o;
+}
+
 // Phase 2: y for every block-row of a tile from the per-block row partials
 // (9-word stride), 4 block-rows x 8 rows per warp pass, 4 chains per row
 // indexed by block position within the block-row, combined (c0+c1)+(c2+c3).
 __device__ __forceinline__ void reduce_tile(uint32_t a_rp, uint32_t a_part, int nbr, int b0, int br0, int lane,
-                                            int64_t m, float alpha, float beta, float *__restrict__ y) {
+                                            int64_t m, float alpha, float beta, float *__restrict__ y,
+                                            const PeerOut &po) {
     const int r = lane & 7;
     for (int base = 0; base < nbr; base += 4) {
         const int brl = base + (lane >> 3);
@@ -301,7 +315,7 @@ __device__ __forceinline__ void reduce_tile(uint32_t a_rp, uint32_t a_part, int 
             if (row < m) {
                 float o = alpha * sum;
                 if (beta != 0.f) o = fmaf(beta, y[row], o);
-                y[row] = o;
+                store_y(y, row, o, po);
             }
         }
     }
@@ -482,7 +496,8 @@ __global__ void __launch_bounds__(32 * (CONSUMERS + 1), MINB)
 k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int ntiles, const int32_t *__restrict__ blk_rowptr,
              const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
              const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
-             int nbc_vec, float alpha, float beta, float *__restrict__ y, int64_t ldx = 0, int64_t ldy = 0) {
+             int nbc_vec, float alpha, float beta, float *__restrict__ y, int64_t ldx, int64_t ldy,
+             const PeerOut po) {
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t full_bar[kMaxStages], empty_bar[kMaxStages];
     __shared__ StageHdr hdr[kMaxStages];
@@ -688,7 +703,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                 if constexpr (K > 1)
                     reduce_tile_k<K>((uint32_t)h2.w, a_part, h0.y, h0.z, h0.x, lane, m, alpha, beta, y, ldy);
                 else
-                    reduce_tile((uint32_t)h2.w, a_part, h0.y, h0.z, h0.x, lane, m, alpha, beta, y);
+                    reduce_tile((uint32_t)h2.w, a_part, h0.y, h0.z, h0.x, lane, m, alpha, beta, y, po);
             }
         }
         __syncwarp();
@@ -807,7 +822,7 @@ k_spmv_warp(int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int 
             }
         }
         __syncwarp();
-        reduce_tile(a_rp, a_part, nbr, b0, br0, lane, m, alpha, beta, y);  // phase 2
+        reduce_tile(a_rp, a_part, nbr, b0, br0, lane, m, alpha, beta, y, PeerOut{});  // phase 2
         __syncwarp();
     }
 }
@@ -865,7 +880,7 @@ k_spmv_long_chunks(int nchunks, const int32_t *__restrict__ long_rows, const int
 
 __global__ void k_spmv_long_fixup(int64_t m, int nlong, const int32_t *__restrict__ long_rows,
                                   const int32_t *__restrict__ chunk_start, const float *__restrict__ carry, float alpha,
-                                  float beta, float *__restrict__ y) {
+                                  float beta, float *__restrict__ y, const PeerOut po) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= 8 * (int64_t)nlong) return;
     const int j = (int)(t >> 3), r = (int)(t & 7);
@@ -875,7 +890,7 @@ __global__ void k_spmv_long_fixup(int64_t m, int nlong, const int32_t *__restric
     if (row < m) {
         float o = alpha * sum;
         if (beta != 0.f) o = fmaf(beta, y[row], o);
-        y[row] = o;
+        store_y(y, row, o, po);
     }
 }
 
@@ -900,7 +915,7 @@ int sm_count() {
 
 template <typename V, int DEC, int CONSUMERS, int MINB>
 cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, const float *x, float beta,
-                             float *y, cudaStream_t st) {
+                             float *y, cudaStream_t st, const PeerOut &po) {
     const int nbc_vec = ((uintptr_t)x & 31u) == 0 ? (int)(A.n / 8) : 0;
     const size_t smem = (size_t)cfg.stages * cfg.stage_bytes;
     static size_t occ_smem = 0;  // resident CTAs per SM (registers, smem), cached per smem size
@@ -918,7 +933,7 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
         const int grid = (int)std::min<int64_t>(A.n_tiles, (int64_t)sm_count() * occ);
         k_spmv_tiled<V, DEC, CONSUMERS, MINB><<<grid, 32 * (CONSUMERS + 1), smem, st>>>(
             cfg.stages, cfg.stage_bytes, A.m, A.tiles, (int)A.n_tiles, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y);
+            A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y, 0, 0, po);
     }
     if (A.n_long > 0) {
         const int64_t threads = 32 * A.n_chunks;
@@ -926,7 +941,7 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
             (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
             A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry);
         k_spmv_long_fixup<<<(unsigned)((8 * A.n_long + 255) / 256), 256, 0, st>>>(
-            A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y);
+            A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, po);
     }
     return cudaGetLastError();
 }
@@ -959,25 +974,26 @@ cudaError_t launch_warp_cfg(const Matrix &A, const TileCfg &cfg, float alpha, co
             (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
             A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry);
         k_spmv_long_fixup<<<(unsigned)((8 * A.n_long + 255) / 256), 256, 0, st>>>(
-            A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y);
+            A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, PeerOut{});
     }
     return cudaGetLastError();
 }
 
 template <typename V, int DEC>
-cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st) {
+cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st,
+                         const PeerOut &po) {
     const TileCfg cfg = tile_cfg(A.tile_cfg);
     switch (A.tile_cfg) {
     case 4: return launch_warp_cfg<V, DEC, 4, 2>(A, cfg, alpha, x, beta, y, st);
-    case 5: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st);
-    case 6: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st);
-    case 7: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
-    case 8: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
-    case 9: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
-    case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st);
-    case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st);
-    case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st);
-    default: return launch_tiled_cfg<V, DEC, 16, 1>(A, cfg, alpha, x, beta, y, st);
+    case 5: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po);
+    case 6: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po);
+    case 7: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
+    case 8: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
+    case 9: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
+    case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po);
+    case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po);
+    case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
+    default: return launch_tiled_cfg<V, DEC, 16, 1>(A, cfg, alpha, x, beta, y, st, po);
     }
 }
 
@@ -1002,7 +1018,7 @@ cudaError_t launch_spmm_cfg(const Matrix &A, const TileCfg &cfg, const TileDesc 
         const int grid = (int)std::min<int64_t>(ntiles, (int64_t)sm_count() * occ);
         k_spmv_tiled<V, 1, CONSUMERS, MINB, K><<<grid, 32 * (CONSUMERS + 1), smem, st>>>(
             cfg.stages, cfg.stage_bytes, A.m, tiles, (int)ntiles, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, X, nbc_vec, alpha, beta, Y, ldx, ldy);
+            A.blk_offset, (const V *)A.values, X, nbc_vec, alpha, beta, Y, ldx, ldy, PeerOut{});
     }
     if (A.n_long > 0) {  // long block-rows: the SpMV chunk path, once per vector (same arithmetic)
         const int nbc1 = ((uintptr_t)X & 31u) == 0 && ((ldx * 4) % 32) == 0 ? (int)(A.n / 8) : 0;
@@ -1012,7 +1028,7 @@ cudaError_t launch_spmm_cfg(const Matrix &A, const TileCfg &cfg, const TileDesc 
                 (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
                 A.blk_offset, (const V *)A.values, X + j * ldx, nbc1, A.carry);
             k_spmv_long_fixup<<<(unsigned)((8 * A.n_long + 255) / 256), 256, 0, st>>>(
-                A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, Y + j * ldy);
+                A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, Y + j * ldy, PeerOut{});
         }
     }
     return cudaGetLastError();
@@ -1070,10 +1086,15 @@ spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx,
 }
 
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,
-                            cudaStream_t st) {
+                            cudaStream_t st, const PeerOut *peers) {
     if (A.m == 0) return SPADEN_OK;
     const bool x_vec = ((uintptr_t)x & 15u) == 0;
-    if (kernel_variant() == 0) {
+    const PeerOut po = peers ? *peers : PeerOut{};
+    if (po.n > 0 && (A.res_nnz > 0 || tile_cfg(A.tile_cfg).warp_mode)) {
+        set_error("the fused all-gather store needs pure bitBSR and a CTA-pipeline tile config");
+        return SPADEN_ERR_UNSUPPORTED;
+    }
+    if (kernel_variant() == 0 && po.n == 0) {
         const int threads = 256;
         const int64_t want = (A.Bnrow + 7) / 8;
         const unsigned grid = (unsigned)std::min<int64_t>(want, 148LL * 64);
@@ -1105,20 +1126,20 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
     cudaError_t e;
     if (A.storage == SPADEN_R_16F) {
         switch (dec) {
-        case 0: e = launch_tiled<__half, 0>(A, alpha, x, beta, y, st); break;
-        case 2: e = launch_tiled<__half, 2>(A, alpha, x, beta, y, st); break;
-        case 4: e = launch_tiled<__half, 4>(A, alpha, x, beta, y, st); break;
-        case 5: e = launch_tiled<__half, 5>(A, alpha, x, beta, y, st); break;
-        case 6: e = launch_tiled<__half, 6>(A, alpha, x, beta, y, st); break;
-        default: e = launch_tiled<__half, 1>(A, alpha, x, beta, y, st);
+        case 0: e = launch_tiled<__half, 0>(A, alpha, x, beta, y, st, po); break;
+        case 2: e = launch_tiled<__half, 2>(A, alpha, x, beta, y, st, po); break;
+        case 4: e = launch_tiled<__half, 4>(A, alpha, x, beta, y, st, po); break;
+        case 5: e = launch_tiled<__half, 5>(A, alpha, x, beta, y, st, po); break;
+        case 6: e = launch_tiled<__half, 6>(A, alpha, x, beta, y, st, po); break;
+        default: e = launch_tiled<__half, 1>(A, alpha, x, beta, y, st, po);
         }
     } else {  // (the tensor-core ablation exists for fp16 values only)
         switch (dec) {
-        case 0: e = launch_tiled<float, 0>(A, alpha, x, beta, y, st); break;
-        case 2: e = launch_tiled<float, 2>(A, alpha, x, beta, y, st); break;
-        case 5: e = launch_tiled<float, 5>(A, alpha, x, beta, y, st); break;
-        case 6: e = launch_tiled<float, 6>(A, alpha, x, beta, y, st); break;
-        default: e = launch_tiled<float, 1>(A, alpha, x, beta, y, st);
+        case 0: e = launch_tiled<float, 0>(A, alpha, x, beta, y, st, po); break;
+        case 2: e = launch_tiled<float, 2>(A, alpha, x, beta, y, st, po); break;
+        case 5: e = launch_tiled<float, 5>(A, alpha, x, beta, y, st, po); break;
+        case 6: e = launch_tiled<float, 6>(A, alpha, x, beta, y, st, po); break;
+        default: e = launch_tiled<float, 1>(A, alpha, x, beta, y, st, po);
         }
     }
     if (e == cudaSuccess) e = residual_spmv(A, alpha, x, y, st);  // hybrid residual (if any)

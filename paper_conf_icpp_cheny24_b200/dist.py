@@ -10,6 +10,11 @@ gloo in the CPU tests) -- the only exchange step the method has.  Because every
 block-row's summation order depends only on that block-row, the gathered
 vector is bitwise equal to the single-GPU result.
 
+``FusedIteratedSpMV`` removes the separate collective:
+each rank's SpMV epilogue stores its slice straight into every rank's next-x
+buffer (``spaden_spmv_scatter``; peer pointers from torch symmetric memory, i.e.
+NVLink-mapped allocations), followed by one device-side barrier per iteration.
+
 Nothing here computes: the SpMV is passed in (the CUDA path in production, the
 oracle in the CPU tests).
 """
@@ -86,3 +91,91 @@ class IteratedSpMV:
         gather_slices(self.x_next[: self.part.padded], slot, self.group)
         self.x, self.x_next = self.x_next, self.x
         return self.x
+
+
+class FusedIteratedSpMV:
+    """Iterated SpMV with the all-gather fused into the SpMV epilogue (NEXT-2).
+
+    Two x buffers (ping/pong), each replicated on every rank.  ``bufs[k][p]`` is
+    rank p's copy of buffer k as seen from this rank (a peer tensor).  One step
+    reads ``bufs[cur][rank][:n]`` and, through ``matrix.spmv_scatter``, writes
+    rows [r0, r1) of y into ``bufs[1-cur][p][r0:r1]`` for every p; then
+    ``barrier()``.  The single barrier per step covers both hazards: every slot
+    of the next x is written before anyone reads it, and no rank writes into a
+    buffer (step k+1 targets bufs[cur]) that a slower rank is still reading.
+
+    ``matrix`` needs ``spmv_scatter(x, out_ptrs, out_offset, y=, alpha=, beta=)``.
+    ``buffers`` = (bufs0, bufs1, barrier) injects the peer views (tests emulate
+    several ranks on one device); by default they come from torch symmetric
+    memory (world > 1) or are local tensors (world == 1 / no process group).
+    """
+
+    def __init__(self, part: RowPartition, n: int, matrix, x0, rank: int, group=None, buffers=None):
+        import torch
+
+        self.part, self.n, self.rank, self.group = part, n, rank, group
+        self.matrix = matrix
+        self.r0, self.r1 = part.range(rank)
+        L = max(part.padded, n)
+        if buffers is None:
+            buffers = _symmetric_buffers(L, part.world, rank, group, x0.device)
+        self.bufs = [list(buffers[0]), list(buffers[1])]
+        self.barrier = buffers[2]
+        if len(self.bufs[0]) != part.world or len(self.bufs[1]) != part.world:
+            raise ValueError("need one peer view per rank")
+        if part.world > 8:
+            raise ValueError("spaden_spmv_scatter stores to at most 8 peers (one node)")
+        self.cur = 0
+        own = self.bufs[0][rank]
+        own.zero_()
+        own[: x0.numel()].copy_(x0)
+        self.barrier()
+        del torch
+
+    @property
+    def x(self):
+        return self.bufs[self.cur][self.rank]
+
+    def step(self, alpha: float = 1.0, c: float | None = None):
+        dst = self.bufs[1 - self.cur]
+        y, beta = None, 0.0
+        if c is not None:
+            y = dst[self.rank][self.r0:self.r1]
+            y.fill_(c)
+            beta = 1.0
+        if self.r1 > self.r0:
+            self.matrix.spmv_scatter(self.x[: self.n], [t.data_ptr() for t in dst], self.r0,
+                                     y=y, alpha=alpha, beta=beta)
+        self.barrier()
+        self.cur = 1 - self.cur
+        return self.x
+
+
+def _symmetric_buffers(L: int, world: int, rank: int, group, device):
+    """Two length-L fp32 buffers visible to every rank (peer views) + a barrier."""
+    import torch
+    import torch.distributed as dist
+
+    if world == 1 or not (dist.is_available() and dist.is_initialized()):
+        if world != 1:
+            raise RuntimeError("world > 1 needs an initialised process group")
+        a = torch.zeros(L, dtype=torch.float32, device=device)
+        b = torch.zeros(L, dtype=torch.float32, device=device)
+        return [a], [b], (lambda: None)
+    import torch.distributed._symmetric_memory as symm_mem
+
+    grp = group if group is not None else dist.group.WORLD
+    views = []
+    handles = []
+    for _ in range(2):
+        t = symm_mem.empty(L, dtype=torch.float32, device=device)
+        h = symm_mem.rendezvous(t, grp)
+        handles.append((t, h))
+        views.append([t if p == rank else h.get_buffer(p, (L,), torch.float32) for p in range(world)])
+    h0 = handles[0][1]
+
+    def barrier():
+        h0.barrier(channel=0)
+
+    barrier._keepalive = handles  # the allocations must outlive the views
+    return views[0], views[1], barrier

@@ -103,3 +103,43 @@ def test_single_process_without_process_group():
     x = it.step(0.01)
     ys, _ = oracle.spmv(A.rowptr, A.colidx, A.values, x0.numpy())
     assert np.array_equal(x[: A.n].numpy(), (0.01 * ys).astype(np.float32))
+
+
+class _HostScatterSlice:
+    """CPU stand-in for Matrix.spmv_scatter: the oracle computes the slice, the
+    result is stored through raw host addresses like the kernel's peer stores."""
+
+    def __init__(self, S):
+        self.S = S
+
+    def spmv_scatter(self, x, out_ptrs, out_offset, y=None, alpha=1.0, beta=0.0):
+        import ctypes
+        ys, _ = oracle.spmv(self.S.rowptr, self.S.colidx, self.S.values, x.numpy())
+        out = alpha * ys + (beta * y.numpy().astype(np.float64) if beta != 0 else 0.0)
+        out = np.ascontiguousarray(out.astype(np.float32))
+        for p in out_ptrs:
+            ctypes.memmove(p + 4 * out_offset, out.ctypes.data, out.nbytes)
+        if y is not None:
+            y.copy_(torch.from_numpy(out))
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 5])
+def test_fused_iterated_host_logic(world):
+    """FusedIteratedSpMV's offsets, ping-pong and peer list (ranks emulated in one
+    process, stepped in turn) reproduce the unfused single-rank iteration."""
+    from paper_conf_icpp_cheny24_b200.dist import FusedIteratedSpMV, IteratedSpMV, RowPartition
+    src, dst = W.rmat_edges(9, 8, seed=5, relabel=True)
+    A = W.pagerank_matrix(512, src, dst)
+    x0 = torch.full((A.n,), 1.0 / A.n)
+    ref = IteratedSpMV(RowPartition(A.m, 1), A.n, oracle_local_spmv(A), x0, 0)
+    part = RowPartition(A.m, world)
+    L = max(part.padded, A.n)
+    bufs = ([torch.zeros(L) for _ in range(world)], [torch.zeros(L) for _ in range(world)])
+    ranks = [FusedIteratedSpMV(part, A.n, _HostScatterSlice(A.row_slice(*part.range(r))), x0, r,
+                               buffers=(*bufs, lambda: None)) for r in range(world)]
+    for _ in range(5):
+        xr = ref.step(0.85, 0.15 / A.n)
+        for rk in ranks:
+            rk.step(0.85, 0.15 / A.n)
+        for rk in ranks:
+            assert torch.equal(rk.x[: A.n], xr[: A.n])

@@ -598,3 +598,84 @@ def test_spmm_hybrid(sp, torch):
     Y = M.spmm(X)
     for j in range(4):
         assert torch.equal(Y[j], M.spmv(X[j].contiguous()))
+
+
+@pytest.mark.parametrize("npeers", [1, 3, 8])
+@pytest.mark.parametrize("name", ["fem", "hub", "tiny", "h2", "empty"])
+@pytest.mark.parametrize("storage", ["fp32", "fp16"])
+def test_spmv_scatter_virtual_peers(sp, torch, npeers, name, storage):
+    """NEXT-2 fused SpMV + all-gather store: every destination buffer ("virtual
+    peers" on one GPU) receives y at out_offset bitwise equal to spaden_spmv,
+    nothing outside [offset, offset+m) is touched, and the local y is written
+    too when given (alpha/beta honoured)."""
+    A = {"fem": lambda: W.fem(7, 8, 9, seed=6), "hub": hub_matrix, "tiny": lambda: W.tiny(2), "h2": W.h2,
+         "empty": lambda: W.from_coo(17, 5, [], [], [])}[name]()
+    M = convert(sp, torch, A, storage=storage)
+    x = torch.from_numpy(W.vector(A.n, 61)).cuda()
+    y0 = torch.from_numpy(W.vector(A.m, 62)).cuda()
+    off = 13
+    total = A.m + off + 29
+    bufs = [torch.full((total,), float(p) - 7.0, device="cuda") for p in range(npeers)]
+    y = y0.clone()
+    M.spmv_scatter(x, [b.data_ptr() for b in bufs], off, y=y, alpha=0.75, beta=0.5)
+    ref = M.spmv(x, y0.clone(), alpha=0.75, beta=0.5)
+    torch.cuda.synchronize()
+    assert torch.equal(y, ref)
+    for p, b in enumerate(bufs):
+        assert torch.equal(b[off:off + A.m], ref), p
+        assert bool((b[:off] == float(p) - 7.0).all()) and bool((b[off + A.m:] == float(p) - 7.0).all())
+    # beta == 0 without a local y: peers only
+    bufs2 = [torch.zeros(total, device="cuda") for _ in range(npeers)]
+    M.spmv_scatter(x, [b.data_ptr() for b in bufs2], off)
+    torch.cuda.synchronize()
+    ref0 = M.spmv(x)
+    for b in bufs2:
+        assert torch.equal(b[off:off + A.m], ref0)
+
+
+def test_spmv_scatter_rejects(sp, torch):
+    A = W.tiny(1)
+    M = convert(sp, torch, A)
+    x = torch.from_numpy(W.vector(A.n, 1)).cuda()
+    b = torch.zeros(A.m, device="cuda")
+    with pytest.raises(sp.SpadenError):
+        M.spmv_scatter(x, [b.data_ptr()] * 9, 0)
+    with pytest.raises(sp.SpadenError):
+        M.spmv_scatter(x, [b.data_ptr()], 0, beta=0.5)          # beta != 0 needs y
+    H = hub_matrix()
+    rp, ci, v = dev(torch, H)
+    Mh = sp.convert(rp, ci, v, H.n, residual_max_popc=2)
+    bh = torch.zeros(H.m, device="cuda")
+    with pytest.raises(sp.SpadenError):                          # hybrid: unsupported
+        Mh.spmv_scatter(torch.from_numpy(W.vector(H.n, 1)).cuda(), [bh.data_ptr()], 0)
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+def test_fused_iterated_spmv_emulated_ranks(sp, torch, world):
+    """dist.FusedIteratedSpMV with `world` ranks emulated on one GPU (peer views =
+    plain device buffers, stepped rank by rank): after every PageRank-style step
+    each rank's x is bitwise equal to the unfused single-rank IteratedSpMV."""
+    from paper_conf_icpp_cheny24_b200 import dist
+    src, dst = W.rmat_edges(12, 8, seed=5, relabel=True)
+    A = W.pagerank_matrix(1 << 12, src, dst)
+    x0 = torch.full((A.n,), 1.0 / A.n, device="cuda")
+    alpha, c = 0.85, 0.15 / A.n
+    full = convert(sp, torch, A)
+    ref = dist.IteratedSpMV(dist.RowPartition(A.m, 1), A.n,
+                            lambda x, y, a, b: full.spmv(x, y, alpha=a, beta=b), x0, 0)
+    part = dist.RowPartition(A.m, world)
+    L = max(part.padded, A.n)
+    bufs = ([torch.zeros(L, device="cuda") for _ in range(world)],
+            [torch.zeros(L, device="cuda") for _ in range(world)])
+    ranks = []
+    for r in range(world):
+        r0, r1 = part.range(r)
+        M = convert(sp, torch, A.row_slice(r0, r1))
+        ranks.append(dist.FusedIteratedSpMV(part, A.n, M, x0, r, buffers=(*bufs, lambda: None)))
+    for _ in range(6):
+        xr = ref.step(alpha, c)
+        for rk in ranks:
+            rk.step(alpha, c)
+        torch.cuda.synchronize()
+        for rk in ranks:
+            assert torch.equal(rk.x[: A.n], xr[: A.n])
