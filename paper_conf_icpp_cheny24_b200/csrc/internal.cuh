@@ -113,7 +113,7 @@ __host__ __device__ inline TileCfg tile_cfg(int i) {
     default: return TileCfg{1, 16, 3, 64 * 1024, 0};
     }
 }
-int default_tile_cfg(int64_t format_bytes);  // SPADEN_TILE_CFG override, else by matrix size
+int default_tile_cfg(int64_t format_bytes, int value_bytes);  // SPADEN_TILE_CFG override, else by matrix size
 constexpr int kStageSlack = 384;
 constexpr int64_t kSmallMatrixBytes = 64ll << 20;  // below: kSmallTileCfg
 constexpr int kSmallTileCfg = 3;  // measured: smaller stages do not help fem62k

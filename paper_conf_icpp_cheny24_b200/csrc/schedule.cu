@@ -111,12 +111,14 @@ __global__ void k_sched_summary(const int32_t *tile_total, const int32_t *long_t
 
 }  // namespace
 
-int default_tile_cfg(int64_t format_bytes) {
+int default_tile_cfg(int64_t format_bytes, int value_bytes) {
     const char *e = getenv("SPADEN_TILE_CFG");
     if (e && e[0] >= '0' && e[0] <= '9' && e[0] - '0' < kNumTileCfgs) return e[0] - '0';
-    // measured best on fem1p5m: 4 CTAs/SM x 8 consumers x 2 x 27 KB;
-    // small matrices need smaller stages to give every CTA several tiles
-    return format_bytes >= kSmallMatrixBytes ? 3 : kSmallTileCfg;
+    // measured best on fem1p5m: fp32 values 3 CTAs/SM x 8 consumers
+    // x 3 x 24 KB, fp16 values 4 x 8 x 2 x 27 KB; small matrices need smaller stages to
+    // give every CTA several tiles
+    if (format_bytes < kSmallMatrixBytes) return kSmallTileCfg;
+    return value_bytes == 4 ? 2 : 3;
 }
 
 spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
@@ -124,7 +126,7 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     const int sv = A->storage == SPADEN_R_16F ? 2 : 4;
     const int64_t nseg = (Bnrow + kSeg - 1) / kSeg;
     const int sv_b = A->storage == SPADEN_R_16F ? 2 : 4;
-    A->tile_cfg = default_tile_cfg(4 * (A->Bnrow + 1) + 16 * A->Bnnz + (int64_t)sv_b * A->nnz);
+    A->tile_cfg = default_tile_cfg(4 * (A->Bnrow + 1) + 16 * A->Bnnz + (int64_t)sv_b * A->nnz, sv_b);
     const TileCfg cfg = tile_cfg(A->tile_cfg);
     const int64_t cap = cfg.stage_bytes - kStageSlack;
     // CTA pipelines: rows above half a stage are long (keeps tiles well packed);

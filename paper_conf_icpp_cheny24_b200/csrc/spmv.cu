@@ -17,6 +17,7 @@
 // instead of loading from memory"): structural zeros are never
 // multiplied (reading R11).  x[8bc .. 8bc+7] is the block's 8-element segment
 // (Alg. 2 lines 7-10).
+#include <mutex>
 #include <cstdlib>
 
 #include "internal.cuh"
@@ -210,9 +211,19 @@ struct XSeg {
 // nbc_vec = number of leading block columns whose x segment may be read as one
 // 32-byte vector (n/8 when x is 32-byte aligned, else 0); other segments read only the
 // columns referenced by `cols` (bit c set = column c used by the block).
-__device__ __forceinline__ void load_x(XSeg &xs, const float *__restrict__ x, int bc, int nbc_vec, uint32_t cols) {
+// texx != 0: x is also bound to a 1-D float4 texture; aligned segments are then
+// fetched through the texture pipe (TLD), which has its own L1TEX data path, so
+// the LSU data pipe -- the kernel's bottleneck, saturated by the shared-memory
+// value loads -- only carries smem traffic.
+__device__ __forceinline__ void load_x(XSeg &xs, const float *__restrict__ x, int bc, int nbc_vec, uint32_t cols,
+                                       unsigned long long texx = 0ull, int tex_off = 0) {
     const float *p = x + 8 * (int64_t)bc;
-    if (bc < nbc_vec) {  // one 32-byte sector, one 256-bit load (LDG.E.ENL2.256)
+    if (texx && bc < nbc_vec) {  // tex_off: float4 index of x in the texture (SpMM vector j)
+        const float4 a = tex1Dfetch<float4>((cudaTextureObject_t)texx, tex_off + 2 * bc);
+        const float4 b = tex1Dfetch<float4>((cudaTextureObject_t)texx, tex_off + 2 * bc + 1);
+        xs.v[0] = a.x, xs.v[1] = a.y, xs.v[2] = a.z, xs.v[3] = a.w;
+        xs.v[4] = b.x, xs.v[5] = b.y, xs.v[6] = b.z, xs.v[7] = b.w;
+    } else if (bc < nbc_vec) {  // one 32-byte sector, one 256-bit load (LDG.E.ENL2.256)
         asm("ld.global.nc.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
             : "=f"(xs.v[0]), "=f"(xs.v[1]), "=f"(xs.v[2]), "=f"(xs.v[3]), "=f"(xs.v[4]), "=f"(xs.v[5]),
               "=f"(xs.v[6]), "=f"(xs.v[7])
@@ -235,6 +246,42 @@ __device__ __forceinline__ uint32_t used_cols(uint2 bm) {
 // rows are independent dependency chains of at most 8 slots.
 template <class VS>
 __device__ __forceinline__ void block_slots(uint2 bm, typename VS::P p0, const XSeg &xs, float acc[8]) {
+#ifdef SPADEN_EXP_BATCH  // loads of RB rows issued before their fma chains (independent registers)
+    constexpr int RB = SPADEN_EXP_BATCH;
+    const int plo0 = __popc(bm.x);
+#pragma unroll
+    for (int r0 = 0; r0 < 8; r0 += RB) {
+        float v[RB][8];
+#pragma unroll
+        for (int rr = 0; rr < RB; ++rr) {
+            const int r = r0 + rr;
+            const uint32_t w = r < 4 ? bm.x : bm.y;
+            const uint32_t byte = (w >> (8 * (r & 3))) & 0xffu;
+            const int below = ((r & 3) == 0 ? 0 : __popc(w & ((1u << (8 * (r & 3))) - 1u))) + (r < 4 ? 0 : plo0);
+            typename VS::P p = p0 + below * VS::step;
+#pragma unroll
+            for (int c = 0; c < 8; ++c) {
+                v[rr][c] = 0.f;
+                if ((byte >> c) & 1u) {
+                    v[rr][c] = VS::get(p);
+                    p += VS::step;
+                }
+            }
+        }
+#pragma unroll
+        for (int rr = 0; rr < RB; ++rr) {
+            const int r = r0 + rr;
+            const uint32_t w = r < 4 ? bm.x : bm.y;
+            const uint32_t byte = (w >> (8 * (r & 3))) & 0xffu;
+            float a = 0.f;
+#pragma unroll
+            for (int c = 0; c < 8; ++c)
+                if ((byte >> c) & 1u) a = fmaf(v[rr][c], xs.v[c], a);
+            acc[r] = a;
+        }
+    }
+    return;
+#endif
     const int plo = __popc(bm.x);
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
@@ -246,7 +293,14 @@ __device__ __forceinline__ void block_slots(uint2 bm, typename VS::P p0, const X
 #pragma unroll
         for (int c = 0; c < 8; ++c) {
             if ((byte >> c) & 1u) {
+#ifdef SPADEN_EXP_NOCONFLICT  // timing experiment only: conflict-free (wrong) addresses
+                if constexpr (sizeof(typename VS::P) == 4)
+                    a = fmaf(VS::get((p0 & ~127u) + 4u * ((threadIdx.x + 8 * r + c) & 31u)), xs.v[c], a);
+                else
+                    a = fmaf(VS::get(p), xs.v[c], a);
+#else
                 a = fmaf(VS::get(p), xs.v[c], a);
+#endif
                 p += VS::step;
             }
         }
@@ -497,7 +551,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
              const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
              const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
              int nbc_vec, float alpha, float beta, float *__restrict__ y, int64_t ldx, int64_t ldy,
-             const PeerOut po) {
+             const PeerOut po, unsigned long long texx) {
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t full_bar[kMaxStages], empty_bar[kMaxStages];
     __shared__ StageHdr hdr[kMaxStages];
@@ -522,6 +576,14 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                 const int4 d1 = __ldg(reinterpret_cast<const int4 *>(tiles + t) + 1);
                 const int br0 = d0.x, br1 = d0.y, b0 = d0.z, b1 = d0.w, v0 = d1.x, v1 = d1.y;
                 if (i >= stages) mbar_wait(smem_u32(&empty_bar[s]), ph ^ 1u);
+#ifdef SPADEN_EXP_NOLOAD  // timing experiment: re-process the stage's first tile, no copies
+                if (i >= stages) {
+                    hdr[s].u_next = 0;
+                    hdr[s].done = 0;
+                    mbar_arrive(smem_u32(&full_bar[s]));
+                    continue;
+                }
+#endif
                 const uint32_t stage = sbase + (uint32_t)s * (uint32_t)stage_bytes;
                 uint32_t cur = stage;
                 struct Reg {
@@ -581,6 +643,12 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
         // units of 32 blocks are grabbed dynamically (shared counter per stage)
         const uint32_t a_next = smem_u32(&hdr[s].u_next);
         int mine = 0;
+#ifdef SPADEN_EXP_NOCOMPUTE  // timing experiment: stream only
+        __syncwarp();
+        if (lane == 0) mbar_arrive(smem_u32(&empty_bar[s]));
+        continue;
+#endif
+
         while (true) {
             int ul = 0;
             if (lane == 0) ul = atom_add_shared(a_next, 1);
@@ -596,7 +664,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                     const uint32_t cols = used_cols(bm);
                     XSeg xs[K];
 #pragma unroll
-                    for (int j = 0; j < K; ++j) load_x(xs[j], x + j * ldx, bc, nbc_vec, cols);
+                    for (int j = 0; j < K; ++j) load_x(xs[j], x + j * ldx, bc, nbc_vec, cols, texx, (int)(j * ldx / 4));
                     block_slots_k<SmemVals<V>, K>(bm, p, xs, a_part + 4u * (8 * K + 1) * lb);
                 }
             } else if constexpr (DEC == 5 || DEC == 6) {
@@ -614,7 +682,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                         const int bc = lds_i32(a_col + 4u * lb);
                         const uint32_t p0 = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
                         XSeg xs;
-                        load_x(xs, x, bc, nbc_vec, used_cols(bm));
+                        load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
                         const int plo = __popc(bm.x);
 #pragma unroll
                         for (int rr = 0; rr < RPL; ++rr) {
@@ -659,7 +727,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                                                         __popc(bm.y & mhi)) *
                                                  (uint32_t)sizeof(V);
                         XSeg xs;
-                        load_x(xs, x, bc, nbc_vec, used_cols(bm));
+                        load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
                         float a = 0.f;
 #pragma unroll
                         for (int c = 0; c < 8; ++c) {
@@ -680,7 +748,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                     float acc[8];
                     if constexpr (DEC == 1) {
                         XSeg xs;
-                        load_x(xs, x, bc, nbc_vec, used_cols(bm));
+                        load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
                         block_slots<SmemVals<V>>(bm, p, xs, acc);
                     } else {
                         block_bits<SmemVals<V>>(bm, p, x + 8 * (int64_t)bc, acc);
@@ -913,6 +981,52 @@ int sm_count() {
     return c;
 }
 
+// Texture objects binding x (n4 float4 elements from x) for load_x, cached per
+// (device, pointer, length); SPADEN_XTEX=0 disables (LDG path, ablation).
+// Entries are never destroyed while the library is loaded, so a CUDA graph that
+// captured one stays valid; at most kTexCache distinct vectors are bound (the
+// least recently created is replaced beyond that).
+constexpr int kTexCache = 64;
+unsigned long long x_texture(const float *x, int64_t n4) {
+    const char *env = getenv("SPADEN_XTEX");  // read per call (tests toggle it)
+    if ((env && env[0] == '0') || n4 <= 0) return 0ull;
+    static std::mutex mu;
+    struct Entry {
+        const float *x;
+        int dev;
+        int64_t n4;
+        cudaTextureObject_t obj;
+    };
+    static Entry cache[kTexCache] = {};
+    static int next = 0;
+    static int max_width = -1;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lock(mu);
+    for (const Entry &e : cache)
+        if (e.obj && e.x == x && e.dev == dev && e.n4 == n4) return e.obj;
+    if (max_width < 0 && cudaDeviceGetAttribute(&max_width, cudaDevAttrMaxTexture1DLinearWidth, dev) != cudaSuccess)
+        max_width = 0;
+    if (n4 > (int64_t)max_width) return 0ull;
+    cudaResourceDesc rd{};
+    rd.resType = cudaResourceTypeLinear;
+    rd.res.linear.devPtr = const_cast<float *>(x);
+    rd.res.linear.desc = cudaCreateChannelDesc<float4>();
+    rd.res.linear.sizeInBytes = (size_t)n4 * 16;
+    cudaTextureDesc td{};
+    td.readMode = cudaReadModeElementType;
+    cudaTextureObject_t o = 0;
+    if (cudaCreateTextureObject(&o, &rd, &td, nullptr) != cudaSuccess) {
+        cudaGetLastError();
+        return 0ull;
+    }
+    Entry &slot = cache[next];
+    next = (next + 1) % kTexCache;
+    if (slot.obj) cudaDestroyTextureObject(slot.obj);
+    slot = Entry{x, dev, n4, o};
+    return o;
+}
+
 template <typename V, int DEC, int CONSUMERS, int MINB>
 cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, const float *x, float beta,
                              float *y, cudaStream_t st, const PeerOut &po) {
@@ -931,9 +1045,10 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
     }
     if (A.n_tiles > 0) {
         const int grid = (int)std::min<int64_t>(A.n_tiles, (int64_t)sm_count() * occ);
+        const unsigned long long texx = x_texture(x, 2 * (int64_t)nbc_vec);
         k_spmv_tiled<V, DEC, CONSUMERS, MINB><<<grid, 32 * (CONSUMERS + 1), smem, st>>>(
             cfg.stages, cfg.stage_bytes, A.m, A.tiles, (int)A.n_tiles, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y, 0, 0, po);
+            A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y, 0, 0, po, texx);
     }
     if (A.n_long > 0) {
         const int64_t threads = 32 * A.n_chunks;
@@ -1016,9 +1131,10 @@ cudaError_t launch_spmm_cfg(const Matrix &A, const TileCfg &cfg, const TileDesc 
     }
     if (ntiles > 0) {
         const int grid = (int)std::min<int64_t>(ntiles, (int64_t)sm_count() * occ);
+        const unsigned long long texx = nbc_vec ? x_texture(X, 2 * (int64_t)nbc_vec + (K - 1) * (ldx / 4)) : 0ull;
         k_spmv_tiled<V, 1, CONSUMERS, MINB, K><<<grid, 32 * (CONSUMERS + 1), smem, st>>>(
             cfg.stages, cfg.stage_bytes, A.m, tiles, (int)ntiles, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, X, nbc_vec, alpha, beta, Y, ldx, ldy, PeerOut{});
+            A.blk_offset, (const V *)A.values, X, nbc_vec, alpha, beta, Y, ldx, ldy, PeerOut{}, texx);
     }
     if (A.n_long > 0) {  // long block-rows: the SpMV chunk path, once per vector (same arithmetic)
         const int nbc1 = ((uintptr_t)X & 31u) == 0 && ((ldx * 4) % 32) == 0 ? (int)(A.n / 8) : 0;

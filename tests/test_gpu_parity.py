@@ -679,3 +679,20 @@ def test_fused_iterated_spmv_emulated_ranks(sp, torch, world):
         torch.cuda.synchronize()
         for rk in ranks:
             assert torch.equal(rk.x[: A.n], xr[: A.n])
+
+
+@pytest.mark.parametrize("storage", ["fp32", "fp16"])
+def test_x_texture_path_bitwise_equal_to_ldg(sp, torch, storage, monkeypatch):
+    """x fetched through the texture pipe (default) and through LDG (SPADEN_XTEX=0)
+    give bitwise identical y, for SpMV and SpMM, aligned and unaligned x."""
+    A = W.fem(7, 8, 9, seed=6)
+    M = convert(sp, torch, A, storage=storage)
+    xb = torch.from_numpy(W.vector(A.n + 1, 71)).cuda()
+    X = torch.from_numpy(np.stack([W.vector(A.n, 80 + j) for j in range(4)])).cuda()
+    outs = {}
+    for mode in ("1", "0"):
+        monkeypatch.setenv("SPADEN_XTEX", mode)
+        outs[mode] = (M.spmv(xb[:A.n]), M.spmv(xb[1:].contiguous()), M.spmv(xb[1:]), M.spmm(X))
+        torch.cuda.synchronize()
+    for a, b in zip(outs["1"], outs["0"]):
+        assert torch.equal(a, b)
