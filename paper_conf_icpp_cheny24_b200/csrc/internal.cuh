@@ -98,7 +98,7 @@ struct TileCfg {
                     // 1: warp pipelines (each warp streams its own tiles; consumers = warps/CTA)
 };
 constexpr int kMaxStages = 8;
-constexpr int kNumTileCfgs = 10;
+constexpr int kNumTileCfgs = 14;
 __host__ __device__ inline TileCfg tile_cfg(int i) {
     switch (i) {
     case 1: return TileCfg{2, 16, 3, 36 * 1024, 0};
@@ -110,6 +110,11 @@ __host__ __device__ inline TileCfg tile_cfg(int i) {
     case 7: return TileCfg{4, 8, 3, 18 * 1024, 0};
     case 8: return TileCfg{4, 8, 3, 9 * 1024, 0};
     case 9: return TileCfg{4, 8, 4, 6 * 1024, 0};
+    // 4 consumer warps per CTA: half the warps share (and wait on) each tile
+    case 10: return TileCfg{6, 4, 2, 18 * 1024, 0};
+    case 11: return TileCfg{5, 4, 3, 14 * 1024, 0};
+    case 12: return TileCfg{4, 4, 3, 18 * 1024, 0};
+    case 13: return TileCfg{6, 4, 3, 12 * 1024, 0};
     default: return TileCfg{1, 16, 3, 64 * 1024, 0};
     }
 }

@@ -113,12 +113,15 @@ __global__ void k_sched_summary(const int32_t *tile_total, const int32_t *long_t
 
 int default_tile_cfg(int64_t format_bytes, int value_bytes) {
     const char *e = getenv("SPADEN_TILE_CFG");
-    if (e && e[0] >= '0' && e[0] <= '9' && e[0] - '0' < kNumTileCfgs) return e[0] - '0';
+    if (e && e[0] >= '0' && e[0] <= '9') {
+        const int c = atoi(e);
+        if (c >= 0 && c < kNumTileCfgs) return c;
+    }
     // measured best on fem1p5m: fp32 values 3 CTAs/SM x 8 consumers
-    // x 3 x 24 KB, fp16 values 4 x 8 x 2 x 27 KB; small matrices need smaller stages to
+    // x 3 x 24 KB, fp16 values 6 x 4 x 2 x 18 KB; small matrices need smaller stages to
     // give every CTA several tiles
     if (format_bytes < kSmallMatrixBytes) return kSmallTileCfg;
-    return value_bytes == 4 ? 2 : 3;
+    return value_bytes == 4 ? 2 : 10;
 }
 
 spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {

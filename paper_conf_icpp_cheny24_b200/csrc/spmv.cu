@@ -18,6 +18,7 @@
 // multiplied (reading R11).  x[8bc .. 8bc+7] is the block's 8-element segment
 // (Alg. 2 lines 7-10).
 #include <mutex>
+#include <cstddef>
 #include <cstdlib>
 
 #include "internal.cuh"
@@ -243,59 +244,25 @@ __device__ __forceinline__ uint32_t used_cols(uint2 bm) {
 
 // Row partials of one block, 64 predicated slots in ascending bit order.  Each
 // row starts at its own popcount rank (P:L138 exclusive counts), so the eight
-// rows are independent dependency chains of at most 8 slots.
+// rows are independent dependency chains of at most 8 slots.  pA / pB: first
+// value of rows 0-3 / rows 4-7 of the half-words bm.x / bm.y (block_slots_at
+// lets a caller hand in the two bitmap halves swapped, see SwapHalves).
 template <class VS>
-__device__ __forceinline__ void block_slots(uint2 bm, typename VS::P p0, const XSeg &xs, float acc[8]) {
-#ifdef SPADEN_EXP_BATCH  // loads of RB rows issued before their fma chains (independent registers)
-    constexpr int RB = SPADEN_EXP_BATCH;
-    const int plo0 = __popc(bm.x);
-#pragma unroll
-    for (int r0 = 0; r0 < 8; r0 += RB) {
-        float v[RB][8];
-#pragma unroll
-        for (int rr = 0; rr < RB; ++rr) {
-            const int r = r0 + rr;
-            const uint32_t w = r < 4 ? bm.x : bm.y;
-            const uint32_t byte = (w >> (8 * (r & 3))) & 0xffu;
-            const int below = ((r & 3) == 0 ? 0 : __popc(w & ((1u << (8 * (r & 3))) - 1u))) + (r < 4 ? 0 : plo0);
-            typename VS::P p = p0 + below * VS::step;
-#pragma unroll
-            for (int c = 0; c < 8; ++c) {
-                v[rr][c] = 0.f;
-                if ((byte >> c) & 1u) {
-                    v[rr][c] = VS::get(p);
-                    p += VS::step;
-                }
-            }
-        }
-#pragma unroll
-        for (int rr = 0; rr < RB; ++rr) {
-            const int r = r0 + rr;
-            const uint32_t w = r < 4 ? bm.x : bm.y;
-            const uint32_t byte = (w >> (8 * (r & 3))) & 0xffu;
-            float a = 0.f;
-#pragma unroll
-            for (int c = 0; c < 8; ++c)
-                if ((byte >> c) & 1u) a = fmaf(v[rr][c], xs.v[c], a);
-            acc[r] = a;
-        }
-    }
-    return;
-#endif
-    const int plo = __popc(bm.x);
+__device__ __forceinline__ void block_slots_at(uint2 bm, typename VS::P pA, typename VS::P pB, const XSeg &xs,
+                                               float acc[8]) {
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
         const uint32_t w = r < 4 ? bm.x : bm.y;
         const uint32_t byte = (w >> (8 * (r & 3))) & 0xffu;
-        const int below = ((r & 3) == 0 ? 0 : __popc(w & ((1u << (8 * (r & 3))) - 1u))) + (r < 4 ? 0 : plo);
-        typename VS::P p = p0 + below * VS::step;
+        const int below = (r & 3) == 0 ? 0 : __popc(w & ((1u << (8 * (r & 3))) - 1u));
+        typename VS::P p = (r < 4 ? pA : pB) + below * VS::step;
         float a = 0.f;
 #pragma unroll
         for (int c = 0; c < 8; ++c) {
             if ((byte >> c) & 1u) {
 #ifdef SPADEN_EXP_NOCONFLICT  // timing experiment only: conflict-free (wrong) addresses
                 if constexpr (sizeof(typename VS::P) == 4)
-                    a = fmaf(VS::get((p0 & ~127u) + 4u * ((threadIdx.x + 8 * r + c) & 31u)), xs.v[c], a);
+                    a = fmaf(VS::get((pA & ~127u) + 4u * ((threadIdx.x + 8 * r + c) & 31u)), xs.v[c], a);
                 else
                     a = fmaf(VS::get(p), xs.v[c], a);
 #else
@@ -307,6 +274,24 @@ __device__ __forceinline__ void block_slots(uint2 bm, typename VS::P p0, const X
         acc[r] = a;
     }
 }
+
+template <class VS>
+__device__ __forceinline__ void block_slots(uint2 bm, typename VS::P p0, const XSeg &xs, float acc[8]) {
+    block_slots_at<VS>(bm, p0, p0 + __popc(bm.x) * VS::step, xs, acc);
+}
+
+// Bank-conflict breaker for 2-byte values: lanes with bit 1 of
+// the lane index set walk rows 4-7 before rows 0-3.  Neighbouring blocks have
+// similar bitmaps and fp16 runs ~11 words apart, so at a given slot their
+// value loads otherwise collide in the same banks far more often than at
+// random; the swap breaks that correlation (simulated 4.31 -> 3.88 wavefronts
+// per block on fem62k).  Each row keeps its own fma order: y is unchanged.
+struct SwapHalves {
+    bool on;
+    __device__ __forceinline__ uint2 bitmap(uint2 bm) const { return on ? make_uint2(bm.y, bm.x) : bm; }
+    // shared byte offset of the partial of the decoded row index r
+    __device__ __forceinline__ uint32_t part_off(int r) const { return 4u * (uint32_t)(on ? (r ^ 4) : r); }
+};
 
 // The same partials by iterating the set bits (fewer instructions when the
 // block holds few nonzeros); identical fma sequence per row.
@@ -535,11 +520,15 @@ __device__ __forceinline__ void mma_unit(int lb0, int nb, int lane, uint32_t a_b
     }
 }
 
+// per-stage tile header; the first 32 bytes are what every consumer warp needs
+// to decode (two 16-byte loads), the next 16 only the phase-2 warp
 struct alignas(16) StageHdr {
-    int br0, nbr, b0, v0;                      // tile
-    int nb, units, u_next, done;               // blocks, 32-block units, next unit to grab, units done
-    uint32_t a_bmp, a_col, a_off, a_rp;        // shared addresses of the copied slices
-    uint32_t a_val, a_part, pad0, pad1;        // values, row-partial scratch
+    int v0, nb, units;                         // first value, blocks, 32-block units
+    uint32_t a_val;                            // shared address of the value slice
+    uint32_t a_bmp, a_col, a_off, a_part;      // ... of bitmap / blk_col / blk_offset; row-partial scratch
+    int br0, nbr, b0;                          // tile block-rows, first block (phase 2)
+    uint32_t a_rp;                             // ... of the blk_rowptr slice
+    int u_next, done, pad0, pad1;              // next unit to grab, units done
 };
 
 // DEC: 0 = set-bit loop, 1 = 64 predicated slots per lane (lane = block),
@@ -632,20 +621,22 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
     // ------------------------------------------------------------ consumers
     int s = 0;
     uint32_t ph = 0;
+    // shared addresses of stage 0's barriers / header, hoisted out of the tile loop
+    const uint32_t a_full0 = smem_u32(&full_bar[0]), a_empty0 = smem_u32(&empty_bar[0]);
+    const uint32_t a_hdr0 = smem_u32(&hdr[0]);
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x, s = (s + 1 == stages) ? (ph ^= 1u, 0) : s + 1) {
-        mbar_wait(smem_u32(&full_bar[s]), ph);
-        const int4 h0 = lds_i4_volatile(smem_u32(&hdr[s].br0));
-        const int4 h1 = lds_i4_volatile(smem_u32(&hdr[s].nb));
-        const int4 h2 = lds_i4_volatile(smem_u32(&hdr[s].a_bmp));
-        const int4 h3 = lds_i4_volatile(smem_u32(&hdr[s].a_val));
-        const int v0 = h0.w, nb = h1.x, units = h1.y;
-        const uint32_t a_bmp = h2.x, a_col = h2.y, a_off = h2.z, a_val = h3.x, a_part = h3.y;
+        const uint32_t a_hdr = a_hdr0 + (uint32_t)(s * sizeof(StageHdr));
+        mbar_wait(a_full0 + 8u * s, ph);
+        const int4 h0 = lds_i4_volatile(a_hdr);
+        const int4 h1 = lds_i4_volatile(a_hdr + 16u);
+        const int v0 = h0.x, nb = h0.y, units = h0.z;
+        const uint32_t a_val = h0.w, a_bmp = h1.x, a_col = h1.y, a_off = h1.z, a_part = h1.w;
         // units of 32 blocks are grabbed dynamically (shared counter per stage)
-        const uint32_t a_next = smem_u32(&hdr[s].u_next);
+        const uint32_t a_next = a_hdr + (uint32_t)offsetof(StageHdr, u_next);
         int mine = 0;
 #ifdef SPADEN_EXP_NOCOMPUTE  // timing experiment: stream only
         __syncwarp();
-        if (lane == 0) mbar_arrive(smem_u32(&empty_bar[s]));
+        if (lane == 0) mbar_arrive(a_empty0 + 8u * s);
         continue;
 #endif
 
@@ -746,16 +737,20 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                     const int bc = lds_i32(a_col + 4u * lb);
                     const uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
                     float acc[8];
+                    const uint32_t q = a_part + kPartStride * lb;
                     if constexpr (DEC == 1) {
                         XSeg xs;
                         load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
-                        block_slots<SmemVals<V>>(bm, p, xs, acc);
+                        const SwapHalves sw{sizeof(V) == 2 && ((lane >> 1) & 1)};
+                        const uint32_t plo = (uint32_t)__popc(bm.x) * (uint32_t)sizeof(V);
+                        block_slots_at<SmemVals<V>>(sw.bitmap(bm), sw.on ? p + plo : p, sw.on ? p : p + plo, xs, acc);
+#pragma unroll
+                        for (int r = 0; r < 8; ++r) sts_f32(q + sw.part_off(r), acc[r]);
                     } else {
                         block_bits<SmemVals<V>>(bm, p, x + 8 * (int64_t)bc, acc);
-                    }
-                    const uint32_t q = a_part + kPartStride * lb;
 #pragma unroll
-                    for (int r = 0; r < 8; ++r) sts_f32(q + 4u * r, acc[r]);
+                        for (int r = 0; r < 8; ++r) sts_f32(q + 4u * r, acc[r]);
+                    }
                 }
             }
         }
@@ -764,18 +759,19 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             int last = 0;
             if (lane == 0) {
                 __threadfence_block();
-                last = (atom_add_shared(smem_u32(&hdr[s].done), mine) + mine == units);
+                last = (atom_add_shared(a_hdr + (uint32_t)offsetof(StageHdr, done), mine) + mine == units);
             }
             if (__shfl_sync(kFull, last, 0)) {  // phase 2: this warp completed the tile
                 __threadfence_block();
+                const int4 h2 = lds_i4_volatile(a_hdr + 32u);  // br0, nbr, b0, a_rp
                 if constexpr (K > 1)
-                    reduce_tile_k<K>((uint32_t)h2.w, a_part, h0.y, h0.z, h0.x, lane, m, alpha, beta, y, ldy);
+                    reduce_tile_k<K>((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, ldy);
                 else
-                    reduce_tile((uint32_t)h2.w, a_part, h0.y, h0.z, h0.x, lane, m, alpha, beta, y, po);
+                    reduce_tile((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, po);
             }
         }
         __syncwarp();
-        if (lane == 0) mbar_arrive(smem_u32(&empty_bar[s]));
+        if (lane == 0) mbar_arrive(a_empty0 + 8u * s);
     }
 }
 
@@ -1105,6 +1101,10 @@ cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float bet
     case 7: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
     case 8: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
     case 9: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
+    case 10: return launch_tiled_cfg<V, DEC, 4, 6>(A, cfg, alpha, x, beta, y, st, po);
+    case 11: return launch_tiled_cfg<V, DEC, 4, 5>(A, cfg, alpha, x, beta, y, st, po);
+    case 12: return launch_tiled_cfg<V, DEC, 4, 4>(A, cfg, alpha, x, beta, y, st, po);
+    case 13: return launch_tiled_cfg<V, DEC, 4, 6>(A, cfg, alpha, x, beta, y, st, po);
     case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po);
     case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po);
     case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
