@@ -118,43 +118,47 @@ __global__ void k_split_summary(const int32_t *a, const int32_t *b, const int32_
     out[2] = *c;
 }
 
-// residual CSR: 8 lanes per row (4 rows per warp).  Fixed per-row order: the
-// row is cut into kResChunk-entry chunks; in a chunk lane l sums entries l,
-// l+8, ... sequentially, a 3-level xor tree combines the 8 lanes, and chunk sums
-// are added in order -- a function of the row alone (partition invariant).
-// Rows longer than kResLongRow are skipped here: their chunks run in parallel
-// (k_res_chunks) and k_res_fixup adds the chunk sums in the same order.
-template <typename V>
+// residual CSR: L lanes per row (32/L rows per warp).  Fixed per-row order:
+// the row is cut into kResChunk-entry chunks; in a chunk lane l sums entries l,
+// l+L, ... sequentially, a log2(L)-level xor tree combines the lanes, and chunk
+// sums are added in order -- a function of the row alone (partition
+// invariant).  Rows longer than kResLongRow are skipped here: their chunks run
+// in parallel (k_res_chunks, same L) and k_res_fixup adds the chunk sums in the
+// same order.
+template <typename V, int L>
 __device__ __forceinline__ float res_chunk_sum(int c0, int c1, int sub, unsigned gmask,
                                                const int32_t *__restrict__ col, const V *__restrict__ val,
                                                const float *__restrict__ x) {
     float a = 0.f;
 #pragma unroll 4
-    for (int k = c0 + sub; k < c1; k += 8) {
+    for (int k = c0 + sub; k < c1; k += L) {
         float v;
         if constexpr (sizeof(V) == 2) v = __half2float(val[k]);
         else v = __ldg(val + k);
         a = fmaf(v, __ldg(x + __ldg(col + k)), a);
     }
 #pragma unroll
-    for (int o = 4; o > 0; o >>= 1) a += __shfl_xor_sync(gmask, a, o);
+    for (int o = L / 2; o > 0; o >>= 1) a += __shfl_xor_sync(gmask, a, o);
     return a;
 }
 
-template <typename V>
+// one L-lane group per row, no grid-stride loop (the block scheduler keeps the
+// SM full of rows, so the rowptr -> colidx -> x gather chains of many rows
+// overlap); the old y is fetched before the gathers so its latency hides too
+template <typename V, int L>
 __global__ void __launch_bounds__(256)
 k_residual(int64_t m, const int32_t *__restrict__ rp, const int32_t *__restrict__ col, const V *__restrict__ val,
            const float *__restrict__ x, float alpha, float *__restrict__ y) {
-    const int64_t ngroups = ((int64_t)gridDim.x * blockDim.x) / 8;
-    const int sub = threadIdx.x & 7;
-    const unsigned gmask = 0xffu << (threadIdx.x & 24);  // this row's 8 lanes
-    for (int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 8; row < m; row += ngroups) {
-        const int k0 = __ldg(rp + row), k1 = __ldg(rp + row + 1);
-        if (k0 == k1 || k1 - k0 > kResLongRow) continue;  // uniform within the 8-lane group
-        float sum = 0.f;
-        for (int c0 = k0; c0 < k1; c0 += kResChunk) sum += res_chunk_sum<V>(c0, min(k1, c0 + kResChunk), sub, gmask, col, val, x);
-        if (sub == 0) y[row] = fmaf(alpha, sum, y[row]);
-    }
+    const int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / L;
+    const int sub = threadIdx.x & (L - 1);
+    const unsigned gmask = (L == 32 ? 0xffffffffu : ((1u << (L & 31)) - 1u)) << (threadIdx.x & (32 - L));  // this row's L lanes
+    if (row >= m) return;  // uniform within the group
+    const int k0 = __ldg(rp + row), k1 = __ldg(rp + row + 1);
+    if (k0 == k1 || k1 - k0 > kResLongRow) return;
+    const float yold = sub == 0 ? y[row] : 0.f;
+    float sum = 0.f;
+    for (int c0 = k0; c0 < k1; c0 += kResChunk) sum += res_chunk_sum<V, L>(c0, min(k1, c0 + kResChunk), sub, gmask, col, val, x);
+    if (sub == 0) y[row] = fmaf(alpha, sum, yold);
 }
 
 template <typename V>
@@ -162,27 +166,34 @@ __global__ void __launch_bounds__(256)
 k_res_chunks(int64_t nchunks, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
              const int32_t *__restrict__ chunk_row, const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
              const V *__restrict__ val, const float *__restrict__ x, float *__restrict__ carry) {
-    const int64_t g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 8;
-    const int sub = threadIdx.x & 7;
-    const unsigned gmask = 0xffu << (threadIdx.x & 24);
+    const int64_t g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / kResLanes;
+    const int sub = threadIdx.x & (kResLanes - 1);
+    const unsigned gmask = (kResLanes == 32 ? 0xffffffffu : ((1u << (kResLanes & 31)) - 1u)) << (threadIdx.x & (32 - kResLanes));
     if (g >= nchunks) return;  // uniform within the group
     const int j = chunk_row[g];
     const int row = long_rows[j];
     const int k1 = rp[row + 1];
     const int c0 = rp[row] + (int)(g - chunk_start[j]) * kResChunk;
-    const float a = res_chunk_sum<V>(c0, min(k1, c0 + kResChunk), sub, gmask, col, val, x);
+    const float a = res_chunk_sum<V, kResLanes>(c0, min(k1, c0 + kResChunk), sub, gmask, col, val, x);
     if (sub == 0) carry[g] = a;
 }
 
-__global__ void k_res_fixup(int64_t nlong, const int32_t *__restrict__ long_rows,
-                            const int32_t *__restrict__ chunk_start, const float *__restrict__ carry, float alpha,
-                            float *__restrict__ y) {
-    const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (j >= nlong) return;
+// one warp per long residual row: lane l adds the chunk sums l, l+32, ... in
+// order, then a fixed xor tree (a function of the row's chunk count)
+__global__ void __launch_bounds__(256)
+k_res_fixup(int64_t nlong, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
+            const float *__restrict__ carry, float alpha, float *__restrict__ y) {
+    const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (j >= nlong) return;  // uniform per warp
     float sum = 0.f;
-    for (int c = chunk_start[j]; c < chunk_start[j + 1]; ++c) sum += carry[c];
-    const int row = long_rows[j];
-    y[row] = fmaf(alpha, sum, y[row]);
+    for (int c = chunk_start[j] + lane; c < chunk_start[j + 1]; c += 32) sum += carry[c];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(kFull, sum, o);
+    if (lane == 0) {
+        const int row = long_rows[j];
+        y[row] = fmaf(alpha, sum, y[row]);
+    }
 }
 
 // long residual rows: flag -> scan -> list; chunk counts -> scan -> chunk owners
@@ -320,16 +331,15 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
 
 cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y, cudaStream_t st) {
     if (A.res_nnz == 0) return cudaSuccess;
-    const int64_t groups = std::min<int64_t>(A.m, 148LL * 64 * 32);  // 8 lanes per row
-    const unsigned grid = (unsigned)((8 * groups + 255) / 256);
+    const unsigned grid = (unsigned)((kResLanes * A.m + 255) / 256);  // one lane group per row
     if (A.storage == SPADEN_R_16F)
-        k_residual<__half><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx, (const __half *)A.res_values, x,
-                                                 alpha, y);
+        k_residual<__half, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
+                                                            (const __half *)A.res_values, x, alpha, y);
     else
-        k_residual<float><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx, (const float *)A.res_values, x,
-                                                alpha, y);
+        k_residual<float, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
+                                                           (const float *)A.res_values, x, alpha, y);
     if (A.res_n_long > 0) {
-        const unsigned gc = (unsigned)((8 * A.res_n_chunks + 255) / 256);
+        const unsigned gc = (unsigned)((kResLanes * A.res_n_chunks + 255) / 256);
         if (A.storage == SPADEN_R_16F)
             k_res_chunks<__half><<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start,
                                                      A.res_chunk_row, A.res_rowptr, A.res_colidx,
@@ -338,7 +348,7 @@ cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y
             k_res_chunks<float><<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start,
                                                     A.res_chunk_row, A.res_rowptr, A.res_colidx,
                                                     (const float *)A.res_values, x, A.res_carry);
-        k_res_fixup<<<(unsigned)((A.res_n_long + 255) / 256), 256, 0, st>>>(A.res_n_long, A.res_long_rows,
+        k_res_fixup<<<(unsigned)((32 * A.res_n_long + 255) / 256), 256, 0, st>>>(A.res_n_long, A.res_long_rows,
                                                                             A.res_chunk_start, A.res_carry, alpha, y);
     }
     return cudaGetLastError();

@@ -127,10 +127,24 @@ constexpr int kSmallTileCfg = 3;  // measured: smaller stages do not help fem62k
 constexpr int kBlockStageBytes = 16 + 36;
 // long block-rows are split into chunks of this many blocks (relative to the
 // block-row start, so the split depends only on the row itself)
-constexpr int kLongChunk = 1024;
+#ifndef SPADEN_LONG_CHUNK
+#define SPADEN_LONG_CHUNK 256
+#endif
+constexpr int kLongChunk = SPADEN_LONG_CHUNK;
+// at most this many block-rows per tile: phase 2 of a tile runs on one warp, so
+// runs of (nearly) empty block-rows are cut into many tiles
+constexpr int kMaxTileRows = 128;
 // hybrid residual rows: fixed 1024-entry chunks; rows above kResLongRow entries
 // have their chunks processed in parallel (carry + ordered fix-up)
-constexpr int kResChunk = 1024;
+#ifndef SPADEN_RES_CHUNK
+#define SPADEN_RES_CHUNK 1024
+#endif
+constexpr int kResChunk = SPADEN_RES_CHUNK;
+// lanes per residual row (the per-row summation tree has log2 of this many levels)
+#ifndef SPADEN_RES_LANES
+#define SPADEN_RES_LANES 16
+#endif
+constexpr int kResLanes = SPADEN_RES_LANES;
 constexpr int kResLongRow = 4096;
 // mean nonzeros per block from which the predicated-slot decode is used
 constexpr int kSlotsMinFill = 8;

@@ -78,7 +78,7 @@ __global__ void k_pack(int64_t Bnrow, const int32_t *__restrict__ brp, const int
         }
         const int64_t c = br_cost(brp, boff, br, sv, pack_blk_bytes, &nb, &nv);
         if (c > cap && too_big) atomicOr(too_big, 1u);
-        if (open_br >= 0 && open_cost + c > cap) close(br);
+        if (open_br >= 0 && (open_cost + c > cap || br - open_br >= kMaxTileRows)) close(br);
         if (open_br < 0) open_br = br;
         open_cost += c;
     }

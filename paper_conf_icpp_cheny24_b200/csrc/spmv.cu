@@ -895,8 +895,10 @@ k_spmv_warp(int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int 
 // k_spmv_long_chunks: one warp per kLongChunk-block chunk; lane j takes blocks
 // j, j+32, ... of the chunk (same per-block arithmetic as the tiled kernel),
 // sums them in that order, then a fixed xor tree over the lanes gives the
-// chunk's 8 row partials (carry).  k_spmv_long_fixup: the chunks of a row are
-// added in chunk order.  The order depends only on the block-row.
+// chunk's 8 row partials (carry).  k_spmv_long_fixup: one warp per long row;
+// lane l adds the carries of chunks l, l+32, ... in order, then a fixed xor
+// tree over the lanes.  The order depends only on the block-row (its chunk
+// count).
 template <typename V, bool SLOTS>
 __global__ void __launch_bounds__(256)
 k_spmv_long_chunks(int nchunks, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
@@ -942,19 +944,37 @@ k_spmv_long_chunks(int nchunks, const int32_t *__restrict__ long_rows, const int
     }
 }
 
-__global__ void k_spmv_long_fixup(int64_t m, int nlong, const int32_t *__restrict__ long_rows,
-                                  const int32_t *__restrict__ chunk_start, const float *__restrict__ carry, float alpha,
-                                  float beta, float *__restrict__ y, const PeerOut po) {
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= 8 * (int64_t)nlong) return;
-    const int j = (int)(t >> 3), r = (int)(t & 7);
-    float sum = 0.f;
-    for (int c = chunk_start[j]; c < chunk_start[j + 1]; ++c) sum += carry[8 * (int64_t)c + r];
-    const int64_t row = 8 * (int64_t)long_rows[j] + r;
-    if (row < m) {
-        float o = alpha * sum;
-        if (beta != 0.f) o = fmaf(beta, y[row], o);
-        store_y(y, row, o, po);
+__global__ void __launch_bounds__(256)
+k_spmv_long_fixup(int64_t m, int nlong, const int32_t *__restrict__ long_rows,
+                  const int32_t *__restrict__ chunk_start, const float *__restrict__ carry, float alpha,
+                  float beta, float *__restrict__ y, const PeerOut po) {
+    const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (j >= nlong) return;  // uniform per warp
+    float tot[8];
+#pragma unroll
+    for (int r = 0; r < 8; ++r) tot[r] = 0.f;
+    for (int c = chunk_start[j] + lane; c < chunk_start[j + 1]; c += 32) {
+        const float4 *c4 = reinterpret_cast<const float4 *>(carry + 8 * (int64_t)c);
+        const float4 lo = c4[0], hi = c4[1];
+        tot[0] += lo.x, tot[1] += lo.y, tot[2] += lo.z, tot[3] += lo.w;
+        tot[4] += hi.x, tot[5] += hi.y, tot[6] += hi.z, tot[7] += hi.w;
+    }
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) tot[r] += __shfl_xor_sync(kFull, tot[r], o);
+    }
+    if (lane == 0) {
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+            const int64_t row = 8 * (int64_t)long_rows[j] + r;
+            if (row < m) {
+                float o = alpha * tot[r];
+                if (beta != 0.f) o = fmaf(beta, y[row], o);
+                store_y(y, row, o, po);
+            }
+        }
     }
 }
 
@@ -1051,7 +1071,7 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
         k_spmv_long_chunks<V, (DEC != 0)><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
             (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
             A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry);
-        k_spmv_long_fixup<<<(unsigned)((8 * A.n_long + 255) / 256), 256, 0, st>>>(
+        k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
             A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, po);
     }
     return cudaGetLastError();
@@ -1084,7 +1104,7 @@ cudaError_t launch_warp_cfg(const Matrix &A, const TileCfg &cfg, float alpha, co
         k_spmv_long_chunks<V, (DEC != 0)><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
             (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
             A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry);
-        k_spmv_long_fixup<<<(unsigned)((8 * A.n_long + 255) / 256), 256, 0, st>>>(
+        k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
             A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, PeerOut{});
     }
     return cudaGetLastError();
@@ -1143,7 +1163,7 @@ cudaError_t launch_spmm_cfg(const Matrix &A, const TileCfg &cfg, const TileDesc 
             k_spmv_long_chunks<V, true><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
                 (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
                 A.blk_offset, (const V *)A.values, X + j * ldx, nbc1, A.carry);
-            k_spmv_long_fixup<<<(unsigned)((8 * A.n_long + 255) / 256), 256, 0, st>>>(
+            k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
                 A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, Y + j * ldy, PeerOut{});
         }
     }
