@@ -387,6 +387,27 @@ def test_fem1p5m_full(sp, torch):
         M.free()
 
 
+def test_tile_row_cap_empty_block_rows(sp, torch):
+    """Long runs of empty block-rows (more than the 128 block-rows a tile may
+    hold) between a few populated ones: y is exact (small integers) and rows
+    with no entries are exactly beta*y0."""
+    m, n = 8 * 1000 + 5, 4096
+    rows = np.array([0, 3, 8 * 300 + 1, 8 * 300 + 1, 8 * 999 + 7, m - 1])
+    cols = np.array([0, 4095, 17, 18, 2048, 5])
+    vals = np.array([1, 2, 3, 4, 5, 6], dtype=np.float32)
+    A = W.from_coo(m, n, rows, cols, vals)
+    x = (np.arange(n) % 7 + 1).astype(np.float32)
+    M = convert(sp, torch, A)
+    y = gpu_spmv(torch, M, x)
+    ref = np.zeros(m, np.float32)
+    np.add.at(ref, rows, vals * x[cols])
+    assert np.array_equal(y, ref)
+    y0 = W.vector(m, 5)
+    y2 = gpu_spmv(torch, M, x, alpha=1.0, beta=0.5, y0=y0)
+    empty = np.setdiff1d(np.arange(m), rows)
+    assert np.array_equal(y2[empty], (np.float32(0.5) * y0[empty]).astype(np.float32))
+
+
 def test_long_rows_deterministic_and_partition_invariant(sp, torch):
     """Block-rows far larger than a pipeline stage (hub rows) go through the
     chunked long-row path; y is deterministic, within tolerance, and identical
@@ -459,6 +480,8 @@ def test_spmv_host_batched(sp, torch, beta):
 
 # ------------------------------------------------------------ hybrid (NEXT-1)
 HYB_CASES = {"h1": W.h1, "tiny": lambda: W.tiny(0), "hub": lambda: hub_matrix(),
+             # residual hub rows of ~100k entries: ~100 chunks, several per fix-up lane
+             "bighub": lambda: hub_matrix(m=40, n=900_007, hub_rows=(0, 17, 33), hub_nnz=100_000, seed=3),
              "pl14": lambda: W.powerlaw(14, 5, seed=1), "fem": lambda: W.fem(6, 7, 8, seed=2)}
 
 
