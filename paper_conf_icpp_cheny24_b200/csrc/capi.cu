@@ -48,7 +48,7 @@ static void release(Matrix *A) {
                     A->pipe_y[0],   A->pipe_y[1], A->pipe_y[2], A->tiles,
                     A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->res_rowptr,
                     A->res_colidx,  A->res_values, A->res_long_rows, A->res_chunk_start,
-                    A->res_chunk_row, A->res_carry, A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
+                    A->res_chunk_row, A->res_carry, A->res_perm, A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (cudaEvent_t e : A->ev)
@@ -318,7 +318,7 @@ spaden_status_t spaden_get_info(spaden_matrix_t A, spaden_info_t *info) {
                          sv * (A->nnz - A->res_nnz);
     if (A->res_max_popc > 0) info->format_bytes += 4 * (A->m + 1) + (4 + sv) * A->res_nnz;
     info->residual_nnz = A->res_nnz;
-    info->aux_bytes = A->aux_bytes;
+    info->aux_bytes = A->aux_bytes + A->res_aux_bytes;
     info->n_tiles = A->n_tiles;
     info->n_long = A->n_long;
     return SPADEN_OK;

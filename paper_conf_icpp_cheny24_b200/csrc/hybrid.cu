@@ -6,12 +6,16 @@
 // hybrid mode the converted bitBSR is split: blocks holding at most t entries
 // become a row-sorted CSR residual (global columns), the rest stay bitBSR.
 // spaden_spmv then runs the bitBSR kernels (y = alpha*A_bit*x + beta*y) followed
-// by a residual pass (y += alpha*A_res*x, 8 lanes per row, fixed chunked order
-// and xor tree: deterministic and independent of the row partition).
+// by a residual pass (y += alpha*A_res*x; rows binned by length, 2^c lanes per
+// row of class c, fixed per-lane order and xor tree: deterministic and
+// independent of the row partition).
 //
 // Split = count kernel (per block-row: kept blocks / values, residual entries
 // per row) -> exclusive scans -> one host sync (sizes) -> fill kernel (compacts
 // the kept blocks, appends residual entries row by row in ascending column).
+#include <algorithm>
+#include <cstdlib>
+
 #include "internal.cuh"
 
 namespace spaden {
@@ -196,6 +200,97 @@ k_res_fixup(int64_t nlong, const int32_t *__restrict__ long_rows, const int32_t 
     }
 }
 
+// Length-binned residual rows (default residual pass).  Rows of 1..kResLongRow
+// entries are grouped by res_class(len) into a row permutation built at convert
+// time; class c runs L = 2^c lanes per row, lane l summing entries l, l+L, ...
+// in ascending order (four gathers in flight per lane per round), then a
+// log2(L)-level xor tree.  L is a function of the row length, so the order is a
+// function of the row alone (deterministic, partition invariant), and a
+// warp's rows have similar lengths: no lane idles on a short row while a long
+// row of the same warp runs, and short rows get one lane each (32 rows, and 32
+// independent gather chains, per warp) instead of a 16-lane group.
+template <typename V, int L>
+__device__ __forceinline__ void res_binned_row(int64_t g, int64_t nrows, const int32_t *__restrict__ perm,
+                                               const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
+                                               const V *__restrict__ val, const float *__restrict__ x, float alpha,
+                                               float *__restrict__ y) {
+    const int sub = threadIdx.x & (L - 1);
+    if (g >= nrows) return;  // uniform within the group
+    const int row = __ldg(perm + g);
+    const int k0 = __ldg(rp + row), k1 = __ldg(rp + row + 1);
+    const float yold = sub == 0 ? y[row] : 0.f;
+    float a = 0.f;
+    for (int base = k0 + sub; base < k1; base += 4 * L) {
+        int c[4];
+        float v[4], xv[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const int k = base + u * L;
+            c[u] = 0;
+            v[u] = 0.f;
+            if (k < k1) {
+                c[u] = __ldg(col + k);
+                if constexpr (sizeof(V) == 2) v[u] = __half2float(val[k]);
+                else v[u] = __ldg(val + k);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) xv[u] = base + u * L < k1 ? __ldg(x + c[u]) : 0.f;
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            if (base + u * L < k1) a = fmaf(v[u], xv[u], a);
+    }
+    if constexpr (L > 1) {
+        const unsigned gmask = (L == 32 ? kFull : ((1u << (L & 31)) - 1u)) << (threadIdx.x & (32 - L));
+#pragma unroll
+        for (int o = L / 2; o > 0; o >>= 1) a += __shfl_xor_sync(gmask, a, o);
+    }
+    if (sub == 0) y[row] = fmaf(alpha, a, yold);
+}
+
+template <typename V>
+__global__ void __launch_bounds__(256)
+k_residual_binned(ResBins bins, const int32_t *__restrict__ perm, const int32_t *__restrict__ rp,
+                  const int32_t *__restrict__ col, const V *__restrict__ val, const float *__restrict__ x,
+                  float alpha, float *__restrict__ y) {
+    // class of this CTA; static indices only (a dynamic index into the kernel
+    // parameter struct would copy it to local memory in every thread)
+    int c = 0;
+    int64_t cs = bins.cta_start[0], r0 = bins.row_start[0], r1 = bins.row_start[1];
+#pragma unroll
+    for (int k = 1; k < kResClasses; ++k)
+        if ((int64_t)blockIdx.x >= bins.cta_start[k]) {
+            c = k;
+            cs = bins.cta_start[k];
+            r0 = bins.row_start[k];
+            r1 = bins.row_start[k + 1];
+        }
+    const int64_t cta = (int64_t)blockIdx.x - cs, nrows = r1 - r0;
+    const int32_t *p = perm + r0;
+    switch (c) {  // block-uniform
+    case 0: res_binned_row<V, 1>(cta * 256 + threadIdx.x, nrows, p, rp, col, val, x, alpha, y); break;
+    case 1: res_binned_row<V, 2>(cta * 128 + threadIdx.x / 2, nrows, p, rp, col, val, x, alpha, y); break;
+    case 2: res_binned_row<V, 4>(cta * 64 + threadIdx.x / 4, nrows, p, rp, col, val, x, alpha, y); break;
+    case 3: res_binned_row<V, 8>(cta * 32 + threadIdx.x / 8, nrows, p, rp, col, val, x, alpha, y); break;
+    case 4: res_binned_row<V, 16>(cta * 16 + threadIdx.x / 16, nrows, p, rp, col, val, x, alpha, y); break;
+    default: res_binned_row<V, 32>(cta * 8 + threadIdx.x / 32, nrows, p, rp, col, val, x, alpha, y);
+    }
+}
+
+// row binning: class flag -> scan -> scatter, one class at a time (ascending
+// row order inside a class)
+__global__ void k_res_class_flag(int64_t m, const int32_t *__restrict__ rp, int c, int32_t *__restrict__ flag) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < m) {
+        const int len = rp[i + 1] - rp[i];
+        flag[i] = (len > 0 && len <= kResLongRow && (c < 0 || res_class(len) == c)) ? 1 : 0;  // c < 0: any
+    }
+}
+__global__ void k_res_class_scatter(int64_t m, const int32_t *__restrict__ pos, int32_t *__restrict__ perm) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < m && pos[i + 1] != pos[i]) perm[pos[i]] = (int32_t)i;
+}
+
 // long residual rows: flag -> scan -> list; chunk counts -> scan -> chunk owners
 __global__ void k_res_long_flag(int64_t m, const int32_t *__restrict__ rp, int32_t *__restrict__ flag) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -248,8 +343,48 @@ spaden_status_t residual_long_rows(Matrix *A, cudaStream_t st) {
             e = cudaGetLastError();
         }
     }
+    // length bins of the other non-empty rows
+    int32_t *perm_pos = nullptr;
+    ResBins bins{};
+    int64_t total = 0;
+    {  // number of binned rows -> permutation size
+        k_res_class_flag<<<g, 256, 0, st>>>(m, A->res_rowptr, -1, flag);
+        if (e == cudaSuccess) e = exclusive_scan_i32(flag, flag, m, scan_tmp, st);
+        int32_t nb = 0;
+        if (e == cudaSuccess) e = cudaMemcpyAsync(&nb, flag + m, 4, cudaMemcpyDeviceToHost, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        if (e == cudaSuccess) e = cudaMalloc(&perm_pos, 4 * (size_t)std::max(1, nb));
+    }
+    for (int c = 0; c < kResClasses && e == cudaSuccess; ++c) {
+        bins.row_start[c] = total;
+        k_res_class_flag<<<g, 256, 0, st>>>(m, A->res_rowptr, c, flag);
+        e = exclusive_scan_i32(flag, flag, m, scan_tmp, st);
+        int32_t cnt = 0;
+        if (e == cudaSuccess) e = cudaMemcpyAsync(&cnt, flag + m, 4, cudaMemcpyDeviceToHost, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        if (e == cudaSuccess && cnt > 0) {
+            k_res_class_scatter<<<g, 256, 0, st>>>(m, flag, perm_pos + total);
+            e = cudaGetLastError();
+        }
+        total += cnt;
+    }
+    bins.row_start[kResClasses] = total;
+    int64_t ctas = 0;
+    for (int c = 0; c < kResClasses; ++c) {
+        bins.cta_start[c] = ctas;
+        const int64_t lanes = (bins.row_start[c + 1] - bins.row_start[c]) << c;  // L = 2^c per row
+        ctas += (lanes + 255) / 256;
+    }
+    bins.cta_start[kResClasses] = ctas;
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     cudaFreeAsync(tmp, st);
-    if (e != cudaSuccess) return cuda_status(e, "hybrid residual long rows");
+    if (e != cudaSuccess) {
+        if (perm_pos) cudaFree(perm_pos);
+        return cuda_status(e, "hybrid residual schedule");
+    }
+    A->res_perm = perm_pos;
+    A->res_bins = bins;
+    A->res_aux_bytes = 4 * total + 4 * (A->res_n_long + 1 + A->res_n_chunks) + 4 * A->res_n_chunks;
     return SPADEN_OK;
 }
 
@@ -331,8 +466,22 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
 
 cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y, cudaStream_t st) {
     if (A.res_nnz == 0) return cudaSuccess;
+    const char *env = getenv("SPADEN_RES");  // "fixed": the 16-lane kernel (ablation), read per call
+    const bool binned = A.res_perm && !(env && env[0] == 'f');
     const unsigned grid = (unsigned)((kResLanes * A.m + 255) / 256);  // one lane group per row
-    if (A.storage == SPADEN_R_16F)
+    if (binned) {
+        const int64_t nc = A.res_bins.cta_start[kResClasses];
+        if (nc > 0) {
+            if (A.storage == SPADEN_R_16F)
+                k_residual_binned<__half><<<(unsigned)nc, 256, 0, st>>>(A.res_bins, A.res_perm, A.res_rowptr,
+                                                                         A.res_colidx, (const __half *)A.res_values,
+                                                                         x, alpha, y);
+            else
+                k_residual_binned<float><<<(unsigned)nc, 256, 0, st>>>(A.res_bins, A.res_perm, A.res_rowptr,
+                                                                        A.res_colidx, (const float *)A.res_values,
+                                                                        x, alpha, y);
+        }
+    } else if (A.storage == SPADEN_R_16F)
         k_residual<__half, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
                                                             (const __half *)A.res_values, x, alpha, y);
     else

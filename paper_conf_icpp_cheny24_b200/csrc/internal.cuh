@@ -57,6 +57,11 @@ struct spaden_matrix_s {
     int32_t *res_chunk_start = nullptr;  // [res_n_long+1]
     int32_t *res_chunk_row = nullptr;    // [res_n_chunks] index into res_long_rows
     float *res_carry = nullptr;          // [res_n_chunks]
+    int32_t *res_perm = nullptr;         // rows of 1..kResLongRow entries, grouped by length class
+    struct ResBins {                     // class c: perm[row_start[c], row_start[c+1]), CTAs from cta_start[c]
+        int64_t row_start[7], cta_start[7];
+    } res_bins = {};
+    int64_t res_aux_bytes = 0;           // perm + long-row chunk lists
 
     // host-API staging buffers (lazily allocated): [2] slots for the batched pipeline
     float *stage_x = nullptr;          // spaden_spmv_host
@@ -146,12 +151,22 @@ constexpr int kResChunk = SPADEN_RES_CHUNK;
 #endif
 constexpr int kResLanes = SPADEN_RES_LANES;
 constexpr int kResLongRow = 4096;
+// length classes of the binned residual pass: class c (L = 2^c lanes per row)
+// holds rows of len entries with 4*2^(c-1) < len <= 4*2^c; the last class takes
+// everything up to kResLongRow
+constexpr int kResClasses = 6;
+__host__ __device__ inline int res_class(int len) {
+    int c = 0;
+    while (c < kResClasses - 1 && len > (4 << c)) ++c;
+    return c;
+}
 // mean nonzeros per block from which the predicated-slot decode is used
 constexpr int kSlotsMinFill = 8;
 // decode used above that fill (1 = lane per block, 2 = lane per block row)
 constexpr int kDenseDecode = 1;
 
 using TileDesc = ::spaden_tile_desc_s;
+using ResBins = ::spaden_matrix_s::ResBins;
 
 spaden_status_t build_schedule(Matrix *A, cudaStream_t stream);
 spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t stream);

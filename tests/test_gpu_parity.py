@@ -536,6 +536,56 @@ def test_hybrid_spmv(sp, torch, name):
         assert np.array_equal(np.concatenate(parts), y1)
 
 
+def binned_rows_matrix(seed=11):
+    """Residual rows at every length-class boundary of the binned residual pass
+    (1, 4 | 5, 8 | 9, 16 | 17, 32 | 33, 64 | 65 .. 4096 | > 4096 long rows) plus
+    empty rows, in shuffled row order; with t = 64 every block is residual."""
+    rng = np.random.default_rng(seed)
+    lens = [0, 1, 2, 3, 4, 5, 7, 8, 9, 15, 16, 17, 31, 32, 33, 63, 64, 65, 100, 127, 128, 129, 1000, 4095, 4096,
+            4097, 9000]
+    lens = np.array(lens * 3)
+    rng.shuffle(lens)
+    n = 20_011
+    rows, cols = [], []
+    for r, k in enumerate(lens):
+        c = np.sort(rng.choice(n, int(k), replace=False))
+        rows.append(np.full(c.size, r))
+        cols.append(c)
+    rows, cols = np.concatenate(rows), np.concatenate(cols)
+    return W.from_coo(lens.size, n, rows, cols, rng.uniform(-1, 1, rows.size))
+
+
+@pytest.mark.parametrize("storage", ["fp32", "fp16"])
+@pytest.mark.parametrize("t", [2, 64])
+def test_residual_length_classes(sp, torch, storage, t, monkeypatch):
+    """Binned residual pass: every length class and the long-row path against the
+    oracle, bitwise deterministic, 8-row-partition invariant, and within tolerance
+    of the fixed 16-lane residual kernel (SPADEN_RES=fixed)."""
+    A = binned_rows_matrix()
+    stored = A.values if storage == "fp32" else oracle.f32_to_f16(A.values)
+    x = W.vector(A.n, 41)
+    rp, ci, v = dev(torch, A)
+    M = sp.convert(rp, ci, v, A.n, storage=storage, residual_max_popc=t)
+    if t == 64:
+        assert M.info.Bnnz == 0 and M.info.residual_nnz == A.nnz
+    y = gpu_spmv(torch, M, x)
+    assert np.array_equal(y, gpu_spmv(torch, M, x))
+    check_spmv(A, y, stored, x)
+    y0 = W.vector(A.m, 42)
+    ys, s = oracle.spmv(A.rowptr, A.colidx, stored, x)
+    y2 = gpu_spmv(torch, M, x, alpha=-0.75, beta=0.5, y0=y0)
+    assert oracle.componentwise_error(y2, -0.75 * ys + 0.5 * y0, 0.75 * s + 0.5 * np.abs(y0)) <= TOL32
+    cut = (A.m // 16) * 8
+    parts = []
+    for r0, r1 in ((0, cut), (cut, A.m)):
+        S = A.row_slice(r0, r1)
+        r, c, vv = dev(torch, S)
+        parts.append(gpu_spmv(torch, sp.convert(r, c, vv, S.n, storage=storage, residual_max_popc=t), x))
+    assert np.array_equal(np.concatenate(parts), y)
+    monkeypatch.setenv("SPADEN_RES", "fixed")
+    check_spmv(A, gpu_spmv(torch, M, x), stored, x)
+
+
 @pytest.mark.parametrize("decode", ["slots", "bits", "rows", "mma", "quad", "pair"])
 @pytest.mark.parametrize("name", ["fem62k_small", "hub", "tiny", "h2"])
 def test_decode_ablations_fp16(sp, torch, decode, name, monkeypatch):
