@@ -122,13 +122,78 @@ __global__ void k_split_summary(const int32_t *a, const int32_t *b, const int32_
     out[2] = *c;
 }
 
+// Load hints of the binned pass (SPADEN_RES_HINT, experiment hook): 0 none;
+// 1 colidx/values streamed with L1::no_allocate; 2 = 1 + L2 evict_first policy
+// on the stream; 3 = 2 + L2 evict_last policy on the x gathers.
+#ifndef SPADEN_RES_HINT
+#define SPADEN_RES_HINT 0
+#endif
+__device__ __forceinline__ uint64_t res_policy(bool last) {
+    uint64_t p;
+    if (last) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    else asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint32_t ld_stream_b32(const void *ptr, uint64_t pol) {
+    uint32_t v;
+    if constexpr (SPADEN_RES_HINT >= 2)
+        asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(ptr), "l"(pol));
+    else if constexpr (SPADEN_RES_HINT == 1)
+        asm("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(v) : "l"(ptr));
+    else
+        v = __ldg((const unsigned int *)ptr);
+    return v;
+}
+__device__ __forceinline__ float ld_x(const float *ptr, uint64_t pol) {
+    float v;
+    if constexpr (SPADEN_RES_HINT >= 3)
+        asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(ptr), "l"(pol));
+    else
+        v = __ldg(ptr);
+    return v;
+}
+
+// One lane's share of entries [kb, k1) at stride L: entries kb, kb+L, ... summed
+// sequentially in ascending order, four colidx/value loads and then four x
+// gathers in flight per round.
+template <typename V, int L>
+__device__ __forceinline__ float res_lane_sum(int kb, int k1, const int32_t *__restrict__ col,
+                                              const V *__restrict__ val, const float *__restrict__ x) {
+    const uint64_t pol_s = SPADEN_RES_HINT >= 2 ? res_policy(false) : 0ull;
+    const uint64_t pol_x = SPADEN_RES_HINT >= 3 ? res_policy(true) : 0ull;
+    float a = 0.f;
+    for (int base = kb; base < k1; base += 4 * L) {
+        int c[4];
+        float v[4], xv[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const int k = base + u * L;
+            c[u] = 0;
+            v[u] = 0.f;
+            if (k < k1) {
+                c[u] = (int)ld_stream_b32(col + k, pol_s);
+                if constexpr (sizeof(V) == 2) v[u] = __half2float(val[k]);
+                else v[u] = __uint_as_float(ld_stream_b32(val + k, pol_s));
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) xv[u] = base + u * L < k1 ? ld_x(x + c[u], pol_x) : 0.f;
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            if (base + u * L < k1) a = fmaf(v[u], xv[u], a);
+    }
+    return a;
+}
+
 // residual CSR: L lanes per row (32/L rows per warp).  Fixed per-row order:
 // the row is cut into kResChunk-entry chunks; in a chunk lane l sums entries l,
 // l+L, ... sequentially, a log2(L)-level xor tree combines the lanes, and chunk
 // sums are added in order -- a function of the row alone (partition
-// invariant).  Rows longer than kResLongRow are skipped here: their chunks run
-// in parallel (k_res_chunks, same L) and k_res_fixup adds the chunk sums in the
-// same order.
+// invariant).  This fixed-L kernel is the SPADEN_RES=fixed ablation of the
+// binned pass below.  Rows longer than kResLongRow are skipped by both: their
+// kResChunk-entry chunks run in parallel (k_res_chunks, one warp per chunk, lane
+// l summing entries l, l+32, ... of the chunk, xor tree) and k_res_fixup adds
+// the chunk sums in chunk order.
 template <typename V, int L>
 __device__ __forceinline__ float res_chunk_sum(int c0, int c1, int sub, unsigned gmask,
                                                const int32_t *__restrict__ col, const V *__restrict__ val,
@@ -170,16 +235,17 @@ __global__ void __launch_bounds__(256)
 k_res_chunks(int64_t nchunks, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
              const int32_t *__restrict__ chunk_row, const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
              const V *__restrict__ val, const float *__restrict__ x, float *__restrict__ carry) {
-    const int64_t g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / kResLanes;
-    const int sub = threadIdx.x & (kResLanes - 1);
-    const unsigned gmask = (kResLanes == 32 ? 0xffffffffu : ((1u << (kResLanes & 31)) - 1u)) << (threadIdx.x & (32 - kResLanes));
-    if (g >= nchunks) return;  // uniform within the group
+    const int64_t g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;  // one warp per chunk
+    const int lane = threadIdx.x & 31;
+    if (g >= nchunks) return;  // uniform per warp
     const int j = chunk_row[g];
     const int row = long_rows[j];
     const int k1 = rp[row + 1];
     const int c0 = rp[row] + (int)(g - chunk_start[j]) * kResChunk;
-    const float a = res_chunk_sum<V, kResLanes>(c0, min(k1, c0 + kResChunk), sub, gmask, col, val, x);
-    if (sub == 0) carry[g] = a;
+    float a = res_lane_sum<V, 32>(c0 + lane, min(k1, c0 + kResChunk), col, val, x);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(kFull, a, o);
+    if (lane == 0) carry[g] = a;
 }
 
 // one warp per long residual row: lane l adds the chunk sums l, l+32, ... in
@@ -219,27 +285,7 @@ __device__ __forceinline__ void res_binned_row(int64_t g, int64_t nrows, const i
     const int row = __ldg(perm + g);
     const int k0 = __ldg(rp + row), k1 = __ldg(rp + row + 1);
     const float yold = sub == 0 ? y[row] : 0.f;
-    float a = 0.f;
-    for (int base = k0 + sub; base < k1; base += 4 * L) {
-        int c[4];
-        float v[4], xv[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            const int k = base + u * L;
-            c[u] = 0;
-            v[u] = 0.f;
-            if (k < k1) {
-                c[u] = __ldg(col + k);
-                if constexpr (sizeof(V) == 2) v[u] = __half2float(val[k]);
-                else v[u] = __ldg(val + k);
-            }
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) xv[u] = base + u * L < k1 ? __ldg(x + c[u]) : 0.f;
-#pragma unroll
-        for (int u = 0; u < 4; ++u)
-            if (base + u * L < k1) a = fmaf(v[u], xv[u], a);
-    }
+    float a = res_lane_sum<V, L>(k0 + sub, k1, col, val, x);
     if constexpr (L > 1) {
         const unsigned gmask = (L == 32 ? kFull : ((1u << (L & 31)) - 1u)) << (threadIdx.x & (32 - L));
 #pragma unroll
@@ -464,6 +510,23 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
     return residual_long_rows(A, st);
 }
 
+namespace {
+__global__ void k_scale(int64_t m, float beta, float *__restrict__ y) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x)
+        y[i] *= beta;
+}
+}  // namespace
+
+cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st) {
+    if (A.m == 0) return cudaSuccess;
+    cudaError_t e = cudaSuccess;
+    if (beta == 0.f) e = cudaMemsetAsync(y, 0, sizeof(float) * (size_t)A.m, st);
+    else if (beta != 1.f) k_scale<<<(unsigned)std::min<int64_t>((A.m + 255) / 256, 148 * 16), 256, 0, st>>>(A.m, beta, y);
+    if (e == cudaSuccess) e = cudaGetLastError();
+    if (e == cudaSuccess) e = residual_spmv(A, alpha, x, y, st);
+    return e;
+}
+
 cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y, cudaStream_t st) {
     if (A.res_nnz == 0) return cudaSuccess;
     const char *env = getenv("SPADEN_RES");  // "fixed": the 16-lane kernel (ablation), read per call
@@ -488,7 +551,7 @@ cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y
         k_residual<float, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
                                                            (const float *)A.res_values, x, alpha, y);
     if (A.res_n_long > 0) {
-        const unsigned gc = (unsigned)((kResLanes * A.res_n_chunks + 255) / 256);
+        const unsigned gc = (unsigned)((32 * A.res_n_chunks + 255) / 256);
         if (A.storage == SPADEN_R_16F)
             k_res_chunks<__half><<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start,
                                                      A.res_chunk_row, A.res_rowptr, A.res_colidx,

@@ -191,6 +191,9 @@ spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *ro
 // hybrid split (hybrid.cu): move blocks with popc <= t into a CSR residual
 spaden_status_t split_residual(Matrix *A, int t, cudaStream_t stream);
 cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y, cudaStream_t stream);
+// hybrid SpMV, first pass: y = beta*y (y not read when beta = 0), then the residual
+// pass y += alpha*A_res*x; the bitBSR kernels follow with beta = 1
+cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t stream);
 
 // SpMV (spmv.cu)
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,

@@ -37,7 +37,8 @@ __device__ __forceinline__ int64_t br_cost(const int32_t *brp, const int32_t *bo
 // a normal row that does not fit a stage under the pack cost sets *too_big.
 template <bool WRITE>
 __global__ void k_pack(int64_t Bnrow, const int32_t *__restrict__ brp, const int32_t *__restrict__ boff,
-                       int sv, int64_t cap, int64_t long_cost, int pack_blk_bytes, uint32_t *too_big,
+                       int sv, int64_t cap, int64_t long_cost, int pack_blk_bytes, bool skip_empty,
+                       uint32_t *too_big,
                        int32_t *__restrict__ seg_tiles,
                        int32_t *__restrict__ seg_long, const int32_t *__restrict__ tile_start,
                        const int32_t *__restrict__ long_start, TileDesc *__restrict__ tiles,
@@ -74,6 +75,10 @@ __global__ void k_pack(int64_t Bnrow, const int32_t *__restrict__ brp, const int
             close(br);
             if (WRITE && long_rows) long_rows[lbase + nl] = (int32_t)br;
             ++nl;
+            continue;
+        }
+        if (skip_empty && nb == 0) {  // hybrid: y of block-rows without blocks is done by the residual pass
+            close(br);
             continue;
         }
         const int64_t c = br_cost(brp, boff, br, sv, pack_blk_bytes, &nb, &nv);
@@ -135,6 +140,7 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     // CTA pipelines: rows above half a stage are long (keeps tiles well packed);
     // warp pipelines: any row that fits a stage alone stays in the tiles
     const int64_t long_cost = cfg.warp_mode ? cap : cfg.stage_bytes / 2;
+    const bool hyb = A->res_max_popc > 0;  // hybrid: tiles skip block-rows without blocks
     if (Bnrow == 0) return SPADEN_OK;
 
     const size_t n_tmp = scan_tmp_ints(nseg + 1);
@@ -145,7 +151,7 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     int32_t *summary = scan_tmp + n_tmp;
     const unsigned grid = (unsigned)((nseg + 127) / 128);
     k_pack<false><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, kBlockStageBytes,
-                                        nullptr, seg_tiles, seg_long, nullptr, nullptr, nullptr, nullptr);
+                                        hyb, nullptr, seg_tiles, seg_long, nullptr, nullptr, nullptr, nullptr);
     cudaError_t e = exclusive_scan_i32(seg_tiles, seg_tiles, nseg, scan_tmp, st);
     if (e == cudaSuccess) e = exclusive_scan_i32(seg_long, seg_long, nseg, scan_tmp, st);
     int32_t h[2] = {0, 0};
@@ -170,7 +176,7 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     }
     A->aux_bytes = (int64_t)(tile_bytes + long_bytes);
     k_pack<true><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, kBlockStageBytes,
-                                       nullptr, nullptr, nullptr, seg_tiles, seg_long, A->tiles, A->long_rows);
+                                       hyb, nullptr, nullptr, nullptr, seg_tiles, seg_long, A->tiles, A->long_rows);
     e = cudaGetLastError();
     cudaFreeAsync(tmp, st);
     if (e != cudaSuccess) return cuda_status(e, "packing SpMV schedule");
@@ -215,6 +221,7 @@ spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t st)
     const int64_t cap = cfg.stage_bytes - kStageSlack;
     const int64_t long_cost = cfg.warp_mode ? cap : cfg.stage_bytes / 2;
     const int pack_bytes = 16 + 4 * (8 * K + 1);
+    const bool hyb = A->res_max_popc > 0;
     const int64_t nseg = (Bnrow + kSeg - 1) / kSeg;
     A->spmm_state[kidx] = -1;
     if (Bnrow == 0 || cfg.warp_mode) return SPADEN_ERR_UNSUPPORTED;
@@ -226,8 +233,8 @@ spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t st)
     uint32_t *too_big = (uint32_t *)(summary + 4);
     cudaMemsetAsync(too_big, 0, 4, st);
     const unsigned grid = (unsigned)((nseg + 127) / 128);
-    k_pack<false><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, pack_bytes, too_big,
-                                        seg_tiles, seg_long, nullptr, nullptr, nullptr, nullptr);
+    k_pack<false><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, pack_bytes, hyb,
+                                        too_big, seg_tiles, seg_long, nullptr, nullptr, nullptr, nullptr);
     cudaError_t e = exclusive_scan_i32(seg_tiles, seg_tiles, nseg, scan_tmp, st);
     int32_t h[2] = {0, 0};
     if (e == cudaSuccess) {
@@ -245,7 +252,7 @@ spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t st)
     e = cudaMalloc(&A->spmm_tiles[kidx], tile_bytes);
     if (e == cudaSuccess) {
         k_pack<true><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, pack_bytes,
-                                           nullptr, nullptr, nullptr, seg_tiles, seg_long, A->spmm_tiles[kidx],
+                                           hyb, nullptr, nullptr, nullptr, seg_tiles, seg_long, A->spmm_tiles[kidx],
                                            nullptr);
         e = cudaGetLastError();
     }

@@ -1205,15 +1205,20 @@ spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx,
             const int64_t nt = A.spmm_ntiles[kidx];
             const float *Xj = X + j * ldx;
             float *Yj = Y + j * ldy;
-            cudaError_t e;
+            cudaError_t e = cudaSuccess;
+            float beta_bit = beta;  // hybrid: residual pass first (y = beta*y + alpha*A_res*x), then accumulate
+            if (A.res_max_popc > 0) {
+                for (int q = 0; q < K && e == cudaSuccess; ++q)
+                    e = residual_first(A, alpha, Xj + q * ldx, beta, Yj + q * ldy, st);
+                beta_bit = 1.f;
+            }
+            if (e != cudaSuccess) return cuda_status(e, "launching the residual pass");
             if (A.storage == SPADEN_R_16F)
-                e = K == 4 ? launch_spmm<__half, 4>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
-                           : launch_spmm<__half, 2>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st);
+                e = K == 4 ? launch_spmm<__half, 4>(A, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st)
+                           : launch_spmm<__half, 2>(A, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st);
             else
-                e = K == 4 ? launch_spmm<float, 4>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st)
-                           : launch_spmm<float, 2>(A, tiles, nt, alpha, Xj, ldx, beta, Yj, ldy, st);
-            for (int q = 0; q < K && e == cudaSuccess; ++q)
-                e = residual_spmv(A, alpha, Xj + q * ldx, Yj + q * ldy, st);
+                e = K == 4 ? launch_spmm<float, 4>(A, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st)
+                           : launch_spmm<float, 2>(A, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st);
             if (e != cudaSuccess) return cuda_status(e, "launching SpMM");
         }
         j += K;
@@ -1230,6 +1235,13 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
         set_error("the fused all-gather store needs pure bitBSR and a CTA-pipeline tile config");
         return SPADEN_ERR_UNSUPPORTED;
     }
+    // hybrid (NEXT-1): the residual pass runs first and applies beta to every row
+    // (y = beta*y + alpha*A_res*x); the bitBSR kernels then accumulate (beta = 1)
+    // over the block-rows that hold blocks (the schedule skips the others)
+    if (A.res_max_popc > 0) {
+        SPADEN_CUDA_TRY(residual_first(A, alpha, x, beta, y, st));
+        beta = 1.f;
+    }
     if (kernel_variant() == 0 && po.n == 0) {
         const int threads = 256;
         const int64_t want = (A.Bnrow + 7) / 8;
@@ -1243,7 +1255,6 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
                                                       A.blk_offset, (const float *)A.values, x, x_vec, alpha,
                                                       beta, y);
         SPADEN_CUDA_TRY(cudaGetLastError());
-        SPADEN_CUDA_TRY(residual_spmv(A, alpha, x, y, st));
         return SPADEN_OK;
     }
     // decode style from the mean block fill (predicated slots for dense-ish blocks)
@@ -1278,7 +1289,6 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
         default: e = launch_tiled<float, 1>(A, alpha, x, beta, y, st, po);
         }
     }
-    if (e == cudaSuccess) e = residual_spmv(A, alpha, x, y, st);  // hybrid residual (if any)
     if (e != cudaSuccess) return cuda_status(e, "launching k_spmv_tiled");
     return SPADEN_OK;
 }
