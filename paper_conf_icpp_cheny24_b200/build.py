@@ -22,6 +22,7 @@ NVCC_FLAGS = [
     "-Xptxas", "-warn-spills",
     "--expt-relaxed-constexpr",
     "-cudart", "static",
+    "-Xlinker", "--no-undefined",
 ]
 
 

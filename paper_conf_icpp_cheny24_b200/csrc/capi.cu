@@ -46,9 +46,9 @@ static void release(Matrix *A) {
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap,   A->blk_offset, A->values,
                     A->stage_x,     A->stage_y,  A->pipe_x[0], A->pipe_x[1], A->pipe_x[2],
                     A->pipe_y[0],   A->pipe_y[1], A->pipe_y[2], A->tiles,
-                    A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->res_rowptr,
+                    A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->chunk_done, A->res_rowptr,
                     A->res_colidx,  A->res_values, A->res_long_rows, A->res_chunk_start,
-                    A->res_chunk_row, A->res_carry, A->res_perm, A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
+                    A->res_chunk_row, A->res_carry, A->res_done, A->res_perm, A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (cudaEvent_t e : A->ev)

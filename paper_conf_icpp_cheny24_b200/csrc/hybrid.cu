@@ -126,7 +126,7 @@ __global__ void k_split_summary(const int32_t *a, const int32_t *b, const int32_
 // 1 colidx/values streamed with L1::no_allocate; 2 = 1 + L2 evict_first policy
 // on the stream; 3 = 2 + L2 evict_last policy on the x gathers.
 #ifndef SPADEN_RES_HINT
-#define SPADEN_RES_HINT 0
+#define SPADEN_RES_HINT 3
 #endif
 __device__ __forceinline__ uint64_t res_policy(bool last) {
     uint64_t p;
@@ -192,8 +192,8 @@ __device__ __forceinline__ float res_lane_sum(int kb, int k1, const int32_t *__r
 // invariant).  This fixed-L kernel is the SPADEN_RES=fixed ablation of the
 // binned pass below.  Rows longer than kResLongRow are skipped by both: their
 // kResChunk-entry chunks run in parallel (k_res_chunks, one warp per chunk, lane
-// l summing entries l, l+32, ... of the chunk, xor tree) and k_res_fixup adds
-// the chunk sums in chunk order.
+// l summing entries l, l+32, ... of the chunk, xor tree) and the warp finishing
+// a row's last chunk adds the chunk sums in chunk order (res_fixup_row).
 template <typename V, int L>
 __device__ __forceinline__ float res_chunk_sum(int c0, int c1, int sub, unsigned gmask,
                                                const int32_t *__restrict__ col, const V *__restrict__ val,
@@ -230,11 +230,38 @@ k_residual(int64_t m, const int32_t *__restrict__ rp, const int32_t *__restrict_
     if (sub == 0) y[row] = fmaf(alpha, sum, yold);
 }
 
-template <typename V>
+// fix-up of long residual row j by one warp: lane l adds the chunk sums l,
+// l+32, ... in order, then a fixed xor tree (a function of the row's chunk count)
+__device__ __forceinline__ void res_fixup_row(int j, int lane, const int32_t *__restrict__ long_rows,
+                                              const int32_t *__restrict__ chunk_start, const float *carry,
+                                              float alpha, float *__restrict__ y) {
+    float sum = 0.f;
+    for (int c = chunk_start[j] + lane; c < chunk_start[j + 1]; c += 32) sum += __ldcg(carry + c);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(kFull, sum, o);
+    if (lane == 0) {
+        const int row = long_rows[j];
+        y[row] = fmaf(alpha, sum, y[row]);
+    }
+}
+
+__global__ void __launch_bounds__(256)
+k_res_fixup(int64_t nlong, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
+            const float *carry, float alpha, float *__restrict__ y) {
+    const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (j < nlong) res_fixup_row((int)j, threadIdx.x & 31, long_rows, chunk_start, carry, alpha, y);
+}
+
+// long residual rows: one warp per kResChunk-entry chunk (lane l sums entries
+// l, l+32, ... of the chunk, xor tree); FUSED (few chunks): the
+// warp finishing a row's last chunk runs the fix-up (threadfence + completion
+// counter, reset for the next call), else k_res_fixup does after the launch
+template <typename V, bool FUSED>
 __global__ void __launch_bounds__(256)
 k_res_chunks(int64_t nchunks, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
              const int32_t *__restrict__ chunk_row, const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
-             const V *__restrict__ val, const float *__restrict__ x, float *__restrict__ carry) {
+             const V *__restrict__ val, const float *__restrict__ x, float *carry, int32_t *__restrict__ done,
+             float alpha, float *__restrict__ y) {
     const int64_t g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;  // one warp per chunk
     const int lane = threadIdx.x & 31;
     if (g >= nchunks) return;  // uniform per warp
@@ -245,24 +272,18 @@ k_res_chunks(int64_t nchunks, const int32_t *__restrict__ long_rows, const int32
     float a = res_lane_sum<V, 32>(c0 + lane, min(k1, c0 + kResChunk), col, val, x);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(kFull, a, o);
-    if (lane == 0) carry[g] = a;
-}
-
-// one warp per long residual row: lane l adds the chunk sums l, l+32, ... in
-// order, then a fixed xor tree (a function of the row's chunk count)
-__global__ void __launch_bounds__(256)
-k_res_fixup(int64_t nlong, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
-            const float *__restrict__ carry, float alpha, float *__restrict__ y) {
-    const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int lane = threadIdx.x & 31;
-    if (j >= nlong) return;  // uniform per warp
-    float sum = 0.f;
-    for (int c = chunk_start[j] + lane; c < chunk_start[j + 1]; c += 32) sum += carry[c];
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(kFull, sum, o);
+    int last = 0;
     if (lane == 0) {
-        const int row = long_rows[j];
-        y[row] = fmaf(alpha, sum, y[row]);
+        __stcg(carry + g, a);
+        if constexpr (FUSED) {
+            __threadfence();
+            last = atomicAdd(done + j, 1) == chunk_start[j + 1] - chunk_start[j] - 1;
+        }
+    }
+    if (FUSED && __shfl_sync(kFull, last, 0)) {
+        __threadfence();
+        res_fixup_row(j, lane, long_rows, chunk_start, carry, alpha, y);
+        if (lane == 0) done[j] = 0;
     }
 }
 
@@ -384,6 +405,8 @@ spaden_status_t residual_long_rows(Matrix *A, cudaStream_t st) {
             e = cudaMalloc(&A->res_chunk_row, 4 * (size_t)std::max(1, nc));
         }
         if (e == cudaSuccess) e = cudaMalloc(&A->res_carry, 4 * (size_t)std::max(1, nc));
+        if (e == cudaSuccess) e = cudaMalloc(&A->res_done, 4 * (size_t)nl);
+        if (e == cudaSuccess) e = cudaMemsetAsync(A->res_done, 0, 4 * (size_t)nl, st);
         if (e == cudaSuccess) {
             k_res_chunk_rows<<<(unsigned)((nl + 255) / 256), 256, 0, st>>>(nl, A->res_chunk_start, A->res_chunk_row);
             e = cudaGetLastError();
@@ -430,7 +453,7 @@ spaden_status_t residual_long_rows(Matrix *A, cudaStream_t st) {
     }
     A->res_perm = perm_pos;
     A->res_bins = bins;
-    A->res_aux_bytes = 4 * total + 4 * (A->res_n_long + 1 + A->res_n_chunks) + 4 * A->res_n_chunks;
+    A->res_aux_bytes = 4 * total + 4 * (2 * A->res_n_long + 1 + A->res_n_chunks) + 4 * A->res_n_chunks;
     return SPADEN_OK;
 }
 
@@ -552,16 +575,19 @@ cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y
                                                            (const float *)A.res_values, x, alpha, y);
     if (A.res_n_long > 0) {
         const unsigned gc = (unsigned)((32 * A.res_n_chunks + 255) / 256);
-        if (A.storage == SPADEN_R_16F)
-            k_res_chunks<__half><<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start,
-                                                     A.res_chunk_row, A.res_rowptr, A.res_colidx,
-                                                     (const __half *)A.res_values, x, A.res_carry);
-        else
-            k_res_chunks<float><<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start,
-                                                    A.res_chunk_row, A.res_rowptr, A.res_colidx,
-                                                    (const float *)A.res_values, x, A.res_carry);
-        k_res_fixup<<<(unsigned)((32 * A.res_n_long + 255) / 256), 256, 0, st>>>(A.res_n_long, A.res_long_rows,
-                                                                            A.res_chunk_start, A.res_carry, alpha, y);
+        const bool fused = A.res_n_chunks <= fused_fixup_max();
+        if (A.storage == SPADEN_R_16F) {
+            auto k = fused ? k_res_chunks<__half, true> : k_res_chunks<__half, false>;
+            k<<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start, A.res_chunk_row, A.res_rowptr,
+                                  A.res_colidx, (const __half *)A.res_values, x, A.res_carry, A.res_done, alpha, y);
+        } else {
+            auto k = fused ? k_res_chunks<float, true> : k_res_chunks<float, false>;
+            k<<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start, A.res_chunk_row, A.res_rowptr,
+                                  A.res_colidx, (const float *)A.res_values, x, A.res_carry, A.res_done, alpha, y);
+        }
+        if (A.res_n_chunks > fused_fixup_max())
+            k_res_fixup<<<(unsigned)((32 * A.res_n_long + 255) / 256), 256, 0, st>>>(
+                A.res_n_long, A.res_long_rows, A.res_chunk_start, A.res_carry, alpha, y);
     }
     return cudaGetLastError();
 }

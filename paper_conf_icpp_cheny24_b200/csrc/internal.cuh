@@ -39,6 +39,7 @@ struct spaden_matrix_s {
     int32_t *chunk_start = nullptr;            // [n_long+1] first chunk of each long row
     int32_t *chunk_row = nullptr;              // [n_chunks] index into long_rows
     float *carry = nullptr;                    // [n_chunks*8] per-chunk row partials
+    int32_t *chunk_done = nullptr;             // [n_long] chunks finished per long row (0 between calls)
 
     // SpMM schedules for K = 2, 4 right-hand sides (index 0, 1; built lazily by spaden_spmm)
     struct spaden_tile_desc_s *spmm_tiles[3] = {};
@@ -57,6 +58,7 @@ struct spaden_matrix_s {
     int32_t *res_chunk_start = nullptr;  // [res_n_long+1]
     int32_t *res_chunk_row = nullptr;    // [res_n_chunks] index into res_long_rows
     float *res_carry = nullptr;          // [res_n_chunks]
+    int32_t *res_done = nullptr;         // [res_n_long] chunks finished per long row (0 between calls)
     int32_t *res_perm = nullptr;         // rows of 1..kResLongRow entries, grouped by length class
     struct ResBins {                     // class c: perm[row_start[c], row_start[c+1]), CTAs from cta_start[c]
         int64_t row_start[7], cta_start[7];
@@ -133,16 +135,25 @@ constexpr int kBlockStageBytes = 16 + 36;
 // long block-rows are split into chunks of this many blocks (relative to the
 // block-row start, so the split depends only on the row itself)
 #ifndef SPADEN_LONG_CHUNK
-#define SPADEN_LONG_CHUNK 256
+#define SPADEN_LONG_CHUNK 128
 #endif
 constexpr int kLongChunk = SPADEN_LONG_CHUNK;
+// With at most this many chunks (latency-bound: about one wave of warps) the
+// warp finishing a long row's last chunk does its fix-up; with more, a separate
+// fix-up kernel runs after the chunks (the per-chunk fence + counter atomic
+// costs more than the launch when chunks are many: DESIGN.md §5)
+#ifndef SPADEN_FUSED_FIXUP_MAX
+#define SPADEN_FUSED_FIXUP_MAX 8192
+#endif
+constexpr int64_t kFusedFixupMaxChunks = SPADEN_FUSED_FIXUP_MAX;
+int64_t fused_fixup_max();  // kFusedFixupMaxChunks, or the SPADEN_FUSED_FIXUP_MAX environment override
 // at most this many block-rows per tile: phase 2 of a tile runs on one warp, so
 // runs of (nearly) empty block-rows are cut into many tiles
 constexpr int kMaxTileRows = 128;
 // hybrid residual rows: fixed 1024-entry chunks; rows above kResLongRow entries
 // have their chunks processed in parallel (carry + ordered fix-up)
 #ifndef SPADEN_RES_CHUNK
-#define SPADEN_RES_CHUNK 1024
+#define SPADEN_RES_CHUNK 256
 #endif
 constexpr int kResChunk = SPADEN_RES_CHUNK;
 // lanes per residual row (the per-row summation tree has log2 of this many levels)

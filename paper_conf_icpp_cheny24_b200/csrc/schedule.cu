@@ -201,12 +201,14 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
         e = cudaMalloc(&A->chunk_row, sizeof(int32_t) * std::max(1, nch));
     }
     if (e == cudaSuccess) e = cudaMalloc(&A->carry, sizeof(float) * 8 * std::max(1, nch));
+    if (e == cudaSuccess) e = cudaMalloc(&A->chunk_done, sizeof(int32_t) * nl);
+    if (e == cudaSuccess) e = cudaMemsetAsync(A->chunk_done, 0, sizeof(int32_t) * nl, st);
     if (e == cudaSuccess) {
         k_chunk_rows<<<(nl + 255) / 256, 256, 0, st>>>(nl, A->chunk_start, A->chunk_row);
         e = cudaGetLastError();
     }
     if (e != cudaSuccess) return cuda_status(e, "long-row chunk schedule");
-    A->aux_bytes += (int64_t)sizeof(int32_t) * (nl + 1 + nch) + (int64_t)sizeof(float) * 8 * nch;
+    A->aux_bytes += (int64_t)sizeof(int32_t) * (2 * nl + 1 + nch) + (int64_t)sizeof(float) * 8 * nch;
     return SPADEN_OK;
 }
 

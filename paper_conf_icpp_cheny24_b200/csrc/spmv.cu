@@ -5,7 +5,7 @@
 //   k_spmv_tiled  (default)  persistent CTAs fed by a TMA bulk-copy pipeline;
 //   k_spmv_v0     (SPADEN_KERNEL=v0) the first, simple row-byte kernel, kept as
 //                 the measured baseline of DESIGN.md.
-// and k_spmv_long_chunks + k_spmv_long_fixup for block-rows too large for a
+// and k_spmv_long_chunks (chunks + fused fix-up) for block-rows too large for a
 // pipeline stage.
 //
 // Decode (both kernels follow PAPER.md §4.3.1 / Alg. 2 semantics):
@@ -891,21 +891,64 @@ k_spmv_warp(int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int 
     }
 }
 
+// fix-up of long block-row j by one warp: lane l adds the 8-float partials of
+// chunks l, l+32, ... in order, then a fixed xor tree (a function of the row's
+// chunk count).  Carries are read from L2 (__ldcg): they were written by other SMs.
+__device__ __forceinline__ void long_fixup_row(int64_t m, int j, int lane, const int32_t *__restrict__ long_rows,
+                                               const int32_t *__restrict__ chunk_start, const float *carry,
+                                               float alpha, float beta, float *__restrict__ y, const PeerOut &po) {
+    float tot[8];
+#pragma unroll
+    for (int r = 0; r < 8; ++r) tot[r] = 0.f;
+    for (int c = chunk_start[j] + lane; c < chunk_start[j + 1]; c += 32) {
+        const float4 *c4 = reinterpret_cast<const float4 *>(carry + 8 * (int64_t)c);
+        const float4 lo = __ldcg(c4), hi = __ldcg(c4 + 1);
+        tot[0] += lo.x, tot[1] += lo.y, tot[2] += lo.z, tot[3] += lo.w;
+        tot[4] += hi.x, tot[5] += hi.y, tot[6] += hi.z, tot[7] += hi.w;
+    }
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) tot[r] += __shfl_xor_sync(kFull, tot[r], o);
+    }
+    if (lane == 0) {
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+            const int64_t row = 8 * (int64_t)long_rows[j] + r;
+            if (row < m) {
+                float o = alpha * tot[r];
+                if (beta != 0.f) o = fmaf(beta, y[row], o);
+                store_y(y, row, o, po);
+            }
+        }
+    }
+}
+
+// separate fix-up launch (more than kFusedFixupMaxChunks chunks)
+__global__ void __launch_bounds__(256)
+k_spmv_long_fixup(int64_t m, int nlong, const int32_t *__restrict__ long_rows,
+                  const int32_t *__restrict__ chunk_start, const float *carry, float alpha, float beta,
+                  float *__restrict__ y, const PeerOut po) {
+    const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (j < nlong) long_fixup_row(m, (int)j, threadIdx.x & 31, long_rows, chunk_start, carry, alpha, beta, y, po);
+}
+
 // Long block-rows (too large for a stage), straight from global memory.
 // k_spmv_long_chunks: one warp per kLongChunk-block chunk; lane j takes blocks
 // j, j+32, ... of the chunk (same per-block arithmetic as the tiled kernel),
 // sums them in that order, then a fixed xor tree over the lanes gives the
-// chunk's 8 row partials (carry).  k_spmv_long_fixup: one warp per long row;
-// lane l adds the carries of chunks l, l+32, ... in order, then a fixed xor
-// tree over the lanes.  The order depends only on the block-row (its chunk
-// count).
-template <typename V, bool SLOTS>
+// chunk's 8 row partials (carry).  The warp that finishes a row's last chunk
+// runs the fix-up (long_fixup_row): lane l adds the carries of chunks l, l+32,
+// ... in order, then a fixed xor tree over the lanes.  The order depends only
+// on the block-row (its chunk count), not on which warp finishes last.
+template <typename V, bool SLOTS, bool FUSED>
 __global__ void __launch_bounds__(256)
 k_spmv_long_chunks(int nchunks, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
                    const int32_t *__restrict__ chunk_row, const int32_t *__restrict__ blk_rowptr,
                    const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
                    const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
-                   int nbc_vec, float *__restrict__ carry) {
+                   int nbc_vec, float *carry, int32_t *__restrict__ done, int64_t m, float alpha, float beta,
+                   float *__restrict__ y, const PeerOut po) {
     const int w = (int)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
     const int lane = threadIdx.x & 31;
     if (w >= nchunks) return;
@@ -937,44 +980,23 @@ k_spmv_long_chunks(int nchunks, const int32_t *__restrict__ long_rows, const int
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) tot[r] += __shfl_xor_sync(kFull, tot[r], o);
     }
+    // FUSED (few chunks): the warp that completes the row's last
+    // chunk does the fix-up (threadfence + completion counter, reset for the
+    // next call); otherwise k_spmv_long_fixup runs after this launch
+    int last = 0;
     if (lane == 0) {
         float4 *c4 = reinterpret_cast<float4 *>(carry + 8 * (int64_t)w);
-        c4[0] = make_float4(tot[0], tot[1], tot[2], tot[3]);
-        c4[1] = make_float4(tot[4], tot[5], tot[6], tot[7]);
-    }
-}
-
-__global__ void __launch_bounds__(256)
-k_spmv_long_fixup(int64_t m, int nlong, const int32_t *__restrict__ long_rows,
-                  const int32_t *__restrict__ chunk_start, const float *__restrict__ carry, float alpha,
-                  float beta, float *__restrict__ y, const PeerOut po) {
-    const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int lane = threadIdx.x & 31;
-    if (j >= nlong) return;  // uniform per warp
-    float tot[8];
-#pragma unroll
-    for (int r = 0; r < 8; ++r) tot[r] = 0.f;
-    for (int c = chunk_start[j] + lane; c < chunk_start[j + 1]; c += 32) {
-        const float4 *c4 = reinterpret_cast<const float4 *>(carry + 8 * (int64_t)c);
-        const float4 lo = c4[0], hi = c4[1];
-        tot[0] += lo.x, tot[1] += lo.y, tot[2] += lo.z, tot[3] += lo.w;
-        tot[4] += hi.x, tot[5] += hi.y, tot[6] += hi.z, tot[7] += hi.w;
-    }
-#pragma unroll
-    for (int r = 0; r < 8; ++r) {
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) tot[r] += __shfl_xor_sync(kFull, tot[r], o);
-    }
-    if (lane == 0) {
-#pragma unroll
-        for (int r = 0; r < 8; ++r) {
-            const int64_t row = 8 * (int64_t)long_rows[j] + r;
-            if (row < m) {
-                float o = alpha * tot[r];
-                if (beta != 0.f) o = fmaf(beta, y[row], o);
-                store_y(y, row, o, po);
-            }
+        __stcg(c4, make_float4(tot[0], tot[1], tot[2], tot[3]));
+        __stcg(c4 + 1, make_float4(tot[4], tot[5], tot[6], tot[7]));
+        if constexpr (FUSED) {
+            __threadfence();
+            last = atomicAdd(done + j, 1) == chunk_start[j + 1] - chunk_start[j] - 1;
         }
+    }
+    if (FUSED && __shfl_sync(kFull, last, 0)) {
+        __threadfence();
+        long_fixup_row(m, j, lane, long_rows, chunk_start, carry, alpha, beta, y, po);
+        if (lane == 0) done[j] = 0;
     }
 }
 
@@ -1068,11 +1090,17 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
     }
     if (A.n_long > 0) {
         const int64_t threads = 32 * A.n_chunks;
-        k_spmv_long_chunks<V, (DEC != 0)><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+        if (A.n_chunks <= fused_fixup_max())
+            k_spmv_long_chunks<V, (DEC != 0), true><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
             (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry);
-        k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
-            A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, po);
+            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, A.m, alpha, beta, y, po);
+        else
+            k_spmv_long_chunks<V, (DEC != 0), false><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+            (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
+            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, A.m, alpha, beta, y, po);
+        if (A.n_chunks > fused_fixup_max())
+            k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
+                A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, po);
     }
     return cudaGetLastError();
 }
@@ -1101,11 +1129,17 @@ cudaError_t launch_warp_cfg(const Matrix &A, const TileCfg &cfg, float alpha, co
     }
     if (A.n_long > 0) {
         const int64_t threads = 32 * A.n_chunks;
-        k_spmv_long_chunks<V, (DEC != 0)><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+        if (A.n_chunks <= fused_fixup_max())
+            k_spmv_long_chunks<V, (DEC != 0), true><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
             (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry);
-        k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
-            A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, PeerOut{});
+            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, A.m, alpha, beta, y, PeerOut{});
+        else
+            k_spmv_long_chunks<V, (DEC != 0), false><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+            (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
+            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, A.m, alpha, beta, y, PeerOut{});
+        if (A.n_chunks > fused_fixup_max())
+            k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
+                A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, PeerOut{});
     }
     return cudaGetLastError();
 }
@@ -1160,11 +1194,19 @@ cudaError_t launch_spmm_cfg(const Matrix &A, const TileCfg &cfg, const TileDesc 
         const int nbc1 = ((uintptr_t)X & 31u) == 0 && ((ldx * 4) % 32) == 0 ? (int)(A.n / 8) : 0;
         for (int j = 0; j < K; ++j) {
             const int64_t threads = 32 * A.n_chunks;
-            k_spmv_long_chunks<V, true><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+            if (A.n_chunks <= fused_fixup_max())
+                k_spmv_long_chunks<V, true, true><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
                 (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
-                A.blk_offset, (const V *)A.values, X + j * ldx, nbc1, A.carry);
-            k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
-                A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, Y + j * ldy, PeerOut{});
+                A.blk_offset, (const V *)A.values, X + j * ldx, nbc1, A.carry, A.chunk_done, A.m, alpha, beta,
+                Y + j * ldy, PeerOut{});
+            else
+                k_spmv_long_chunks<V, true, false><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
+                (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
+                A.blk_offset, (const V *)A.values, X + j * ldx, nbc1, A.carry, A.chunk_done, A.m, alpha, beta,
+                Y + j * ldy, PeerOut{});
+            if (A.n_chunks > fused_fixup_max())
+                k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
+                    A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, Y + j * ldy, PeerOut{});
         }
     }
     return cudaGetLastError();
@@ -1184,6 +1226,12 @@ cudaError_t launch_spmm(const Matrix &A, const TileDesc *tiles, int64_t ntiles, 
 }
 
 }  // namespace
+
+int64_t fused_fixup_max() {  // SPADEN_FUSED_FIXUP_MAX overrides (tests), read per call
+    const char *e = getenv("SPADEN_FUSED_FIXUP_MAX");
+    return e ? atoll(e) : kFusedFixupMaxChunks;
+}
+
 
 spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx, int k, float beta, float *Y,
                             int64_t ldy, cudaStream_t st) {

@@ -408,17 +408,23 @@ def test_tile_row_cap_empty_block_rows(sp, torch):
     assert np.array_equal(y2[empty], (np.float32(0.5) * y0[empty]).astype(np.float32))
 
 
-def test_long_rows_deterministic_and_partition_invariant(sp, torch):
+@pytest.mark.parametrize("fixup", ["fused", "separate"])
+def test_long_rows_deterministic_and_partition_invariant(sp, torch, fixup, monkeypatch):
     """Block-rows far larger than a pipeline stage (hub rows) go through the
     chunked long-row path; y is deterministic, within tolerance, and identical
-    under an 8-row-aligned row split."""
+    under an 8-row-aligned row split -- with the fix-up fused into the chunk
+    kernel (last warp per row) and as a separate launch, bitwise equal."""
     A = hub_matrix(m=96, n=400_003, hub_rows=(3, 9, 60, 61), hub_nnz=120_000, seed=11)
     M = convert(sp, torch, A)
     assert M.info.n_long >= 2
     x = W.vector(A.n, 13)
+    ref = gpu_spmv(torch, M, x)
+    if fixup == "separate":
+        monkeypatch.setenv("SPADEN_FUSED_FIXUP_MAX", "0")
     y1 = gpu_spmv(torch, M, x)
-    y2 = gpu_spmv(torch, M, x)
-    assert np.array_equal(y1, y2)
+    assert np.array_equal(y1, ref)
+    y2 = gpu_spmv(torch, M, x, alpha=2.0, beta=-1.0, y0=y1)
+    assert np.array_equal(gpu_spmv(torch, M, x, alpha=2.0, beta=-1.0, y0=y1), y2)
     check_spmv(A, y1, A.values, x)
     parts = [gpu_spmv(torch, convert(sp, torch, A.row_slice(r0, r1)), x) for r0, r1 in ((0, 56), (56, 96))]
     assert np.array_equal(np.concatenate(parts), y1)
@@ -557,10 +563,13 @@ def binned_rows_matrix(seed=11):
 
 @pytest.mark.parametrize("storage", ["fp32", "fp16"])
 @pytest.mark.parametrize("t", [2, 64])
-def test_residual_length_classes(sp, torch, storage, t, monkeypatch):
+@pytest.mark.parametrize("fixup", ["fused", "separate"])
+def test_residual_length_classes(sp, torch, storage, t, fixup, monkeypatch):
     """Binned residual pass: every length class and the long-row path against the
     oracle, bitwise deterministic, 8-row-partition invariant, and within tolerance
     of the fixed 16-lane residual kernel (SPADEN_RES=fixed)."""
+    if fixup == "separate":  # long-row fix-up as its own launch (as with many chunks)
+        monkeypatch.setenv("SPADEN_FUSED_FIXUP_MAX", "0")
     A = binned_rows_matrix()
     stored = A.values if storage == "fp32" else oracle.f32_to_f16(A.values)
     x = W.vector(A.n, 41)

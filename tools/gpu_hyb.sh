@@ -2,7 +2,7 @@
 # gpu_hyb.sh "workload:hybrid ...": hybrid-path GPU tests + kernel ms per workload
 mkdir -p gpurun_out
 : > gpurun_out/hyb.txt
-timeout 900 python -m pytest tests -m gpu -q -x -k "hybrid or residual or random_shapes or spmm or tile_row_cap or host or graph" > gpurun_out/pytest_hyb.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_hyb.log
+timeout 900 python -m pytest tests -m gpu -q -x -k "hybrid or residual or random_shapes or spmm or tile_row_cap or host or graph or long or pagerank or hub or configs" > gpurun_out/pytest_hyb.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_hyb.log
 tail -3 gpurun_out/pytest_hyb.log >> gpurun_out/hyb.txt
 for w in $1; do
   wl=${w%%:*}; hy=${w##*:}
