@@ -249,6 +249,7 @@ __global__ void __launch_bounds__(256)
 k_res_fixup(int64_t nlong, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ chunk_start,
             const float *carry, float alpha, float *__restrict__ y) {
     const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    pdl_wait();
     if (j < nlong) res_fixup_row((int)j, threadIdx.x & 31, long_rows, chunk_start, carry, alpha, y);
 }
 
@@ -262,6 +263,7 @@ k_res_chunks(int64_t nchunks, const int32_t *__restrict__ long_rows, const int32
              const int32_t *__restrict__ chunk_row, const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
              const V *__restrict__ val, const float *__restrict__ x, float *carry, int32_t *__restrict__ done,
              float alpha, float *__restrict__ y) {
+    pdl_trigger();
     const int64_t g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;  // one warp per chunk
     const int lane = threadIdx.x & 31;
     if (g >= nchunks) return;  // uniform per warp
@@ -280,6 +282,7 @@ k_res_chunks(int64_t nchunks, const int32_t *__restrict__ long_rows, const int32
             last = atomicAdd(done + j, 1) == chunk_start[j + 1] - chunk_start[j] - 1;
         }
     }
+    pdl_wait();  // fix-up below reads y; unfused: still complete only after the predecessor
     if (FUSED && __shfl_sync(kFull, last, 0)) {
         __threadfence();
         res_fixup_row(j, lane, long_rows, chunk_start, carry, alpha, y);
@@ -302,11 +305,15 @@ __device__ __forceinline__ void res_binned_row(int64_t g, int64_t nrows, const i
                                                const V *__restrict__ val, const float *__restrict__ x, float alpha,
                                                float *__restrict__ y) {
     const int sub = threadIdx.x & (L - 1);
-    if (g >= nrows) return;  // uniform within the group
+    if (g >= nrows) {  // uniform within the group
+        pdl_wait();    // (every PDL kernel completes after its predecessor: keeps the chain ordered)
+        return;
+    }
     const int row = __ldg(perm + g);
     const int k0 = __ldg(rp + row), k1 = __ldg(rp + row + 1);
-    const float yold = sub == 0 ? y[row] : 0.f;
     float a = res_lane_sum<V, L>(k0 + sub, k1, col, val, x);
+    pdl_wait();  // y (beta pass) from the previous kernel
+    const float yold = sub == 0 ? y[row] : 0.f;
     if constexpr (L > 1) {
         const unsigned gmask = (L == 32 ? kFull : ((1u << (L & 31)) - 1u)) << (threadIdx.x & (32 - L));
 #pragma unroll
@@ -320,6 +327,7 @@ __global__ void __launch_bounds__(256)
 k_residual_binned(ResBins bins, const int32_t *__restrict__ perm, const int32_t *__restrict__ rp,
                   const int32_t *__restrict__ col, const V *__restrict__ val, const float *__restrict__ x,
                   float alpha, float *__restrict__ y) {
+    pdl_trigger();
     // class of this CTA; static indices only (a dynamic index into the kernel
     // parameter struct would copy it to local memory in every thread)
     int c = 0;
@@ -555,17 +563,18 @@ cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y
     const char *env = getenv("SPADEN_RES");  // "fixed": the 16-lane kernel (ablation), read per call
     const bool binned = A.res_perm && !(env && env[0] == 'f');
     const unsigned grid = (unsigned)((kResLanes * A.m + 255) / 256);  // one lane group per row
+    cudaError_t e = cudaSuccess;
     if (binned) {
         const int64_t nc = A.res_bins.cta_start[kResClasses];
         if (nc > 0) {
             if (A.storage == SPADEN_R_16F)
-                k_residual_binned<__half><<<(unsigned)nc, 256, 0, st>>>(A.res_bins, A.res_perm, A.res_rowptr,
-                                                                         A.res_colidx, (const __half *)A.res_values,
-                                                                         x, alpha, y);
+                e = launch_k(true, k_residual_binned<__half>, dim3((unsigned)nc), dim3(256), 0, st, A.res_bins,
+                             (const int32_t *)A.res_perm, (const int32_t *)A.res_rowptr,
+                             (const int32_t *)A.res_colidx, (const __half *)A.res_values, x, alpha, y);
             else
-                k_residual_binned<float><<<(unsigned)nc, 256, 0, st>>>(A.res_bins, A.res_perm, A.res_rowptr,
-                                                                        A.res_colidx, (const float *)A.res_values,
-                                                                        x, alpha, y);
+                e = launch_k(true, k_residual_binned<float>, dim3((unsigned)nc), dim3(256), 0, st, A.res_bins,
+                             (const int32_t *)A.res_perm, (const int32_t *)A.res_rowptr,
+                             (const int32_t *)A.res_colidx, (const float *)A.res_values, x, alpha, y);
         }
     } else if (A.storage == SPADEN_R_16F)
         k_residual<__half, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
@@ -576,19 +585,26 @@ cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y
     if (A.res_n_long > 0) {
         const unsigned gc = (unsigned)((32 * A.res_n_chunks + 255) / 256);
         const bool fused = A.res_n_chunks <= fused_fixup_max();
-        if (A.storage == SPADEN_R_16F) {
-            auto k = fused ? k_res_chunks<__half, true> : k_res_chunks<__half, false>;
-            k<<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start, A.res_chunk_row, A.res_rowptr,
-                                  A.res_colidx, (const __half *)A.res_values, x, A.res_carry, A.res_done, alpha, y);
-        } else {
-            auto k = fused ? k_res_chunks<float, true> : k_res_chunks<float, false>;
-            k<<<gc, 256, 0, st>>>(A.res_n_chunks, A.res_long_rows, A.res_chunk_start, A.res_chunk_row, A.res_rowptr,
-                                  A.res_colidx, (const float *)A.res_values, x, A.res_carry, A.res_done, alpha, y);
+        if (e == cudaSuccess) {
+            if (A.storage == SPADEN_R_16F)
+                e = launch_k(true, fused ? k_res_chunks<__half, true> : k_res_chunks<__half, false>, dim3(gc),
+                             dim3(256), 0, st, (int64_t)A.res_n_chunks, (const int32_t *)A.res_long_rows,
+                             (const int32_t *)A.res_chunk_start, (const int32_t *)A.res_chunk_row,
+                             (const int32_t *)A.res_rowptr, (const int32_t *)A.res_colidx,
+                             (const __half *)A.res_values, x, A.res_carry, A.res_done, alpha, y);
+            else
+                e = launch_k(true, fused ? k_res_chunks<float, true> : k_res_chunks<float, false>, dim3(gc),
+                             dim3(256), 0, st, (int64_t)A.res_n_chunks, (const int32_t *)A.res_long_rows,
+                             (const int32_t *)A.res_chunk_start, (const int32_t *)A.res_chunk_row,
+                             (const int32_t *)A.res_rowptr, (const int32_t *)A.res_colidx,
+                             (const float *)A.res_values, x, A.res_carry, A.res_done, alpha, y);
         }
-        if (A.res_n_chunks > fused_fixup_max())
-            k_res_fixup<<<(unsigned)((32 * A.res_n_long + 255) / 256), 256, 0, st>>>(
-                A.res_n_long, A.res_long_rows, A.res_chunk_start, A.res_carry, alpha, y);
+        if (e == cudaSuccess && !fused)
+            e = launch_k(true, k_res_fixup, dim3((unsigned)((32 * A.res_n_long + 255) / 256)), dim3(256), 0, st,
+                         (int64_t)A.res_n_long, (const int32_t *)A.res_long_rows, (const int32_t *)A.res_chunk_start,
+                         (const float *)A.res_carry, alpha, y);
     }
+    if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }
 

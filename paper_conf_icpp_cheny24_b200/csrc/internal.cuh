@@ -219,6 +219,34 @@ size_t scan_tmp_ints(int64_t count);
 cudaError_t exclusive_scan_i32(const int32_t *in, int32_t *out, int64_t count, int32_t *tmp,
                                cudaStream_t stream);
 
+// Programmatic dependent launch (PDL): a kernel launched with launch_k(dep =
+// true, ...) may start while the previous kernel of the same SpMV call still
+// runs (its prologue and the work that reads only A and x overlap the
+// predecessor's tail); it calls pdl_wait() before touching anything the
+// predecessor writes (y, chunk carries).  Only kernels that follow another
+// kernel of the same call use it, so x -- produced before the call -- is
+// complete.  Both device calls are no-ops under a normal launch.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+bool pdl_enabled();  // SPADEN_PDL=0 disables (A/B), read per call
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k(bool dep, void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                     Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    if (dep && pdl_enabled()) {
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+    }
+    return cudaLaunchKernelEx(&cfg, kernel, args...);
+}
+
 // device helpers
 __device__ __forceinline__ int warp_min_i32(int v) {
 #pragma unroll

@@ -545,6 +545,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
     __shared__ uint64_t full_bar[kMaxStages], empty_bar[kMaxStages];
     __shared__ StageHdr hdr[kMaxStages];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    pdl_trigger();
     if (threadIdx.x == 0) {
         for (int s = 0; s < stages; ++s) {
             mbar_init(smem_u32(&full_bar[s]), 1);
@@ -763,6 +764,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             }
             if (__shfl_sync(kFull, last, 0)) {  // phase 2: this warp completed the tile
                 __threadfence_block();
+                pdl_wait();  // y of the previous kernel (hybrid residual pass); no-op when not PDL-launched
                 const int4 h2 = lds_i4_volatile(a_hdr + 32u);  // br0, nbr, b0, a_rp
                 if constexpr (K > 1)
                     reduce_tile_k<K>((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, ldy);
@@ -886,6 +888,7 @@ k_spmv_warp(int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int 
             }
         }
         __syncwarp();
+        pdl_wait();
         reduce_tile(a_rp, a_part, nbr, b0, br0, lane, m, alpha, beta, y, PeerOut{});  // phase 2
         __syncwarp();
     }
@@ -929,6 +932,7 @@ __global__ void __launch_bounds__(256)
 k_spmv_long_fixup(int64_t m, int nlong, const int32_t *__restrict__ long_rows,
                   const int32_t *__restrict__ chunk_start, const float *carry, float alpha, float beta,
                   float *__restrict__ y, const PeerOut po) {
+    pdl_wait();
     const int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (j < nlong) long_fixup_row(m, (int)j, threadIdx.x & 31, long_rows, chunk_start, carry, alpha, beta, y, po);
 }
@@ -949,6 +953,7 @@ k_spmv_long_chunks(int nchunks, const int32_t *__restrict__ long_rows, const int
                    const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
                    int nbc_vec, float *carry, int32_t *__restrict__ done, int64_t m, float alpha, float beta,
                    float *__restrict__ y, const PeerOut po) {
+    pdl_trigger();
     const int w = (int)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
     const int lane = threadIdx.x & 31;
     if (w >= nchunks) return;
@@ -993,6 +998,7 @@ k_spmv_long_chunks(int nchunks, const int32_t *__restrict__ long_rows, const int
             last = atomicAdd(done + j, 1) == chunk_start[j + 1] - chunk_start[j] - 1;
         }
     }
+    pdl_wait();  // fix-up below reads y; unfused: still complete only after the predecessor
     if (FUSED && __shfl_sync(kFull, last, 0)) {
         __threadfence();
         long_fixup_row(m, j, lane, long_rows, chunk_start, carry, alpha, beta, y, po);
@@ -1067,7 +1073,7 @@ unsigned long long x_texture(const float *x, int64_t n4) {
 
 template <typename V, int DEC, int CONSUMERS, int MINB>
 cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, const float *x, float beta,
-                             float *y, cudaStream_t st, const PeerOut &po) {
+                             float *y, cudaStream_t st, const PeerOut &po, bool dep) {
     const int nbc_vec = ((uintptr_t)x & 31u) == 0 ? (int)(A.n / 8) : 0;
     const size_t smem = (size_t)cfg.stages * cfg.stage_bytes;
     static size_t occ_smem = 0;  // resident CTAs per SM (registers, smem), cached per smem size
@@ -1081,27 +1087,34 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
         occ = std::max(1, std::min(occ, MINB));
         occ_smem = smem;
     }
+    cudaError_t e = cudaSuccess;
     if (A.n_tiles > 0) {
         const int grid = (int)std::min<int64_t>(A.n_tiles, (int64_t)sm_count() * occ);
         const unsigned long long texx = x_texture(x, 2 * (int64_t)nbc_vec);
-        k_spmv_tiled<V, DEC, CONSUMERS, MINB><<<grid, 32 * (CONSUMERS + 1), smem, st>>>(
-            cfg.stages, cfg.stage_bytes, A.m, A.tiles, (int)A.n_tiles, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y, 0, 0, po, texx);
+        e = launch_k(dep, k_spmv_tiled<V, DEC, CONSUMERS, MINB>, dim3(grid), dim3(32 * (CONSUMERS + 1)), smem, st,
+                     cfg.stages, cfg.stage_bytes, (int64_t)A.m, (const TileDesc *)A.tiles, (int)A.n_tiles,
+                     (const int32_t *)A.blk_rowptr, (const int32_t *)A.blk_col, (const uint64_t *)A.bitmap,
+                     (const int32_t *)A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y, (int64_t)0,
+                     (int64_t)0, po, texx);
+        dep = true;
     }
-    if (A.n_long > 0) {
-        const int64_t threads = 32 * A.n_chunks;
-        if (A.n_chunks <= fused_fixup_max())
-            k_spmv_long_chunks<V, (DEC != 0), true><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
-            (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, A.m, alpha, beta, y, po);
-        else
-            k_spmv_long_chunks<V, (DEC != 0), false><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
-            (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, A.m, alpha, beta, y, po);
-        if (A.n_chunks > fused_fixup_max())
-            k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
-                A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, po);
+    if (A.n_long > 0 && e == cudaSuccess) {
+        const unsigned g = (unsigned)((32 * A.n_chunks + 255) / 256);
+        const bool fused = A.n_chunks <= fused_fixup_max();
+        // many chunks: a normal launch (an early-launched grid of many waves would
+        // park finished CTAs in pdl_wait next to the tiled kernel: rmat22 pure
+        // 1.33 -> 2.20 ms); few chunks: PDL hides the launch and ramp latency
+        e = launch_k(dep && fused, fused ? k_spmv_long_chunks<V, (DEC != 0), true> : k_spmv_long_chunks<V, (DEC != 0), false>,
+                     dim3(g), dim3(256), 0, st, (int)A.n_chunks, (const int32_t *)A.long_rows,
+                     (const int32_t *)A.chunk_start, (const int32_t *)A.chunk_row, (const int32_t *)A.blk_rowptr,
+                     (const int32_t *)A.blk_col, (const uint64_t *)A.bitmap, (const int32_t *)A.blk_offset,
+                     (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, (int64_t)A.m, alpha, beta, y, po);
+        if (e == cudaSuccess && !fused)
+            e = launch_k(true, k_spmv_long_fixup, dim3((unsigned)((32 * A.n_long + 255) / 256)), dim3(256), 0, st,
+                         (int64_t)A.m, (int)A.n_long, (const int32_t *)A.long_rows, (const int32_t *)A.chunk_start,
+                         (const float *)A.carry, alpha, beta, y, po);
     }
+    if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }
 
@@ -1146,23 +1159,23 @@ cudaError_t launch_warp_cfg(const Matrix &A, const TileCfg &cfg, float alpha, co
 
 template <typename V, int DEC>
 cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st,
-                         const PeerOut &po) {
+                         const PeerOut &po, bool dep) {
     const TileCfg cfg = tile_cfg(A.tile_cfg);
     switch (A.tile_cfg) {
     case 4: return launch_warp_cfg<V, DEC, 4, 2>(A, cfg, alpha, x, beta, y, st);
-    case 5: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po);
-    case 6: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po);
-    case 7: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
-    case 8: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
-    case 9: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
-    case 10: return launch_tiled_cfg<V, DEC, 4, 6>(A, cfg, alpha, x, beta, y, st, po);
-    case 11: return launch_tiled_cfg<V, DEC, 4, 5>(A, cfg, alpha, x, beta, y, st, po);
-    case 12: return launch_tiled_cfg<V, DEC, 4, 4>(A, cfg, alpha, x, beta, y, st, po);
-    case 13: return launch_tiled_cfg<V, DEC, 4, 6>(A, cfg, alpha, x, beta, y, st, po);
-    case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po);
-    case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po);
-    case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po);
-    default: return launch_tiled_cfg<V, DEC, 16, 1>(A, cfg, alpha, x, beta, y, st, po);
+    case 5: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 6: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 7: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 8: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 9: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 10: return launch_tiled_cfg<V, DEC, 4, 6>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 11: return launch_tiled_cfg<V, DEC, 4, 5>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 12: return launch_tiled_cfg<V, DEC, 4, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 13: return launch_tiled_cfg<V, DEC, 4, 6>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
+    default: return launch_tiled_cfg<V, DEC, 16, 1>(A, cfg, alpha, x, beta, y, st, po, dep);
     }
 }
 
@@ -1227,6 +1240,11 @@ cudaError_t launch_spmm(const Matrix &A, const TileDesc *tiles, int64_t ntiles, 
 
 }  // namespace
 
+bool pdl_enabled() {
+    const char *e = getenv("SPADEN_PDL");
+    return !(e && e[0] == '0');
+}
+
 int64_t fused_fixup_max() {  // SPADEN_FUSED_FIXUP_MAX overrides (tests), read per call
     const char *e = getenv("SPADEN_FUSED_FIXUP_MAX");
     return e ? atoll(e) : kFusedFixupMaxChunks;
@@ -1286,6 +1304,7 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
     // hybrid (NEXT-1): the residual pass runs first and applies beta to every row
     // (y = beta*y + alpha*A_res*x); the bitBSR kernels then accumulate (beta = 1)
     // over the block-rows that hold blocks (the schedule skips the others)
+    const bool dep = A.res_max_popc > 0;  // bitBSR kernels follow the residual pass (PDL)
     if (A.res_max_popc > 0) {
         SPADEN_CUDA_TRY(residual_first(A, alpha, x, beta, y, st));
         beta = 1.f;
@@ -1321,20 +1340,20 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
     cudaError_t e;
     if (A.storage == SPADEN_R_16F) {
         switch (dec) {
-        case 0: e = launch_tiled<__half, 0>(A, alpha, x, beta, y, st, po); break;
-        case 2: e = launch_tiled<__half, 2>(A, alpha, x, beta, y, st, po); break;
-        case 4: e = launch_tiled<__half, 4>(A, alpha, x, beta, y, st, po); break;
-        case 5: e = launch_tiled<__half, 5>(A, alpha, x, beta, y, st, po); break;
-        case 6: e = launch_tiled<__half, 6>(A, alpha, x, beta, y, st, po); break;
-        default: e = launch_tiled<__half, 1>(A, alpha, x, beta, y, st, po);
+        case 0: e = launch_tiled<__half, 0>(A, alpha, x, beta, y, st, po, dep); break;
+        case 2: e = launch_tiled<__half, 2>(A, alpha, x, beta, y, st, po, dep); break;
+        case 4: e = launch_tiled<__half, 4>(A, alpha, x, beta, y, st, po, dep); break;
+        case 5: e = launch_tiled<__half, 5>(A, alpha, x, beta, y, st, po, dep); break;
+        case 6: e = launch_tiled<__half, 6>(A, alpha, x, beta, y, st, po, dep); break;
+        default: e = launch_tiled<__half, 1>(A, alpha, x, beta, y, st, po, dep);
         }
     } else {  // (the tensor-core ablation exists for fp16 values only)
         switch (dec) {
-        case 0: e = launch_tiled<float, 0>(A, alpha, x, beta, y, st, po); break;
-        case 2: e = launch_tiled<float, 2>(A, alpha, x, beta, y, st, po); break;
-        case 5: e = launch_tiled<float, 5>(A, alpha, x, beta, y, st, po); break;
-        case 6: e = launch_tiled<float, 6>(A, alpha, x, beta, y, st, po); break;
-        default: e = launch_tiled<float, 1>(A, alpha, x, beta, y, st, po);
+        case 0: e = launch_tiled<float, 0>(A, alpha, x, beta, y, st, po, dep); break;
+        case 2: e = launch_tiled<float, 2>(A, alpha, x, beta, y, st, po, dep); break;
+        case 5: e = launch_tiled<float, 5>(A, alpha, x, beta, y, st, po, dep); break;
+        case 6: e = launch_tiled<float, 6>(A, alpha, x, beta, y, st, po, dep); break;
+        default: e = launch_tiled<float, 1>(A, alpha, x, beta, y, st, po, dep);
         }
     }
     if (e != cudaSuccess) return cuda_status(e, "launching k_spmv_tiled");
