@@ -303,37 +303,42 @@ template <typename V, int L>
 __device__ __forceinline__ void res_binned_row(int64_t g, int64_t nrows, const int32_t *__restrict__ perm,
                                                const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
                                                const V *__restrict__ val, const float *__restrict__ x, float alpha,
-                                               float *__restrict__ y) {
+                                               float beta, float *__restrict__ y) {
     const int sub = threadIdx.x & (L - 1);
-    if (g >= nrows) {  // uniform within the group
-        pdl_wait();    // (every PDL kernel completes after its predecessor: keeps the chain ordered)
-        return;
-    }
+    if (g >= nrows) return;  // uniform within the group
     const int row = __ldg(perm + g);
     const int k0 = __ldg(rp + row), k1 = __ldg(rp + row + 1);
+    const float yold = (sub == 0 && beta != 0.f) ? y[row] : 0.f;  // fetched before the gathers
     float a = res_lane_sum<V, L>(k0 + sub, k1, col, val, x);
-    pdl_wait();  // y (beta pass) from the previous kernel
-    const float yold = sub == 0 ? y[row] : 0.f;
     if constexpr (L > 1) {
         const unsigned gmask = (L == 32 ? kFull : ((1u << (L & 31)) - 1u)) << (threadIdx.x & (32 - L));
 #pragma unroll
         for (int o = L / 2; o > 0; o >>= 1) a += __shfl_xor_sync(gmask, a, o);
     }
-    if (sub == 0) y[row] = fmaf(alpha, a, yold);
+    if (sub == 0) y[row] = fmaf(alpha, a, beta != 0.f ? beta * yold : 0.f);
+}
+
+// rows without binned entries (empty, or long: their chunks accumulate later):
+// y = beta*y only (y not read when beta = 0, untouched when beta = 1)
+__device__ __forceinline__ void res_scale_row(int64_t g, int64_t nrows, const int32_t *__restrict__ perm, float beta,
+                                              float *__restrict__ y) {
+    if (g >= nrows || beta == 1.f) return;
+    const int row = __ldg(perm + g);
+    y[row] = beta != 0.f ? beta * y[row] : 0.f;
 }
 
 template <typename V>
 __global__ void __launch_bounds__(256)
 k_residual_binned(ResBins bins, const int32_t *__restrict__ perm, const int32_t *__restrict__ rp,
                   const int32_t *__restrict__ col, const V *__restrict__ val, const float *__restrict__ x,
-                  float alpha, float *__restrict__ y) {
+                  float alpha, float beta, float *__restrict__ y) {
     pdl_trigger();
     // class of this CTA; static indices only (a dynamic index into the kernel
     // parameter struct would copy it to local memory in every thread)
     int c = 0;
     int64_t cs = bins.cta_start[0], r0 = bins.row_start[0], r1 = bins.row_start[1];
 #pragma unroll
-    for (int k = 1; k < kResClasses; ++k)
+    for (int k = 1; k <= kResClasses; ++k)
         if ((int64_t)blockIdx.x >= bins.cta_start[k]) {
             c = k;
             cs = bins.cta_start[k];
@@ -343,12 +348,13 @@ k_residual_binned(ResBins bins, const int32_t *__restrict__ perm, const int32_t 
     const int64_t cta = (int64_t)blockIdx.x - cs, nrows = r1 - r0;
     const int32_t *p = perm + r0;
     switch (c) {  // block-uniform
-    case 0: res_binned_row<V, 1>(cta * 256 + threadIdx.x, nrows, p, rp, col, val, x, alpha, y); break;
-    case 1: res_binned_row<V, 2>(cta * 128 + threadIdx.x / 2, nrows, p, rp, col, val, x, alpha, y); break;
-    case 2: res_binned_row<V, 4>(cta * 64 + threadIdx.x / 4, nrows, p, rp, col, val, x, alpha, y); break;
-    case 3: res_binned_row<V, 8>(cta * 32 + threadIdx.x / 8, nrows, p, rp, col, val, x, alpha, y); break;
-    case 4: res_binned_row<V, 16>(cta * 16 + threadIdx.x / 16, nrows, p, rp, col, val, x, alpha, y); break;
-    default: res_binned_row<V, 32>(cta * 8 + threadIdx.x / 32, nrows, p, rp, col, val, x, alpha, y);
+    case 0: res_binned_row<V, 1>(cta * 256 + threadIdx.x, nrows, p, rp, col, val, x, alpha, beta, y); break;
+    case 1: res_binned_row<V, 2>(cta * 128 + threadIdx.x / 2, nrows, p, rp, col, val, x, alpha, beta, y); break;
+    case 2: res_binned_row<V, 4>(cta * 64 + threadIdx.x / 4, nrows, p, rp, col, val, x, alpha, beta, y); break;
+    case 3: res_binned_row<V, 8>(cta * 32 + threadIdx.x / 8, nrows, p, rp, col, val, x, alpha, beta, y); break;
+    case 4: res_binned_row<V, 16>(cta * 16 + threadIdx.x / 16, nrows, p, rp, col, val, x, alpha, beta, y); break;
+    case 5: res_binned_row<V, 32>(cta * 8 + threadIdx.x / 32, nrows, p, rp, col, val, x, alpha, beta, y); break;
+    default: res_scale_row(cta * 256 + threadIdx.x, nrows, p, beta, y);  // class kResClasses
     }
 }
 
@@ -358,7 +364,8 @@ __global__ void k_res_class_flag(int64_t m, const int32_t *__restrict__ rp, int 
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i < m) {
         const int len = rp[i + 1] - rp[i];
-        flag[i] = (len > 0 && len <= kResLongRow && (c < 0 || res_class(len) == c)) ? 1 : 0;  // c < 0: any
+        const bool binned = len > 0 && len <= kResLongRow;
+        flag[i] = (c == kResClasses ? !binned : (binned && res_class(len) == c)) ? 1 : 0;
     }
 }
 __global__ void k_res_class_scatter(int64_t m, const int32_t *__restrict__ pos, int32_t *__restrict__ perm) {
@@ -420,19 +427,13 @@ spaden_status_t residual_long_rows(Matrix *A, cudaStream_t st) {
             e = cudaGetLastError();
         }
     }
-    // length bins of the other non-empty rows
+    // every row in one class: length bins of the rows with 1..kResLongRow
+    // entries, then class kResClasses (empty or long rows: beta only)
     int32_t *perm_pos = nullptr;
     ResBins bins{};
     int64_t total = 0;
-    {  // number of binned rows -> permutation size
-        k_res_class_flag<<<g, 256, 0, st>>>(m, A->res_rowptr, -1, flag);
-        if (e == cudaSuccess) e = exclusive_scan_i32(flag, flag, m, scan_tmp, st);
-        int32_t nb = 0;
-        if (e == cudaSuccess) e = cudaMemcpyAsync(&nb, flag + m, 4, cudaMemcpyDeviceToHost, st);
-        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-        if (e == cudaSuccess) e = cudaMalloc(&perm_pos, 4 * (size_t)std::max(1, nb));
-    }
-    for (int c = 0; c < kResClasses && e == cudaSuccess; ++c) {
+    if (e == cudaSuccess) e = cudaMalloc(&perm_pos, 4 * (size_t)std::max<int64_t>(1, m));
+    for (int c = 0; c <= kResClasses && e == cudaSuccess; ++c) {
         bins.row_start[c] = total;
         k_res_class_flag<<<g, 256, 0, st>>>(m, A->res_rowptr, c, flag);
         e = exclusive_scan_i32(flag, flag, m, scan_tmp, st);
@@ -445,14 +446,15 @@ spaden_status_t residual_long_rows(Matrix *A, cudaStream_t st) {
         }
         total += cnt;
     }
-    bins.row_start[kResClasses] = total;
+    bins.row_start[kResClasses + 1] = total;
     int64_t ctas = 0;
-    for (int c = 0; c < kResClasses; ++c) {
+    for (int c = 0; c <= kResClasses; ++c) {
         bins.cta_start[c] = ctas;
-        const int64_t lanes = (bins.row_start[c + 1] - bins.row_start[c]) << c;  // L = 2^c per row
+        const int lpr = c < kResClasses ? (1 << c) : 1;  // lanes per row
+        const int64_t lanes = (bins.row_start[c + 1] - bins.row_start[c]) * lpr;
         ctas += (lanes + 255) / 256;
     }
-    bins.cta_start[kResClasses] = ctas;
+    bins.cta_start[kResClasses + 1] = ctas;
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     cudaFreeAsync(tmp, st);
     if (e != cudaSuccess) {
@@ -548,57 +550,57 @@ __global__ void k_scale(int64_t m, float beta, float *__restrict__ y) {
 }
 }  // namespace
 
+// Hybrid SpMV, first part: y = beta*y + alpha*A_res*x on every row.  The binned
+// kernel (a normal launch: it follows whatever produced x) applies beta itself
+// -- rows of the last class only get y = beta*y -- so y is fetched before the
+// gathers; long residual rows then accumulate their chunks (PDL launches).
+// SPADEN_RES=fixed: beta pass (memset / scale) + the 16-lane kernel (ablation).
 cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st) {
     if (A.m == 0) return cudaSuccess;
-    cudaError_t e = cudaSuccess;
-    if (beta == 0.f) e = cudaMemsetAsync(y, 0, sizeof(float) * (size_t)A.m, st);
-    else if (beta != 1.f) k_scale<<<(unsigned)std::min<int64_t>((A.m + 255) / 256, 148 * 16), 256, 0, st>>>(A.m, beta, y);
-    if (e == cudaSuccess) e = cudaGetLastError();
-    if (e == cudaSuccess) e = residual_spmv(A, alpha, x, y, st);
-    return e;
-}
-
-cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y, cudaStream_t st) {
-    if (A.res_nnz == 0) return cudaSuccess;
-    const char *env = getenv("SPADEN_RES");  // "fixed": the 16-lane kernel (ablation), read per call
+    const char *env = getenv("SPADEN_RES");  // read per call
     const bool binned = A.res_perm && !(env && env[0] == 'f');
-    const unsigned grid = (unsigned)((kResLanes * A.m + 255) / 256);  // one lane group per row
     cudaError_t e = cudaSuccess;
     if (binned) {
-        const int64_t nc = A.res_bins.cta_start[kResClasses];
+        const int64_t nc = A.res_bins.cta_start[kResClasses + 1];
         if (nc > 0) {
             if (A.storage == SPADEN_R_16F)
-                e = launch_k(true, k_residual_binned<__half>, dim3((unsigned)nc), dim3(256), 0, st, A.res_bins,
+                e = launch_k(false, k_residual_binned<__half>, dim3((unsigned)nc), dim3(256), 0, st, A.res_bins,
                              (const int32_t *)A.res_perm, (const int32_t *)A.res_rowptr,
-                             (const int32_t *)A.res_colidx, (const __half *)A.res_values, x, alpha, y);
+                             (const int32_t *)A.res_colidx, (const __half *)A.res_values, x, alpha, beta, y);
             else
-                e = launch_k(true, k_residual_binned<float>, dim3((unsigned)nc), dim3(256), 0, st, A.res_bins,
+                e = launch_k(false, k_residual_binned<float>, dim3((unsigned)nc), dim3(256), 0, st, A.res_bins,
                              (const int32_t *)A.res_perm, (const int32_t *)A.res_rowptr,
-                             (const int32_t *)A.res_colidx, (const float *)A.res_values, x, alpha, y);
+                             (const int32_t *)A.res_colidx, (const float *)A.res_values, x, alpha, beta, y);
         }
-    } else if (A.storage == SPADEN_R_16F)
-        k_residual<__half, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
-                                                            (const __half *)A.res_values, x, alpha, y);
-    else
-        k_residual<float, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
-                                                           (const float *)A.res_values, x, alpha, y);
-    if (A.res_n_long > 0) {
+    } else {
+        if (beta == 0.f) e = cudaMemsetAsync(y, 0, sizeof(float) * (size_t)A.m, st);
+        else if (beta != 1.f)
+            k_scale<<<(unsigned)std::min<int64_t>((A.m + 255) / 256, 148 * 16), 256, 0, st>>>(A.m, beta, y);
+        const unsigned grid = (unsigned)((kResLanes * A.m + 255) / 256);  // one lane group per row
+        if (e == cudaSuccess && A.res_nnz > 0) {
+            if (A.storage == SPADEN_R_16F)
+                k_residual<__half, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
+                                                                    (const __half *)A.res_values, x, alpha, y);
+            else
+                k_residual<float, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
+                                                                   (const float *)A.res_values, x, alpha, y);
+        }
+    }
+    if (e == cudaSuccess && A.res_n_long > 0) {
         const unsigned gc = (unsigned)((32 * A.res_n_chunks + 255) / 256);
         const bool fused = A.res_n_chunks <= fused_fixup_max();
-        if (e == cudaSuccess) {
-            if (A.storage == SPADEN_R_16F)
-                e = launch_k(true, fused ? k_res_chunks<__half, true> : k_res_chunks<__half, false>, dim3(gc),
-                             dim3(256), 0, st, (int64_t)A.res_n_chunks, (const int32_t *)A.res_long_rows,
-                             (const int32_t *)A.res_chunk_start, (const int32_t *)A.res_chunk_row,
-                             (const int32_t *)A.res_rowptr, (const int32_t *)A.res_colidx,
-                             (const __half *)A.res_values, x, A.res_carry, A.res_done, alpha, y);
-            else
-                e = launch_k(true, fused ? k_res_chunks<float, true> : k_res_chunks<float, false>, dim3(gc),
-                             dim3(256), 0, st, (int64_t)A.res_n_chunks, (const int32_t *)A.res_long_rows,
-                             (const int32_t *)A.res_chunk_start, (const int32_t *)A.res_chunk_row,
-                             (const int32_t *)A.res_rowptr, (const int32_t *)A.res_colidx,
-                             (const float *)A.res_values, x, A.res_carry, A.res_done, alpha, y);
-        }
+        if (A.storage == SPADEN_R_16F)
+            e = launch_k(true, fused ? k_res_chunks<__half, true> : k_res_chunks<__half, false>, dim3(gc), dim3(256),
+                         0, st, (int64_t)A.res_n_chunks, (const int32_t *)A.res_long_rows,
+                         (const int32_t *)A.res_chunk_start, (const int32_t *)A.res_chunk_row,
+                         (const int32_t *)A.res_rowptr, (const int32_t *)A.res_colidx, (const __half *)A.res_values,
+                         x, A.res_carry, A.res_done, alpha, y);
+        else
+            e = launch_k(true, fused ? k_res_chunks<float, true> : k_res_chunks<float, false>, dim3(gc), dim3(256),
+                         0, st, (int64_t)A.res_n_chunks, (const int32_t *)A.res_long_rows,
+                         (const int32_t *)A.res_chunk_start, (const int32_t *)A.res_chunk_row,
+                         (const int32_t *)A.res_rowptr, (const int32_t *)A.res_colidx, (const float *)A.res_values,
+                         x, A.res_carry, A.res_done, alpha, y);
         if (e == cudaSuccess && !fused)
             e = launch_k(true, k_res_fixup, dim3((unsigned)((32 * A.res_n_long + 255) / 256)), dim3(256), 0, st,
                          (int64_t)A.res_n_long, (const int32_t *)A.res_long_rows, (const int32_t *)A.res_chunk_start,

@@ -59,9 +59,9 @@ struct spaden_matrix_s {
     int32_t *res_chunk_row = nullptr;    // [res_n_chunks] index into res_long_rows
     float *res_carry = nullptr;          // [res_n_chunks]
     int32_t *res_done = nullptr;         // [res_n_long] chunks finished per long row (0 between calls)
-    int32_t *res_perm = nullptr;         // rows of 1..kResLongRow entries, grouped by length class
+    int32_t *res_perm = nullptr;         // all rows, grouped by length class (then empty / long rows)
     struct ResBins {                     // class c: perm[row_start[c], row_start[c+1]), CTAs from cta_start[c]
-        int64_t row_start[7], cta_start[7];
+        int64_t row_start[8], cta_start[8];  // classes 0..kResClasses (the last: empty / long rows)
     } res_bins = {};
     int64_t res_aux_bytes = 0;           // perm + long-row chunk lists
 
@@ -201,9 +201,8 @@ spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *ro
 
 // hybrid split (hybrid.cu): move blocks with popc <= t into a CSR residual
 spaden_status_t split_residual(Matrix *A, int t, cudaStream_t stream);
-cudaError_t residual_spmv(const Matrix &A, float alpha, const float *x, float *y, cudaStream_t stream);
-// hybrid SpMV, first pass: y = beta*y (y not read when beta = 0), then the residual
-// pass y += alpha*A_res*x; the bitBSR kernels follow with beta = 1
+// hybrid SpMV, first part: y = beta*y + alpha*A_res*x on every row (y not read
+// when beta = 0); the bitBSR kernels follow with beta = 1
 cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t stream);
 
 // SpMV (spmv.cu)

@@ -348,6 +348,50 @@ def test_cuda_graph_capture(sp, torch):
     assert torch.equal(y, ref)
 
 
+@pytest.mark.parametrize("t", [0, 2])
+def test_cuda_graph_capture_chain(sp, torch, t):
+    """The multi-kernel chains (hybrid residual pass, long-row chunks with the
+    fused fix-up, programmatic dependent launches) captured in a CUDA graph and
+    replayed repeatedly give the eager result bitwise, with alpha/beta."""
+    A = hub_matrix(m=96, n=200_003, hub_rows=(3, 60, 61), hub_nnz=60_000, seed=5)
+    rp, ci, v = dev(torch, A)
+    M = sp.convert(rp, ci, v, A.n, residual_max_popc=t)
+    torch.cuda.synchronize()
+    assert M.info.n_long >= 1 or M.info.residual_nnz > 0
+    x = torch.from_numpy(W.vector(A.n, 19)).cuda()
+    y0 = torch.from_numpy(W.vector(A.m, 20)).cuda()
+    s = torch.cuda.Stream()
+    y = y0.clone()
+    with torch.cuda.stream(s):
+        M.spmv(x, y, alpha=0.5, beta=-2.0, stream=s)
+    torch.cuda.synchronize()
+    ref = y.clone()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        M.spmv(x, y, alpha=0.5, beta=-2.0, stream=s)
+    for _ in range(3):
+        y.copy_(y0)
+        g.replay()
+        torch.cuda.synchronize()
+        assert torch.equal(y, ref)
+
+
+@pytest.mark.parametrize("t", [0, 3])
+def test_pdl_off_bitwise_equal(sp, torch, t, monkeypatch):
+    """Programmatic dependent launch only changes when kernels may start:
+    SPADEN_PDL=0 (plain stream order) gives the same y bitwise."""
+    A = W.powerlaw(14, 6, seed=3)
+    rp, ci, v = dev(torch, A)
+    M = sp.convert(rp, ci, v, A.n, residual_max_popc=t)
+    x = W.vector(A.n, 21)
+    y0 = W.vector(A.m, 22)
+    ref = gpu_spmv(torch, M, x, alpha=1.25, beta=0.5, y0=y0)
+    monkeypatch.setenv("SPADEN_PDL", "0")
+    assert np.array_equal(gpu_spmv(torch, M, x, alpha=1.25, beta=0.5, y0=y0), ref)
+    ys, s = oracle.spmv(A.rowptr, A.colidx, A.values, x)
+    assert oracle.componentwise_error(ref, 1.25 * ys + 0.5 * y0, 1.25 * s + 0.5 * np.abs(y0)) <= TOL32
+
+
 @pytest.mark.parametrize("name", ["fem62k", "powerlaw1m"])
 def test_configs_full(sp, torch, name):
     A = W.make(name)
