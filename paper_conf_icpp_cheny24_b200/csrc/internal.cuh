@@ -105,7 +105,7 @@ struct TileCfg {
                     // 1: warp pipelines (each warp streams its own tiles; consumers = warps/CTA)
 };
 constexpr int kMaxStages = 8;
-constexpr int kNumTileCfgs = 14;
+constexpr int kNumTileCfgs = 17;
 __host__ __device__ inline TileCfg tile_cfg(int i) {
     switch (i) {
     case 1: return TileCfg{2, 16, 3, 36 * 1024, 0};
@@ -122,6 +122,10 @@ __host__ __device__ inline TileCfg tile_cfg(int i) {
     case 11: return TileCfg{5, 4, 3, 14 * 1024, 0};
     case 12: return TileCfg{4, 4, 3, 18 * 1024, 0};
     case 13: return TileCfg{6, 4, 3, 12 * 1024, 0};
+    // 2 CTAs per SM, deeper rings (4 stages)
+    case 14: return TileCfg{2, 12, 4, 24 * 1024, 0};
+    case 15: return TileCfg{2, 16, 4, 27 * 1024, 0};
+    case 16: return TileCfg{2, 8, 4, 27 * 1024, 0};
     default: return TileCfg{1, 16, 3, 64 * 1024, 0};
     }
 }

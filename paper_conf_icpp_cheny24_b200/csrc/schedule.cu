@@ -123,10 +123,10 @@ int default_tile_cfg(int64_t format_bytes, int value_bytes) {
         if (c >= 0 && c < kNumTileCfgs) return c;
     }
     // measured best on fem1p5m: fp32 values 3 CTAs/SM x 8 consumers
-    // x 3 x 24 KB, fp16 values 6 x 4 x 2 x 18 KB; small matrices need smaller stages to
+    // x 3 x 24 KB, fp16 values 2 x 16 x 4 x 27 KB; small matrices need smaller stages to
     // give every CTA several tiles
     if (format_bytes < kSmallMatrixBytes) return kSmallTileCfg;
-    return value_bytes == 4 ? 2 : 10;
+    return value_bytes == 4 ? 2 : 15;
 }
 
 spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {

@@ -1172,6 +1172,9 @@ cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float bet
     case 11: return launch_tiled_cfg<V, DEC, 4, 5>(A, cfg, alpha, x, beta, y, st, po, dep);
     case 12: return launch_tiled_cfg<V, DEC, 4, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
     case 13: return launch_tiled_cfg<V, DEC, 4, 6>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 14: return launch_tiled_cfg<V, DEC, 12, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 15: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 16: return launch_tiled_cfg<V, DEC, 8, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
     case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
     case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po, dep);
     case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po, dep);

@@ -493,7 +493,7 @@ def test_pagerank_iteration_vs_oracle(sp, torch):
     assert rel.max() <= 1e-5, rel.max()
 
 
-@pytest.mark.parametrize("cfg", list(range(14)))
+@pytest.mark.parametrize("cfg", list(range(17)))
 def test_every_tile_config_same_result(sp, torch, cfg, monkeypatch):
     """All launch shapes (CTA or warp pipelines, SPADEN_TILE_CFG) give the oracle's
     y within tolerance, and block-rows classified alike give bitwise equal y."""
