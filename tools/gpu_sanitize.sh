@@ -1,9 +1,7 @@
 #!/bin/bash
+# compute-sanitizer (memcheck / racecheck / synccheck / initcheck) over tools/sanitize_run.py
 mkdir -p gpurun_out
-timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke.log
-timeout 1500 python -m pytest tests -m gpu -q -x --timeout 900 > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
 for tool in memcheck racecheck synccheck initcheck; do
   timeout 900 compute-sanitizer --tool $tool --target-processes all python tools/sanitize_run.py > gpurun_out/sanitizer_$tool.log 2>&1; echo "rc=$?" >> gpurun_out/sanitizer_$tool.log
 done
-timeout 900 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
-echo done
+for tool in memcheck racecheck synccheck initcheck; do echo "== $tool"; tail -4 gpurun_out/sanitizer_$tool.log; done

@@ -1,6 +1,8 @@
 """Small end-to-end exercise of every kernel for compute-sanitizer
 (memcheck / racecheck / synccheck): conversions in all dtype modes, the tiled
-SpMV, the long-row chunk path, alpha/beta, the batched host pipeline."""
+SpMV, the long-row chunk path (fused and separate fix-up), alpha/beta, the
+hybrid format (binned residual, long residual rows, PDL chain), SpMM, the
+batched host pipeline."""
 import os
 import sys
 
@@ -13,14 +15,14 @@ sys.path.insert(0, os.path.join(ROOT, "tests"))
 
 import paper_conf_icpp_cheny24_b200 as sp  # noqa: E402
 import workloads as W  # noqa: E402
-from test_gpu_parity import hub_matrix  # noqa: E402
+from test_gpu_parity import binned_rows_matrix, hub_matrix  # noqa: E402
 
 
-def run(A, storage):
+def run(A, storage, t=0):
     rp = torch.from_numpy(A.rowptr).cuda()
     ci = torch.from_numpy(A.colidx).cuda()
     v = torch.from_numpy(A.values).cuda()
-    M = sp.convert(rp, ci, v, A.n, storage=storage)
+    M = sp.convert(rp, ci, v, A.n, storage=storage, residual_max_popc=t)
     x = torch.from_numpy(W.vector(A.n, 1)).cuda()
     y = torch.from_numpy(W.vector(A.m, 2)).cuda()
     M.spmv(x, y, alpha=1.0, beta=0.5)
@@ -32,6 +34,17 @@ def run(A, storage):
 for A in (W.h2(), W.tiny(0), W.fem(6, 7, 8, seed=2), hub_matrix(m=40, n=70_001, hub_rows=(3, 30), hub_nnz=40_000)):
     for st in ("fp32", "fp16"):
         run(A, st)
+        run(A, st, t=2)
+for fixup in ("8192", "0"):  # long-row fix-up fused into the chunk kernel / separate launch
+    os.environ["SPADEN_FUSED_FIXUP_MAX"] = fixup
+    run(binned_rows_matrix(), "fp32", t=64)
+    run(hub_matrix(m=40, n=70_001, hub_rows=(3, 30), hub_nnz=40_000), "fp32")
+os.environ.pop("SPADEN_FUSED_FIXUP_MAX")
+B = hub_matrix()
+MB = sp.convert(torch.from_numpy(B.rowptr).cuda(), torch.from_numpy(B.colidx).cuda(),
+                torch.from_numpy(B.values).cuda(), B.n, residual_max_popc=2)
+MB.spmm(torch.from_numpy(np.stack([W.vector(B.n, k) for k in range(4)])).cuda())
+torch.cuda.synchronize()
 A = W.fem(5, 5, 6, seed=1)
 M = sp.convert(torch.from_numpy(A.rowptr).cuda(), torch.from_numpy(A.colidx).cuda(),
                torch.from_numpy(A.values).cuda(), A.n)
