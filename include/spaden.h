@@ -234,6 +234,15 @@ SPADEN_API spaden_status_t spaden_free(spaden_matrix_t A);
 SPADEN_API spaden_status_t spaden_get_info(spaden_matrix_t A, spaden_info_t *info);
 SPADEN_API spaden_status_t spaden_get_arrays(spaden_matrix_t A, spaden_arrays_t *arrays);
 
+/*
+ * spaden_spmv_launch_count -- number of kernel launches (and memsets) one
+ * spaden_spmv(A, ..., beta, ...) call issues on its stream with the current
+ * environment (decode / ablation overrides): the tiled kernel, long-row chunk
+ * and fix-up kernels, the hybrid residual pass.  For the bench's launch
+ * accounting; no device work, no synchronisation.  *count must be non-NULL.
+ */
+SPADEN_API spaden_status_t spaden_spmv_launch_count(spaden_matrix_t A, float beta, int32_t *count);
+
 /* Static strings; never NULL. */
 SPADEN_API const char *spaden_status_string(spaden_status_t s);
 SPADEN_API const char *spaden_last_error_message(void);

@@ -89,6 +89,9 @@ spaden_free.restype = _ST
 spaden_get_info = _lib.spaden_get_info
 spaden_get_info.argtypes = [_P, ctypes.POINTER(spaden_info_t)]
 spaden_get_info.restype = _ST
+spaden_spmv_launch_count = _lib.spaden_spmv_launch_count
+spaden_spmv_launch_count.argtypes = [_P, _F, ctypes.POINTER(ctypes.c_int32)]
+spaden_spmv_launch_count.restype = _ST
 spaden_get_arrays = _lib.spaden_get_arrays
 spaden_get_arrays.argtypes = [_P, ctypes.POINTER(spaden_arrays_t)]
 spaden_get_arrays.restype = _ST
@@ -105,7 +108,7 @@ spaden_version.restype = ctypes.c_char_p
 EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_spmv", "spaden_spmm",
             "spaden_spmv_scatter", "spaden_spmv_host", "spaden_spmv_host_batched",
             "spaden_free",
-            "spaden_get_info", "spaden_get_arrays", "spaden_status_string",
+            "spaden_get_info", "spaden_get_arrays", "spaden_spmv_launch_count", "spaden_status_string",
             "spaden_last_error_message", "spaden_version"]
 
 
@@ -203,6 +206,12 @@ class Matrix:
             out["res_colidx"] = mk(a.res_colidx, i.residual_nnz, "<i4")
             out["res_values"] = mk(a.res_values, i.residual_nnz, vt)
         return out
+
+    def launch_count(self, beta: float = 0.0) -> int:
+        """Kernel launches (and memsets) one spmv(..., beta) call issues (bench accounting)."""
+        c = ctypes.c_int32()
+        _check(spaden_spmv_launch_count(self._h, beta, ctypes.byref(c)), "spaden_spmv_launch_count")
+        return c.value
 
     def spmv(self, x, y=None, alpha: float = 1.0, beta: float = 0.0, stream=None):
         """y = alpha * A x + beta * y on the device (x, y float32 CUDA tensors)."""

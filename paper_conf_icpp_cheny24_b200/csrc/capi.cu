@@ -301,6 +301,15 @@ spaden_status_t spaden_free(spaden_matrix_t A) {
     return SPADEN_OK;
 }
 
+spaden_status_t spaden_spmv_launch_count(spaden_matrix_t A, float beta, int32_t *count) {
+    if (!A || !count) {
+        set_error("NULL handle or count");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    *count = spmv_launch_count(*A, beta);
+    return SPADEN_OK;
+}
+
 spaden_status_t spaden_get_info(spaden_matrix_t A, spaden_info_t *info) {
     if (!A || !info) {
         set_error("NULL handle or info");

@@ -212,6 +212,7 @@ cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float b
 // SpMV (spmv.cu)
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,
                             cudaStream_t stream, const PeerOut *peers = nullptr);
+int spmv_launch_count(const Matrix &A, float beta);  // launches of one spmv_launch (no peers)
 // SpMM: k column-major vectors (spmv.cu)
 spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx, int k, float beta, float *Y,
                             int64_t ldy, cudaStream_t stream);

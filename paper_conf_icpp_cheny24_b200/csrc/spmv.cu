@@ -1295,6 +1295,22 @@ spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx,
     return SPADEN_OK;
 }
 
+// launches issued by spmv_launch (mirrors its dispatch; spaden_spmv_launch_count)
+int spmv_launch_count(const Matrix &A, float beta) {
+    if (A.m == 0) return 0;
+    int n = 0;
+    if (A.res_max_popc > 0) {  // residual_first
+        const char *env = getenv("SPADEN_RES");
+        if (A.res_perm && !(env && env[0] == 'f')) n += A.res_bins.cta_start[kResClasses + 1] > 0 ? 1 : 0;
+        else n += (beta != 1.f ? 1 : 0) + (A.res_nnz > 0 ? 1 : 0);
+        if (A.res_n_long > 0) n += 1 + (A.res_n_chunks > fused_fixup_max() ? 1 : 0);
+    }
+    if (kernel_variant() == 0) return n + 1;
+    n += A.n_tiles > 0 ? 1 : 0;
+    if (A.n_long > 0) n += 1 + (A.n_chunks > fused_fixup_max() ? 1 : 0);
+    return n;
+}
+
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,
                             cudaStream_t st, const PeerOut *peers) {
     if (A.m == 0) return SPADEN_OK;

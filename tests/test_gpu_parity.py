@@ -376,6 +376,42 @@ def test_cuda_graph_capture_chain(sp, torch, t):
         assert torch.equal(y, ref)
 
 
+def graph_nodes(torch, fn):
+    """Number of nodes (kernel launches, memsets) fn() puts on a captured stream."""
+    rt = pytest.importorskip("cuda.bindings.runtime")
+    s = torch.cuda.Stream()
+    fn(s)  # eager warm-up (lazy module loading outside the capture)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph(keep_graph=True)
+    with torch.cuda.graph(g, stream=s):
+        fn(s)
+    out = rt.cudaGraphGetNodes(rt.cudaGraph_t(init_value=g.raw_cuda_graph()))
+    assert int(out[0]) == 0
+    return int(out[-1])
+
+
+@pytest.mark.parametrize("case", ["fem", "hub_fused", "hub_separate", "hyb_long", "hyb_long_sep", "hyb_fixed"])
+@pytest.mark.parametrize("beta", [0.0, 0.5, 1.0])
+def test_launch_count_matches_graph(sp, torch, case, beta, monkeypatch):
+    """spaden_spmv_launch_count (the bench's gpu_launches) equals the number of
+    nodes a captured spaden_spmv puts in a CUDA graph."""
+    if case.endswith("sep"):
+        monkeypatch.setenv("SPADEN_FUSED_FIXUP_MAX", "0")
+    if case == "hub_separate":
+        monkeypatch.setenv("SPADEN_FUSED_FIXUP_MAX", "0")
+    if case == "hyb_fixed":
+        monkeypatch.setenv("SPADEN_RES", "fixed")
+    A = W.fem(6, 7, 8, seed=2) if case == "fem" else (
+        binned_rows_matrix() if case.startswith("hyb") else hub_matrix(m=40, n=70_001, hub_rows=(3, 30), hub_nnz=40_000))
+    t = 2 if case.startswith("hyb") else 0
+    rp, ci, v = dev(torch, A)
+    M = sp.convert(rp, ci, v, A.n, residual_max_popc=t)
+    x = torch.from_numpy(W.vector(A.n, 3)).cuda()
+    y = torch.from_numpy(W.vector(A.m, 4)).cuda()
+    n = graph_nodes(torch, lambda s: M.spmv(x, y, alpha=1.0, beta=beta, stream=s))
+    assert n == M.launch_count(beta) >= 1
+
+
 @pytest.mark.parametrize("t", [0, 3])
 def test_pdl_off_bitwise_equal(sp, torch, t, monkeypatch):
     """Programmatic dependent launch only changes when kernels may start:
