@@ -540,7 +540,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
              const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
              const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
              int nbc_vec, float alpha, float beta, float *__restrict__ y, int64_t ldx, int64_t ldy,
-             const PeerOut po, unsigned long long texx) {
+             const PeerOut po, unsigned long long texx, int wait_y) {
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t full_bar[kMaxStages], empty_bar[kMaxStages];
     __shared__ StageHdr hdr[kMaxStages];
@@ -616,6 +616,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                 }
             }
         }
+        pdl_wait();  // a PDL-launched grid completes only after its predecessor
         return;
     }
 
@@ -764,7 +765,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             }
             if (__shfl_sync(kFull, last, 0)) {  // phase 2: this warp completed the tile
                 __threadfence_block();
-                pdl_wait();  // y of the previous kernel (hybrid residual pass); no-op when not PDL-launched
+                if (wait_y) pdl_wait();  // y of the previous kernels (hybrid residual pass)
                 const int4 h2 = lds_i4_volatile(a_hdr + 32u);  // br0, nbr, b0, a_rp
                 if constexpr (K > 1)
                     reduce_tile_k<K>((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, ldy);
@@ -775,6 +776,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
         __syncwarp();
         if (lane == 0) mbar_arrive(a_empty0 + 8u * s);
     }
+    pdl_wait();  // a PDL-launched grid completes only after its predecessor
 }
 
 // ==========================================================================
@@ -1088,28 +1090,39 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
         occ_smem = smem;
     }
     cudaError_t e = cudaSuccess;
-    if (A.n_tiles > 0) {
+    const bool hyb = A.res_max_popc > 0;  // the residual pass wrote y before these kernels
+    const bool fused = A.n_long > 0 && A.n_chunks <= fused_fixup_max();
+    auto launch_long = [&](bool d) {
+        const unsigned g = (unsigned)((32 * A.n_chunks + 255) / 256);
+        return launch_k(d, fused ? k_spmv_long_chunks<V, (DEC != 0), true> : k_spmv_long_chunks<V, (DEC != 0), false>,
+                        dim3(g), dim3(256), 0, st, (int)A.n_chunks, (const int32_t *)A.long_rows,
+                        (const int32_t *)A.chunk_start, (const int32_t *)A.chunk_row, (const int32_t *)A.blk_rowptr,
+                        (const int32_t *)A.blk_col, (const uint64_t *)A.bitmap, (const int32_t *)A.blk_offset,
+                        (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, (int64_t)A.m, alpha, beta, y, po);
+    };
+    // few long-row chunks (one wave): launch them first, the tiled kernel then
+    // starts (PDL) while they run -- their rows are disjoint, so it waits for
+    // them only before exiting.  Many chunks: tiled kernel, then the chunks as a
+    // normal launch (an early-launched grid of many waves would park finished
+    // CTAs in pdl_wait next to the tiled kernel: rmat22 pure 1.33 -> 2.20 ms),
+    // then the separate fix-up.
+    if (fused) {
+        e = launch_long(dep);
+        dep = true;
+    }
+    if (A.n_tiles > 0 && e == cudaSuccess) {
         const int grid = (int)std::min<int64_t>(A.n_tiles, (int64_t)sm_count() * occ);
         const unsigned long long texx = x_texture(x, 2 * (int64_t)nbc_vec);
         e = launch_k(dep, k_spmv_tiled<V, DEC, CONSUMERS, MINB>, dim3(grid), dim3(32 * (CONSUMERS + 1)), smem, st,
                      cfg.stages, cfg.stage_bytes, (int64_t)A.m, (const TileDesc *)A.tiles, (int)A.n_tiles,
                      (const int32_t *)A.blk_rowptr, (const int32_t *)A.blk_col, (const uint64_t *)A.bitmap,
                      (const int32_t *)A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y, (int64_t)0,
-                     (int64_t)0, po, texx);
+                     (int64_t)0, po, texx, (int)hyb);
         dep = true;
     }
-    if (A.n_long > 0 && e == cudaSuccess) {
-        const unsigned g = (unsigned)((32 * A.n_chunks + 255) / 256);
-        const bool fused = A.n_chunks <= fused_fixup_max();
-        // many chunks: a normal launch (an early-launched grid of many waves would
-        // park finished CTAs in pdl_wait next to the tiled kernel: rmat22 pure
-        // 1.33 -> 2.20 ms); few chunks: PDL hides the launch and ramp latency
-        e = launch_k(dep && fused, fused ? k_spmv_long_chunks<V, (DEC != 0), true> : k_spmv_long_chunks<V, (DEC != 0), false>,
-                     dim3(g), dim3(256), 0, st, (int)A.n_chunks, (const int32_t *)A.long_rows,
-                     (const int32_t *)A.chunk_start, (const int32_t *)A.chunk_row, (const int32_t *)A.blk_rowptr,
-                     (const int32_t *)A.blk_col, (const uint64_t *)A.bitmap, (const int32_t *)A.blk_offset,
-                     (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, (int64_t)A.m, alpha, beta, y, po);
-        if (e == cudaSuccess && !fused)
+    if (A.n_long > 0 && !fused && e == cudaSuccess) {
+        e = launch_long(false);
+        if (e == cudaSuccess)
             e = launch_k(true, k_spmv_long_fixup, dim3((unsigned)((32 * A.n_long + 255) / 256)), dim3(256), 0, st,
                          (int64_t)A.m, (int)A.n_long, (const int32_t *)A.long_rows, (const int32_t *)A.chunk_start,
                          (const float *)A.carry, alpha, beta, y, po);
@@ -1204,7 +1217,7 @@ cudaError_t launch_spmm_cfg(const Matrix &A, const TileCfg &cfg, const TileDesc 
         const unsigned long long texx = nbc_vec ? x_texture(X, 2 * (int64_t)nbc_vec + (K - 1) * (ldx / 4)) : 0ull;
         k_spmv_tiled<V, 1, CONSUMERS, MINB, K><<<grid, 32 * (CONSUMERS + 1), smem, st>>>(
             cfg.stages, cfg.stage_bytes, A.m, tiles, (int)ntiles, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, X, nbc_vec, alpha, beta, Y, ldx, ldy, PeerOut{}, texx);
+            A.blk_offset, (const V *)A.values, X, nbc_vec, alpha, beta, Y, ldx, ldy, PeerOut{}, texx, 1);
     }
     if (A.n_long > 0) {  // long block-rows: the SpMV chunk path, once per vector (same arithmetic)
         const int nbc1 = ((uintptr_t)X & 31u) == 0 && ((ldx * 4) % 32) == 0 ? (int)(A.n / 8) : 0;
