@@ -46,11 +46,16 @@ static void release(Matrix *A) {
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap,   A->blk_offset, A->values,
                     A->stage_x,     A->stage_y,  A->pipe_x[0], A->pipe_x[1], A->pipe_x[2],
                     A->pipe_y[0],   A->pipe_y[1], A->pipe_y[2], A->tiles,
-                    A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->chunk_done, A->res_rowptr,
-                    A->res_colidx,  A->res_values, A->res_long_rows, A->res_chunk_start,
-                    A->res_chunk_row, A->res_carry, A->res_done, A->res_perm, A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
+                    A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->chunk_done,
+                    A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
     for (void *p : ptrs)
         if (p) cudaFree(p);
+    for (int q = 0; q < A->n_res_parts; ++q) {
+        const spaden::ResPart &P = A->res[q];
+        void *rp[] = {P.rowptr, P.colidx, P.values, P.long_rows, P.chunk_start, P.chunk_row, P.carry, P.done, P.perm};
+        for (void *p : rp)
+            if (p) cudaFree(p);
+    }
     for (cudaEvent_t e : A->ev)
         if (e) cudaEventDestroy(e);
     if (A->s_h2d) cudaStreamDestroy(A->s_h2d);
@@ -343,9 +348,11 @@ spaden_status_t spaden_get_arrays(spaden_matrix_t A, spaden_arrays_t *v) {
     v->bitmap = A->bitmap;
     v->blk_offset = A->blk_offset;
     v->values = A->values;
-    v->res_rowptr = A->res_rowptr;
-    v->res_colidx = A->res_colidx;
-    v->res_values = A->res_values;
+    // the residual CSR (NULL when it is split into column parts)
+    const bool one = A->n_res_parts == 1;
+    v->res_rowptr = one ? A->res[0].rowptr : nullptr;
+    v->res_colidx = one ? A->res[0].colidx : nullptr;
+    v->res_values = one ? A->res[0].values : nullptr;
     return SPADEN_OK;
 }
 

@@ -392,38 +392,39 @@ __global__ void k_res_chunk_rows(int64_t nlong, const int32_t *__restrict__ cs, 
         for (int c = cs[j]; c < cs[j + 1]; ++c) crow[c] = (int32_t)j;
 }
 
-spaden_status_t residual_long_rows(Matrix *A, cudaStream_t st) {
+// long-row chunk lists and the length-class row permutation of one residual part
+spaden_status_t residual_schedule(Matrix *A, ResPart &P, cudaStream_t st) {
     const int64_t m = A->m;
     const size_t nt = scan_tmp_ints(m + 1);
     int32_t *tmp = nullptr;
     SPADEN_CUDA_TRY(cudaMallocAsync(&tmp, ((size_t)m + 1 + nt + 4) * sizeof(int32_t), st));
     int32_t *flag = tmp, *scan_tmp = tmp + (m + 1);
     const unsigned g = (unsigned)((m + 255) / 256);
-    k_res_long_flag<<<g, 256, 0, st>>>(m, A->res_rowptr, flag);
+    k_res_long_flag<<<g, 256, 0, st>>>(m, P.rowptr, flag);
     cudaError_t e = exclusive_scan_i32(flag, flag, m, scan_tmp, st);
     int32_t nl = 0;
     if (e == cudaSuccess) e = cudaMemcpyAsync(&nl, flag + m, 4, cudaMemcpyDeviceToHost, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     if (e == cudaSuccess && nl > 0) {
-        A->res_n_long = nl;
-        e = cudaMalloc(&A->res_long_rows, 4 * (size_t)nl);
-        if (e == cudaSuccess) e = cudaMalloc(&A->res_chunk_start, 4 * ((size_t)nl + 1));
+        P.n_long = nl;
+        e = cudaMalloc(&P.long_rows, 4 * (size_t)nl);
+        if (e == cudaSuccess) e = cudaMalloc(&P.chunk_start, 4 * ((size_t)nl + 1));
         if (e == cudaSuccess) {
-            k_res_long_list<<<g, 256, 0, st>>>(m, A->res_rowptr, flag, A->res_long_rows, A->res_chunk_start);
-            e = exclusive_scan_i32(A->res_chunk_start, A->res_chunk_start, nl, scan_tmp, st);
+            k_res_long_list<<<g, 256, 0, st>>>(m, P.rowptr, flag, P.long_rows, P.chunk_start);
+            e = exclusive_scan_i32(P.chunk_start, P.chunk_start, nl, scan_tmp, st);
         }
         int32_t nc = 0;
-        if (e == cudaSuccess) e = cudaMemcpyAsync(&nc, A->res_chunk_start + nl, 4, cudaMemcpyDeviceToHost, st);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(&nc, P.chunk_start + nl, 4, cudaMemcpyDeviceToHost, st);
         if (e == cudaSuccess) e = cudaStreamSynchronize(st);
         if (e == cudaSuccess) {
-            A->res_n_chunks = nc;
-            e = cudaMalloc(&A->res_chunk_row, 4 * (size_t)std::max(1, nc));
+            P.n_chunks = nc;
+            e = cudaMalloc(&P.chunk_row, 4 * (size_t)std::max(1, nc));
         }
-        if (e == cudaSuccess) e = cudaMalloc(&A->res_carry, 4 * (size_t)std::max(1, nc));
-        if (e == cudaSuccess) e = cudaMalloc(&A->res_done, 4 * (size_t)nl);
-        if (e == cudaSuccess) e = cudaMemsetAsync(A->res_done, 0, 4 * (size_t)nl, st);
+        if (e == cudaSuccess) e = cudaMalloc(&P.carry, 4 * (size_t)std::max(1, nc));
+        if (e == cudaSuccess) e = cudaMalloc(&P.done, 4 * (size_t)nl);
+        if (e == cudaSuccess) e = cudaMemsetAsync(P.done, 0, 4 * (size_t)nl, st);
         if (e == cudaSuccess) {
-            k_res_chunk_rows<<<(unsigned)((nl + 255) / 256), 256, 0, st>>>(nl, A->res_chunk_start, A->res_chunk_row);
+            k_res_chunk_rows<<<(unsigned)((nl + 255) / 256), 256, 0, st>>>(nl, P.chunk_start, P.chunk_row);
             e = cudaGetLastError();
         }
     }
@@ -435,7 +436,7 @@ spaden_status_t residual_long_rows(Matrix *A, cudaStream_t st) {
     if (e == cudaSuccess) e = cudaMalloc(&perm_pos, 4 * (size_t)std::max<int64_t>(1, m));
     for (int c = 0; c <= kResClasses && e == cudaSuccess; ++c) {
         bins.row_start[c] = total;
-        k_res_class_flag<<<g, 256, 0, st>>>(m, A->res_rowptr, c, flag);
+        k_res_class_flag<<<g, 256, 0, st>>>(m, P.rowptr, c, flag);
         e = exclusive_scan_i32(flag, flag, m, scan_tmp, st);
         int32_t cnt = 0;
         if (e == cudaSuccess) e = cudaMemcpyAsync(&cnt, flag + m, 4, cudaMemcpyDeviceToHost, st);
@@ -461,13 +462,127 @@ spaden_status_t residual_long_rows(Matrix *A, cudaStream_t st) {
         if (perm_pos) cudaFree(perm_pos);
         return cuda_status(e, "hybrid residual schedule");
     }
-    A->res_perm = perm_pos;
-    A->res_bins = bins;
-    A->res_aux_bytes = 4 * total + 4 * (2 * A->res_n_long + 1 + A->res_n_chunks) + 4 * A->res_n_chunks;
+    P.perm = perm_pos;
+    P.bins = bins;
+    A->res_aux_bytes += 4 * total + 4 * (2 * P.n_long + 1 + P.n_chunks) + 4 * P.n_chunks;
     return SPADEN_OK;
 }
 
+// Column segmentation of the residual (rows keep ascending columns): part s
+// holds columns [c_s, c_{s+1}).  One warp per row: lane s < S finds the row's
+// first entry with column >= c_s by binary search; counts per (part, row) ->
+// per-part scans -> the warp copies each part's slice of the row.
+__global__ void k_seg_count(int64_t m, int S, int64_t seg_cols, const int32_t *__restrict__ rp,
+                            const int32_t *__restrict__ col, int32_t *__restrict__ cnt /* [S][m+1] */) {
+    const int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (row >= m) return;
+    const int k0 = rp[row], k1 = rp[row + 1];
+    int lo = k1;  // lane s: first entry of part s
+    if (lane <= S) {
+        const int64_t c = (int64_t)lane * seg_cols;
+        int a = k0, b = k1;
+        while (a < b) {
+            const int mid = (a + b) >> 1;
+            if ((int64_t)col[mid] < c) a = mid + 1;
+            else b = mid;
+        }
+        lo = lane == S ? k1 : a;
+    }
+    const int hi = __shfl_down_sync(0xffffffffu, lo, 1);
+    if (lane < S) cnt[(int64_t)lane * (m + 1) + row] = hi - lo;
+}
+template <typename V>
+__global__ void k_seg_fill(int64_t m, int S, int64_t seg_cols, const int32_t *__restrict__ rp,
+                           const int32_t *__restrict__ col, const V *__restrict__ val,
+                           const int32_t *__restrict__ pos /* [S][m+1] scanned */, int32_t *const *dst_col,
+                           V *const *dst_val) {
+    const int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (row >= m) return;
+    const int k0 = rp[row];
+    for (int s = 0; s < S; ++s) {
+        const int o = pos[(int64_t)s * (m + 1) + row], n = pos[(int64_t)s * (m + 1) + row + 1] - o;
+        // this part's slice starts after the row's slices of parts < s
+        int skip = 0;
+        for (int q = 0; q < s; ++q) skip += pos[(int64_t)q * (m + 1) + row + 1] - pos[(int64_t)q * (m + 1) + row];
+        for (int j = lane; j < n; j += 32) {
+            dst_col[s][o + j] = col[k0 + skip + j];
+            dst_val[s][o + j] = val[k0 + skip + j];
+        }
+    }
+}
+
 }  // namespace
+
+// x larger than kXSegBytes: split the residual into S column parts (each a CSR
+// over all rows) so that every part's x gathers stay L2-resident; part q covers
+// columns [q*seg_cols, (q+1)*seg_cols).  Conversion-time only.
+static spaden_status_t segment_residual(Matrix *A, cudaStream_t st) {
+    const int64_t m = A->m, n = A->n;
+    int64_t seg_cols = kXSegBytes / 4;
+    if (const char *e = getenv("SPADEN_XSEG_COLS")) seg_cols = std::max<int64_t>(8, atoll(e));
+    const int S = (int)std::min<int64_t>(Matrix::kMaxResParts, (n + seg_cols - 1) / std::max<int64_t>(1, seg_cols));
+    if (S <= 1 || A->res_nnz == 0) return SPADEN_OK;
+    seg_cols = (n + S - 1) / S;  // balanced parts
+    const size_t sv = A->storage == SPADEN_R_16F ? 2 : 4;
+    ResPart full = A->res[0];
+    const size_t nt = scan_tmp_ints(m + 1);
+    int32_t *cnt = nullptr, *scan_tmp = nullptr;
+    int32_t **d_cols = nullptr;
+    void **d_vals = nullptr;
+    cudaError_t e = cudaMalloc(&cnt, 4 * (size_t)S * (m + 1));
+    if (e == cudaSuccess) e = cudaMalloc(&scan_tmp, 4 * (nt + 4));
+    if (e == cudaSuccess) e = cudaMalloc(&d_cols, sizeof(void *) * 2 * S);
+    d_vals = (void **)(d_cols + S);
+    const unsigned g = (unsigned)((32 * m + 255) / 256);
+    if (e == cudaSuccess) {
+        k_seg_count<<<g, 256, 0, st>>>(m, S, seg_cols, full.rowptr, full.colidx, cnt);
+        e = cudaGetLastError();
+    }
+    int32_t *h_cols[Matrix::kMaxResParts] = {};
+    void *h_vals[Matrix::kMaxResParts] = {};
+    for (int q = 0; q < S && e == cudaSuccess; ++q) {
+        ResPart &P = A->res[q];
+        P = ResPart{};
+        P.col0 = q * seg_cols;
+        P.col1 = std::min<int64_t>(n, (q + 1) * seg_cols);
+        int32_t *c = cnt + (size_t)q * (m + 1);
+        e = exclusive_scan_i32(c, c, m, scan_tmp, st);
+        int32_t tot = 0;
+        if (e == cudaSuccess) e = cudaMemcpyAsync(&tot, c + m, 4, cudaMemcpyDeviceToHost, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        P.nnz = tot;
+        if (e == cudaSuccess) e = cudaMalloc(&P.rowptr, pad16(4 * (m + 1)));
+        if (e == cudaSuccess) e = cudaMalloc(&P.colidx, pad16(4 * (size_t)tot));
+        if (e == cudaSuccess) e = cudaMalloc(&P.values, pad16(sv * (size_t)tot));
+        if (e == cudaSuccess) e = cudaMemcpyAsync(P.rowptr, c, 4 * (m + 1), cudaMemcpyDeviceToDevice, st);
+        h_cols[q] = P.colidx;
+        h_vals[q] = P.values;
+    }
+    A->n_res_parts = S;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(d_cols, h_cols, sizeof(void *) * S, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(d_vals, h_vals, sizeof(void *) * S, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) {
+        if (A->storage == SPADEN_R_16F)
+            k_seg_fill<__half><<<g, 256, 0, st>>>(m, S, seg_cols, full.rowptr, full.colidx,
+                                                  (const __half *)full.values, cnt, d_cols, (__half *const *)d_vals);
+        else
+            k_seg_fill<float><<<g, 256, 0, st>>>(m, S, seg_cols, full.rowptr, full.colidx,
+                                                 (const float *)full.values, cnt, d_cols, (float *const *)d_vals);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    cudaFree(full.rowptr);
+    cudaFree(full.colidx);
+    cudaFree(full.values);
+    if (cnt) cudaFree(cnt);
+    if (scan_tmp) cudaFree(scan_tmp);
+    if (d_cols) cudaFree(d_cols);
+    if (e != cudaSuccess) return cuda_status(e, "hybrid residual column segmentation");
+    A->res_aux_bytes += 4 * (int64_t)(S - 1) * (m + 1);  // rowptrs beyond the first
+    return SPADEN_OK;
+}
 
 spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
     A->res_max_popc = t;
@@ -504,7 +619,8 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
     if (e == cudaSuccess) e = cudaMalloc(&n_bmp, pad16(8 * nB));
     if (e == cudaSuccess) e = cudaMalloc(&n_off, pad16(4 * (nB + 1)));
     if (e == cudaSuccess) e = cudaMalloc(&n_vals, pad16(sv * nV));
-    if (e == cudaSuccess) e = cudaMalloc(&A->res_rowptr, pad16(4 * (m + 1)));
+    ResPart &P0 = A->res[0];
+    if (e == cudaSuccess) e = cudaMalloc(&P0.rowptr, pad16(4 * (m + 1)));
     if (e == cudaSuccess) e = cudaMalloc(&r_col, pad16(4 * res_nnz));
     if (e == cudaSuccess) e = cudaMalloc(&r_vals, pad16(sv * res_nnz));
     if (e != cudaSuccess) {
@@ -513,15 +629,15 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
         return fail(e, "hybrid split (allocation)");
     }
     cudaMemsetAsync(n_off, 0, pad16(4 * (nB + 1)), st);
-    e = cudaMemcpyAsync(A->res_rowptr, res_cnt, 4 * (m + 1), cudaMemcpyDeviceToDevice, st);
+    e = cudaMemcpyAsync(P0.rowptr, res_cnt, 4 * (m + 1), cudaMemcpyDeviceToDevice, st);
     if (A->storage == SPADEN_R_16F)
         k_split_fill<__half><<<grid, 256, 0, st>>>(m, Bnrow, t, A->blk_rowptr, A->blk_col, A->bitmap, A->blk_offset,
                                                    (const __half *)A->values, kept_blk, kept_val, n_col, n_bmp, n_off,
-                                                   (__half *)n_vals, A->res_rowptr, r_col, (__half *)r_vals);
+                                                   (__half *)n_vals, P0.rowptr, r_col, (__half *)r_vals);
     else
         k_split_fill<float><<<grid, 256, 0, st>>>(m, Bnrow, t, A->blk_rowptr, A->blk_col, A->bitmap, A->blk_offset,
                                                   (const float *)A->values, kept_blk, kept_val, n_col, n_bmp, n_off,
-                                                  (float *)n_vals, A->res_rowptr, r_col, (float *)r_vals);
+                                                  (float *)n_vals, P0.rowptr, r_col, (float *)r_vals);
     if (e == cudaSuccess) e = cudaMemcpyAsync(A->blk_rowptr, kept_blk, 4 * (Bnrow + 1), cudaMemcpyDeviceToDevice, st);
     if (e == cudaSuccess) e = cudaGetLastError();
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
@@ -535,12 +651,18 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
     A->bitmap = n_bmp;
     A->blk_offset = n_off;
     A->values = n_vals;
-    A->res_colidx = r_col;
-    A->res_values = r_vals;
+    P0.colidx = r_col;
+    P0.values = r_vals;
+    P0.col0 = 0;
+    P0.col1 = A->n;
+    P0.nnz = res_nnz;
+    A->n_res_parts = 1;
     A->Bnnz = nB;
     A->res_nnz = res_nnz;
     if (e != cudaSuccess) return cuda_status(e, "hybrid split (fill)");
-    return residual_long_rows(A, st);
+    spaden_status_t ss = segment_residual(A, st);
+    for (int q = 0; q < A->n_res_parts && ss == SPADEN_OK; ++q) ss = residual_schedule(A, A->res[q], st);
+    return ss;
 }
 
 namespace {
@@ -550,62 +672,75 @@ __global__ void k_scale(int64_t m, float beta, float *__restrict__ y) {
 }
 }  // namespace
 
-// Hybrid SpMV, first part: y = beta*y + alpha*A_res*x on every row.  The binned
-// kernel (a normal launch: it follows whatever produced x) applies beta itself
-// -- rows of the last class only get y = beta*y -- so y is fetched before the
-// gathers; long residual rows then accumulate their chunks (PDL launches).
+// Hybrid SpMV, first part: y = beta*y + alpha*A_res*x on every row.  Per
+// residual part (column segment) the binned kernel (a normal launch: it follows
+// whatever produced x, or the previous part) applies beta itself -- part 0 with
+// the caller's beta, later parts with 1 -- rows of the last class only get
+// y = beta*y, so y is fetched before the gathers; long residual rows then
+// accumulate their chunks (PDL launches).  Per row the parts are added in
+// column order (a function of the row and of n: partition invariant).
 // SPADEN_RES=fixed: beta pass (memset / scale) + the 16-lane kernel (ablation).
-cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st) {
-    if (A.m == 0) return cudaSuccess;
-    const char *env = getenv("SPADEN_RES");  // read per call
-    const bool binned = A.res_perm && !(env && env[0] == 'f');
+static cudaError_t residual_part(const Matrix &A, const ResPart &P, bool binned, float alpha, const float *x,
+                                 float beta, float *y, cudaStream_t st) {
     cudaError_t e = cudaSuccess;
     if (binned) {
-        const int64_t nc = A.res_bins.cta_start[kResClasses + 1];
+        const int64_t nc = P.bins.cta_start[kResClasses + 1];
         if (nc > 0) {
             if (A.storage == SPADEN_R_16F)
-                e = launch_k(false, k_residual_binned<__half>, dim3((unsigned)nc), dim3(256), 0, st, A.res_bins,
-                             (const int32_t *)A.res_perm, (const int32_t *)A.res_rowptr,
-                             (const int32_t *)A.res_colidx, (const __half *)A.res_values, x, alpha, beta, y);
+                e = launch_k(false, k_residual_binned<__half>, dim3((unsigned)nc), dim3(256), 0, st, P.bins,
+                             (const int32_t *)P.perm, (const int32_t *)P.rowptr, (const int32_t *)P.colidx,
+                             (const __half *)P.values, x, alpha, beta, y);
             else
-                e = launch_k(false, k_residual_binned<float>, dim3((unsigned)nc), dim3(256), 0, st, A.res_bins,
-                             (const int32_t *)A.res_perm, (const int32_t *)A.res_rowptr,
-                             (const int32_t *)A.res_colidx, (const float *)A.res_values, x, alpha, beta, y);
+                e = launch_k(false, k_residual_binned<float>, dim3((unsigned)nc), dim3(256), 0, st, P.bins,
+                             (const int32_t *)P.perm, (const int32_t *)P.rowptr, (const int32_t *)P.colidx,
+                             (const float *)P.values, x, alpha, beta, y);
         }
     } else {
         if (beta == 0.f) e = cudaMemsetAsync(y, 0, sizeof(float) * (size_t)A.m, st);
         else if (beta != 1.f)
             k_scale<<<(unsigned)std::min<int64_t>((A.m + 255) / 256, 148 * 16), 256, 0, st>>>(A.m, beta, y);
         const unsigned grid = (unsigned)((kResLanes * A.m + 255) / 256);  // one lane group per row
-        if (e == cudaSuccess && A.res_nnz > 0) {
+        if (e == cudaSuccess && P.nnz > 0) {
             if (A.storage == SPADEN_R_16F)
-                k_residual<__half, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
-                                                                    (const __half *)A.res_values, x, alpha, y);
+                k_residual<__half, kResLanes><<<grid, 256, 0, st>>>(A.m, P.rowptr, P.colidx,
+                                                                    (const __half *)P.values, x, alpha, y);
             else
-                k_residual<float, kResLanes><<<grid, 256, 0, st>>>(A.m, A.res_rowptr, A.res_colidx,
-                                                                   (const float *)A.res_values, x, alpha, y);
+                k_residual<float, kResLanes><<<grid, 256, 0, st>>>(A.m, P.rowptr, P.colidx,
+                                                                   (const float *)P.values, x, alpha, y);
         }
     }
-    if (e == cudaSuccess && A.res_n_long > 0) {
-        const unsigned gc = (unsigned)((32 * A.res_n_chunks + 255) / 256);
-        const bool fused = A.res_n_chunks <= fused_fixup_max();
+    if (e == cudaSuccess && P.n_long > 0) {
+        const unsigned gc = (unsigned)((32 * P.n_chunks + 255) / 256);
+        const bool fused = P.n_chunks <= fused_fixup_max();
         if (A.storage == SPADEN_R_16F)
             e = launch_k(true, fused ? k_res_chunks<__half, true> : k_res_chunks<__half, false>, dim3(gc), dim3(256),
-                         0, st, (int64_t)A.res_n_chunks, (const int32_t *)A.res_long_rows,
-                         (const int32_t *)A.res_chunk_start, (const int32_t *)A.res_chunk_row,
-                         (const int32_t *)A.res_rowptr, (const int32_t *)A.res_colidx, (const __half *)A.res_values,
-                         x, A.res_carry, A.res_done, alpha, y);
+                         0, st, (int64_t)P.n_chunks, (const int32_t *)P.long_rows, (const int32_t *)P.chunk_start,
+                         (const int32_t *)P.chunk_row, (const int32_t *)P.rowptr, (const int32_t *)P.colidx,
+                         (const __half *)P.values, x, P.carry, P.done, alpha, y);
         else
             e = launch_k(true, fused ? k_res_chunks<float, true> : k_res_chunks<float, false>, dim3(gc), dim3(256),
-                         0, st, (int64_t)A.res_n_chunks, (const int32_t *)A.res_long_rows,
-                         (const int32_t *)A.res_chunk_start, (const int32_t *)A.res_chunk_row,
-                         (const int32_t *)A.res_rowptr, (const int32_t *)A.res_colidx, (const float *)A.res_values,
-                         x, A.res_carry, A.res_done, alpha, y);
+                         0, st, (int64_t)P.n_chunks, (const int32_t *)P.long_rows, (const int32_t *)P.chunk_start,
+                         (const int32_t *)P.chunk_row, (const int32_t *)P.rowptr, (const int32_t *)P.colidx,
+                         (const float *)P.values, x, P.carry, P.done, alpha, y);
         if (e == cudaSuccess && !fused)
-            e = launch_k(true, k_res_fixup, dim3((unsigned)((32 * A.res_n_long + 255) / 256)), dim3(256), 0, st,
-                         (int64_t)A.res_n_long, (const int32_t *)A.res_long_rows, (const int32_t *)A.res_chunk_start,
-                         (const float *)A.res_carry, alpha, y);
+            e = launch_k(true, k_res_fixup, dim3((unsigned)((32 * P.n_long + 255) / 256)), dim3(256), 0, st,
+                         (int64_t)P.n_long, (const int32_t *)P.long_rows, (const int32_t *)P.chunk_start,
+                         (const float *)P.carry, alpha, y);
     }
+    return e;
+}
+
+bool residual_binned_enabled(const Matrix &A) {
+    const char *env = getenv("SPADEN_RES");  // "fixed": the 16-lane kernel (ablation), read per call
+    return A.n_res_parts > 0 && A.res[0].perm && !(env && env[0] == 'f');
+}
+
+cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st) {
+    if (A.m == 0 || A.n_res_parts == 0) return cudaSuccess;
+    const bool binned = residual_binned_enabled(A);
+    cudaError_t e = cudaSuccess;
+    for (int q = 0; q < A.n_res_parts && e == cudaSuccess; ++q)
+        e = residual_part(A, A.res[q], binned, alpha, x, q == 0 ? beta : 1.f, y, st);
     if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }

@@ -46,24 +46,33 @@ struct spaden_matrix_s {
     int64_t spmm_ntiles[3] = {};
     int spmm_state[3] = {};                    // 0 not built, 1 built, -1 unsupported
 
-    // hybrid residual CSR (csrc/hybrid.cu), empty in pure bitBSR mode
+    // hybrid residual (csrc/hybrid.cu), empty in pure bitBSR mode: a CSR with
+    // global columns, split into column segments (parts) when x is larger than
+    // kXSegBytes so that each part's x gathers stay L2-resident
     int64_t res_nnz = 0;
     int res_max_popc = 0;
-    int32_t *res_rowptr = nullptr;   // [m+1]
-    int32_t *res_colidx = nullptr;   // [res_nnz]
-    void *res_values = nullptr;      // [res_nnz]
-    int64_t res_n_long = 0;          // residual rows longer than kResLongRow (chunked)
-    int64_t res_n_chunks = 0;
-    int32_t *res_long_rows = nullptr;    // [res_n_long]
-    int32_t *res_chunk_start = nullptr;  // [res_n_long+1]
-    int32_t *res_chunk_row = nullptr;    // [res_n_chunks] index into res_long_rows
-    float *res_carry = nullptr;          // [res_n_chunks]
-    int32_t *res_done = nullptr;         // [res_n_long] chunks finished per long row (0 between calls)
-    int32_t *res_perm = nullptr;         // all rows, grouped by length class (then empty / long rows)
     struct ResBins {                     // class c: perm[row_start[c], row_start[c+1]), CTAs from cta_start[c]
         int64_t row_start[8], cta_start[8];  // classes 0..kResClasses (the last: empty / long rows)
-    } res_bins = {};
-    int64_t res_aux_bytes = 0;           // perm + long-row chunk lists
+    };
+    struct ResPart {
+        int64_t col0 = 0, col1 = 0, nnz = 0;  // columns [col0, col1) of the residual
+        int32_t *rowptr = nullptr;           // [m+1]
+        int32_t *colidx = nullptr;           // [nnz]
+        void *values = nullptr;              // [nnz]
+        int64_t n_long = 0;                  // rows longer than kResLongRow (chunked)
+        int64_t n_chunks = 0;
+        int32_t *long_rows = nullptr;        // [n_long]
+        int32_t *chunk_start = nullptr;      // [n_long+1]
+        int32_t *chunk_row = nullptr;        // [n_chunks] index into long_rows
+        float *carry = nullptr;              // [n_chunks]
+        int32_t *done = nullptr;             // [n_long] chunks finished per long row (0 between calls)
+        int32_t *perm = nullptr;             // all rows, grouped by length class (then empty / long rows)
+        ResBins bins = {};
+    };
+    static constexpr int kMaxResParts = 16;
+    ResPart res[kMaxResParts];
+    int n_res_parts = 0;
+    int64_t res_aux_bytes = 0;           // perms, long-row chunk lists, per-part rowptrs beyond the first
 
     // host-API staging buffers (lazily allocated): [2] slots for the batched pipeline
     float *stage_x = nullptr;          // spaden_spmv_host
@@ -166,6 +175,10 @@ constexpr int kResChunk = SPADEN_RES_CHUNK;
 #endif
 constexpr int kResLanes = SPADEN_RES_LANES;
 constexpr int kResLongRow = 4096;
+// x bytes per residual column segment (part): a part's x slice plus the stream
+// must stay in the 126 MB L2; larger x is split (SPADEN_XSEG_COLS overrides the
+// columns per part, tests)
+constexpr int64_t kXSegBytes = 32ll << 20;
 // length classes of the binned residual pass: class c (L = 2^c lanes per row)
 // holds rows of len entries with 4*2^(c-1) < len <= 4*2^c; the last class takes
 // everything up to kResLongRow
@@ -182,6 +195,7 @@ constexpr int kDenseDecode = 1;
 
 using TileDesc = ::spaden_tile_desc_s;
 using ResBins = ::spaden_matrix_s::ResBins;
+using ResPart = ::spaden_matrix_s::ResPart;
 
 spaden_status_t build_schedule(Matrix *A, cudaStream_t stream);
 spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t stream);
@@ -208,6 +222,7 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t stream);
 // hybrid SpMV, first part: y = beta*y + alpha*A_res*x on every row (y not read
 // when beta = 0); the bitBSR kernels follow with beta = 1
 cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t stream);
+bool residual_binned_enabled(const Matrix &A);  // binned residual kernel (not the SPADEN_RES=fixed ablation)
 
 // SpMV (spmv.cu)
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,

@@ -1313,10 +1313,14 @@ int spmv_launch_count(const Matrix &A, float beta) {
     if (A.m == 0) return 0;
     int n = 0;
     if (A.res_max_popc > 0) {  // residual_first
-        const char *env = getenv("SPADEN_RES");
-        if (A.res_perm && !(env && env[0] == 'f')) n += A.res_bins.cta_start[kResClasses + 1] > 0 ? 1 : 0;
-        else n += (beta != 1.f ? 1 : 0) + (A.res_nnz > 0 ? 1 : 0);
-        if (A.res_n_long > 0) n += 1 + (A.res_n_chunks > fused_fixup_max() ? 1 : 0);
+        const bool binned = residual_binned_enabled(A);
+        for (int q = 0; q < A.n_res_parts; ++q) {
+            const ResPart &P = A.res[q];
+            const float b = q == 0 ? beta : 1.f;
+            if (binned) n += P.bins.cta_start[kResClasses + 1] > 0 ? 1 : 0;
+            else n += (b != 1.f ? 1 : 0) + (P.nnz > 0 ? 1 : 0);
+            if (P.n_long > 0) n += 1 + (P.n_chunks > fused_fixup_max() ? 1 : 0);
+        }
     }
     if (kernel_variant() == 0) return n + 1;
     n += A.n_tiles > 0 ? 1 : 0;

@@ -376,6 +376,43 @@ def test_cuda_graph_capture_chain(sp, torch, t):
         assert torch.equal(y, ref)
 
 
+@pytest.mark.parametrize("storage", ["fp32", "fp16"])
+@pytest.mark.parametrize("fixup", ["fused", "separate"])
+@pytest.mark.parametrize("seg_cols", [3000, 20_011 // 2 + 1, 64])
+def test_residual_column_parts(sp, torch, storage, fixup, seg_cols, monkeypatch):
+    """Residual split into column parts (as for x > 32 MB; forced here with
+    SPADEN_XSEG_COLS): every part's rows binned, parts added in column order.
+    Within tolerance of the oracle, deterministic, 8-row-partition invariant,
+    alpha/beta, launch count = CUDA-graph nodes."""
+    monkeypatch.setenv("SPADEN_XSEG_COLS", str(seg_cols))
+    if fixup == "separate":
+        monkeypatch.setenv("SPADEN_FUSED_FIXUP_MAX", "0")
+    A = binned_rows_matrix(seed=13)
+    stored = A.values if storage == "fp32" else oracle.f32_to_f16(A.values)
+    x = W.vector(A.n, 43)
+    rp, ci, v = dev(torch, A)
+    M = sp.convert(rp, ci, v, A.n, storage=storage, residual_max_popc=64)
+    assert M.info.residual_nnz == A.nnz and M.info.Bnnz == 0
+    assert "res_rowptr" not in M.arrays()  # split into parts
+    y = gpu_spmv(torch, M, x)
+    assert np.array_equal(y, gpu_spmv(torch, M, x))
+    check_spmv(A, y, stored, x)
+    y0 = W.vector(A.m, 44)
+    ys, s = oracle.spmv(A.rowptr, A.colidx, stored, x)
+    y2 = gpu_spmv(torch, M, x, alpha=0.5, beta=-1.5, y0=y0)
+    assert oracle.componentwise_error(y2, 0.5 * ys - 1.5 * y0, 0.5 * s + 1.5 * np.abs(y0)) <= TOL32
+    cut = (A.m // 16) * 8
+    parts = []
+    for r0, r1 in ((0, cut), (cut, A.m)):
+        S = A.row_slice(r0, r1)
+        r, c, vv = dev(torch, S)
+        parts.append(gpu_spmv(torch, sp.convert(r, c, vv, S.n, storage=storage, residual_max_popc=64), x))
+    assert np.array_equal(np.concatenate(parts), y)
+    xd = torch.from_numpy(x).cuda()
+    yd = torch.from_numpy(y0).cuda()
+    assert graph_nodes(torch, lambda st: M.spmv(xd, yd, alpha=1.0, beta=0.5, stream=st)) == M.launch_count(0.5)
+
+
 def graph_nodes(torch, fn):
     """Number of nodes (kernel launches, memsets) fn() puts on a captured stream."""
     rt = pytest.importorskip("cuda.bindings.runtime")
