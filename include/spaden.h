@@ -90,7 +90,7 @@ typedef struct {                /* borrowed device views; valid until spaden_fre
     const int32_t  *blk_offset; /* [Bnnz+1]  */
     const void     *values;     /* [nnz - residual_nnz] of storage_dtype */
     const int32_t  *res_rowptr; /* [m+1] hybrid residual CSR (NULL when residual_nnz == 0, or when
-                                   the residual is split into column parts because 4n > 32 MB) */
+                                   the residual is split into column parts because 4n > 64 MB) */
     const int32_t  *res_colidx; /* [residual_nnz] */
     const void     *res_values; /* [residual_nnz] of storage_dtype */
 } spaden_arrays_t;

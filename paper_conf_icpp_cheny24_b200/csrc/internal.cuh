@@ -178,7 +178,7 @@ constexpr int kResLongRow = 4096;
 // x bytes per residual column segment (part): a part's x slice plus the stream
 // must stay in the 126 MB L2; larger x is split (SPADEN_XSEG_COLS overrides the
 // columns per part, tests)
-constexpr int64_t kXSegBytes = 32ll << 20;
+constexpr int64_t kXSegBytes = 64ll << 20;
 // length classes of the binned residual pass: class c (L = 2^c lanes per row)
 // holds rows of len entries with 4*2^(c-1) < len <= 4*2^c; the last class takes
 // everything up to kResLongRow
