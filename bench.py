@@ -53,7 +53,8 @@ def parse():
     p.add_argument("--no-variants", action="store_true", help="skip the other-precision kernel timing")
     p.add_argument("--spmm", default="4", help="comma list of right-hand-side counts for the SpMM extra ('' = skip)")
     p.add_argument("--hybrid", type=int, default=0,
-                   help="hybrid format: blocks with <= HYBRID entries go to a CSR residual (0 = pure bitBSR)")
+                   help="hybrid format: blocks with <= HYBRID entries go to a CSR residual (0 = pure bitBSR, "
+                        "-1 = automatic by mean block fill)")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     p.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
                    help="x rebuild for N>1: NCCL all-gather after the SpMV, or peer stores fused into the "
@@ -475,7 +476,7 @@ def main():
             "config": {"workload": args.workload, "m": wl.m, "n": wl.n, "nnz": wl.nnz,
                        "Bnrow": int((wl.m + 7) // 8), "Bnnz_rank0": int(info.Bnnz),
                        "fill_rank0": wl.local_nnz / max(1, info.Bnnz),
-                       "values": args.dtype, "hybrid_residual_max_popc": args.hybrid,
+                       "values": args.dtype, "hybrid_residual_max_popc": int(info.residual_max_popc), "residual_parts": int(info.residual_parts),
                        "residual_nnz_rank0": int(info.residual_nnz),
                        "parallelism": f"row-partition x{world}" + (
                            (" + NCCL all-gather" if args.exchange == "nccl" else " + fused peer-store all-gather")

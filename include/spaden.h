@@ -81,6 +81,9 @@ typedef struct {
     int64_t n_long;             /* block-rows too large for a tile (processed in chunks)  */
     int64_t residual_nnz;       /* entries held in the CSR residual (hybrid mode, else 0);
                                    format_bytes then also counts 4(m+1) + (4+s_v)*residual_nnz */
+    int32_t residual_max_popc;  /* hybrid threshold t in effect (0 = pure bitBSR; the value the
+                                   automatic choice took when opts asked for -1)              */
+    int32_t residual_parts;     /* column parts of the residual (x > 64 MB), 0 when pure      */
 } spaden_info_t;
 
 typedef struct {                /* borrowed device views; valid until spaden_free         */
@@ -100,7 +103,9 @@ typedef struct {
     int32_t struct_size;        /* sizeof(spaden_convert_opts_t)                          */
     int32_t residual_max_popc;  /* hybrid format: blocks holding at
                                    most this many entries are stored as a CSR residual
-                                   instead of bitBSR blocks (0 = pure bitBSR, max 64)     */
+                                   instead of bitBSR blocks (0 = pure bitBSR, max 64;
+                                   -1 = automatic: 4 when the mean block fill nnz/Bnnz
+                                   is below 8, else 0)                                     */
     int32_t reserved[6];
 } spaden_convert_opts_t;
 

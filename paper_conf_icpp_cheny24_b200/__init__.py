@@ -6,7 +6,7 @@ There is no CPU fallback: importing this package on a machine without the
 built library raises ImportError, and every call on a missing device fails.
 
 Raw entry points keep the C names (spaden_convert_csr_to_bitmap, spaden_spmv,
-spaden_spmv_host, spaden_free, spaden_get_info, spaden_get_arrays,
+spaden_spmv_host, spaden_free, spaden_get_info, spaden_get_arrays, spaden_spmv_launch_count,
 spaden_status_string, spaden_last_error_message, spaden_version); `convert`
 and `Matrix` wrap them for torch tensors.
 """
@@ -40,7 +40,8 @@ class spaden_info_t(ctypes.Structure):
                 ("Bnrow", ctypes.c_int64), ("Bnnz", ctypes.c_int64),
                 ("storage_dtype", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("format_bytes", ctypes.c_int64), ("aux_bytes", ctypes.c_int64),
-                ("n_tiles", ctypes.c_int64), ("n_long", ctypes.c_int64), ("residual_nnz", ctypes.c_int64)]
+                ("n_tiles", ctypes.c_int64), ("n_long", ctypes.c_int64), ("residual_nnz", ctypes.c_int64),
+                ("residual_max_popc", ctypes.c_int32), ("residual_parts", ctypes.c_int32)]
 
 
 class spaden_arrays_t(ctypes.Structure):
@@ -283,7 +284,8 @@ class Matrix:
 
 def convert(rowptr, colidx, values, n: int, storage=None, stream=None, residual_max_popc: int = 0) -> Matrix:
     """CSR (int32 CUDA tensors + fp32/fp16 values) -> bitBSR Matrix (hybrid with a CSR
-    residual for blocks of <= residual_max_popc entries when that is > 0)."""
+    residual for blocks of <= residual_max_popc entries when that is > 0; -1 = automatic:
+    4 when the mean block fill is below 8, else pure bitBSR)."""
     torch = _torch()
     assert rowptr.dtype == torch.int32 and colidx.dtype == torch.int32
     assert rowptr.is_cuda and colidx.is_cuda and values.is_cuda

@@ -115,10 +115,10 @@ spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n, int64_t nn
     g_last_error.clear();
     int res_t = 0;
     if (opts) {
-        if (opts->struct_size != (int32_t)sizeof(spaden_convert_opts_t) || opts->residual_max_popc < 0 ||
+        if (opts->struct_size != (int32_t)sizeof(spaden_convert_opts_t) || opts->residual_max_popc < -1 ||
             opts->residual_max_popc > 64) {
             if (out) *out = nullptr;
-            set_error("bad spaden_convert_opts_t (struct_size or residual_max_popc not in [0, 64])");
+            set_error("bad spaden_convert_opts_t (struct_size or residual_max_popc not in [-1, 64])");
             return SPADEN_ERR_INVALID_ARGUMENT;
         }
         res_t = opts->residual_max_popc;
@@ -332,6 +332,8 @@ spaden_status_t spaden_get_info(spaden_matrix_t A, spaden_info_t *info) {
                          sv * (A->nnz - A->res_nnz);
     if (A->res_max_popc > 0) info->format_bytes += 4 * (A->m + 1) + (4 + sv) * A->res_nnz;
     info->residual_nnz = A->res_nnz;
+    info->residual_max_popc = A->res_max_popc;
+    info->residual_parts = A->n_res_parts;
     info->aux_bytes = A->aux_bytes + A->res_aux_bytes;
     info->n_tiles = A->n_tiles;
     info->n_long = A->n_long;

@@ -402,7 +402,12 @@ spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *ro
     k_finalize<<<grid_for(Bnrow + 1, 256), 256, 0, st>>>(Bnrow, Bnnz, nnz, chunk_start, cnt_blk,
                                                          A->blk_rowptr, A->blk_offset);
     SPADEN_CUDA_TRY(cudaGetLastError());
-    // hybrid mode: move low-fill blocks into the CSR residual (one more sync)
+    // hybrid mode: move low-fill blocks into the CSR residual (one more sync);
+    // -1 = automatic: t = kAutoResidualPopc when the mean block fill is below
+    // kSlotsMinFill (the low-degree regime of P:L236, where the measured best t
+    // on powerlaw1m / rmat22 / rmat25 is 3-4), else pure bitBSR
+    if (residual_max_popc < 0)
+        residual_max_popc = (Bnnz > 0 && nnz < (int64_t)kSlotsMinFill * Bnnz) ? kAutoResidualPopc : 0;
     if (residual_max_popc > 0) {
         spaden_status_t hs = split_residual(A, residual_max_popc, st);
         if (hs != SPADEN_OK) return hs;

@@ -190,6 +190,8 @@ __host__ __device__ inline int res_class(int len) {
 }
 // mean nonzeros per block from which the predicated-slot decode is used
 constexpr int kSlotsMinFill = 8;
+// hybrid threshold of the automatic choice (residual_max_popc = -1)
+constexpr int kAutoResidualPopc = 4;
 // decode used above that fill (1 = lane per block, 2 = lane per block row)
 constexpr int kDenseDecode = 1;
 

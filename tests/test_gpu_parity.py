@@ -413,6 +413,25 @@ def test_residual_column_parts(sp, torch, storage, fixup, seg_cols, monkeypatch)
     assert graph_nodes(torch, lambda st: M.spmv(xd, yd, alpha=1.0, beta=0.5, stream=st)) == M.launch_count(0.5)
 
 
+def test_hybrid_auto_threshold(sp, torch):
+    """residual_max_popc = -1: hybrid (t = 4) for low mean block fill, pure bitBSR
+    for FEM-like blocks; the choice is reported in spaden_info_t; results within
+    tolerance; values outside [-1, 64] are rejected."""
+    for A, want in ((W.powerlaw(13, 6, seed=1), 4), (W.fem(6, 7, 8, seed=2), 0)):
+        rp, ci, v = dev(torch, A)
+        M = sp.convert(rp, ci, v, A.n, residual_max_popc=-1)
+        assert M.info.residual_max_popc == want
+        assert (M.info.residual_nnz > 0) == (want > 0)
+        assert M.info.residual_parts == (1 if want else 0)
+        x = W.vector(A.n, 45)
+        check_spmv(A, gpu_spmv(torch, M, x), A.values, x)
+    A = W.tiny(0)
+    rp, ci, v = dev(torch, A)
+    for bad in (-2, 65):
+        with pytest.raises(sp.SpadenError):
+            sp.convert(rp, ci, v, A.n, residual_max_popc=bad)
+
+
 def graph_nodes(torch, fn):
     """Number of nodes (kernel launches, memsets) fn() puts on a captured stream."""
     rt = pytest.importorskip("cuda.bindings.runtime")
