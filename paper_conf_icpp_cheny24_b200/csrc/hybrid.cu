@@ -5,14 +5,17 @@
 // burdensome, e.g., if one block only contains a single nonzero element."  In
 // hybrid mode the converted bitBSR is split: blocks holding at most t entries
 // become a row-sorted CSR residual (global columns), the rest stay bitBSR.
-// spaden_spmv then runs the bitBSR kernels (y = alpha*A_bit*x + beta*y) followed
-// by a residual pass (y += alpha*A_res*x; rows binned by length, 2^c lanes per
-// row of class c, fixed per-lane order and xor tree: deterministic and
-// independent of the row partition).
+// spaden_spmv then runs the residual pass first (y = beta*y + alpha*A_res*x;
+// rows binned by length, 2^c lanes per row of class c, fixed per-lane order and
+// xor tree: deterministic and independent of the row partition), followed by
+// the bitBSR kernels accumulating with beta = 1 (programmatic dependent launch
+// along the chain).
 //
 // Split = count kernel (per block-row: kept blocks / values, residual entries
 // per row) -> exclusive scans -> one host sync (sizes) -> fill kernel (compacts
-// the kept blocks, appends residual entries row by row in ascending column).
+// the kept blocks, appends residual entries row by row in ascending column) ->
+// column parts when x > kXSegBytes (segment_residual) -> per part: long-row
+// chunk lists and the length-class row permutation (residual_schedule).
 #include <algorithm>
 #include <cstdlib>
 
