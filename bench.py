@@ -52,7 +52,7 @@ def parse():
     p.add_argument("--no-cusparse", action="store_true")
     p.add_argument("--no-variants", action="store_true", help="skip the other-precision kernel timing")
     p.add_argument("--spmm", default="4", help="comma list of right-hand-side counts for the SpMM extra ('' = skip)")
-    p.add_argument("--hybrid", type=int, default=0,
+    p.add_argument("--hybrid", type=int, default=-1,
                    help="hybrid format: blocks with <= HYBRID entries go to a CSR residual (0 = pure bitBSR, "
                         "-1 = automatic by mean block fill)")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -297,8 +297,8 @@ def main():
                 ev_pair[0][1].record(stream)
 
     if args.exchange == "fused":
-        if args.hybrid:
-            raise SystemExit("--exchange fused needs pure bitBSR (no --hybrid)")
+        if info.residual_max_popc > 0:
+            raise SystemExit("--exchange fused needs pure bitBSR (--hybrid 0)")
         it = FusedIteratedSpMV(wl.part, wl.n, _Timed(), wl.x0, rank)
     else:
         it = IteratedSpMV(wl.part, wl.n, local_spmv, wl.x0, rank)
