@@ -492,7 +492,8 @@ def main():
                          "frac": achieved / peak, "traffic": traffic, "frac_of_8tbps_spec": achieved / 8000.0,
                          "peak_kind": f"{peak_kind} copy bandwidth (MEASURED_PEAKS.json hbm_gbs)",
                          "kernel": "spaden_spmv (k_spmv_tiled [+ long-row chunks/fix-up])",
-                         "kernel_ms": kavg_ms, "alg_bytes_per_launch": abytes},
+                         "kernel_ms": kavg_ms, "alg_bytes_per_launch": abytes,
+                         "kernel_ms_p10_p50_p90": [float(np.percentile(kernel_ms, q)) for q in (10, 50, 90)]},
             "convert": {"seconds": convert_s, "ns_per_nnz": convert_s * 1e9 / max(1, wl.local_nnz)},
             "cusparse_csr": cus,
             "variants": variants,
