@@ -687,7 +687,8 @@ static cudaError_t residual_part(const Matrix &A, const ResPart &P, bool binned,
                                  float beta, float *y, cudaStream_t st) {
     cudaError_t e = cudaSuccess;
     if (binned) {
-        const int64_t nc = P.bins.cta_start[kResClasses + 1];
+        // the last class (empty / long rows) only scales y: skipped when beta = 1
+        const int64_t nc = P.bins.cta_start[beta == 1.f ? kResClasses : kResClasses + 1];
         if (nc > 0) {
             if (A.storage == SPADEN_R_16F)
                 e = launch_k(false, k_residual_binned<__half>, dim3((unsigned)nc), dim3(256), 0, st, P.bins,

@@ -1317,7 +1317,7 @@ int spmv_launch_count(const Matrix &A, float beta) {
         for (int q = 0; q < A.n_res_parts; ++q) {
             const ResPart &P = A.res[q];
             const float b = q == 0 ? beta : 1.f;
-            if (binned) n += P.bins.cta_start[kResClasses + 1] > 0 ? 1 : 0;
+            if (binned) n += P.bins.cta_start[b == 1.f ? kResClasses : kResClasses + 1] > 0 ? 1 : 0;
             else n += (b != 1.f ? 1 : 0) + (P.nnz > 0 ? 1 : 0);
             if (P.n_long > 0) n += 1 + (P.n_chunks > fused_fixup_max() ? 1 : 0);
         }
