@@ -523,6 +523,36 @@ def test_fem1p5m_full(sp, torch):
         M.free()
 
 
+def test_rmat25_full_hybrid_sampled(sp, torch):
+    """BASELINE configs[4] (R-MAT scale 25, edge factor 32, 1.05B nnz, PageRank
+    values) at full size on one GPU, converted as bench.py does (automatic
+    hybrid: t = 4, residual split into 2 column parts because x is 134 MB): y on
+    4096 sampled rows (incl. the longest ones) against the fp64 oracle on those rows."""
+    rp, ci, v, n, nnz = W.pagerank_slice_torch(25, 32, 0, 1 << 25, seed=0, device="cuda")
+    M = sp.convert(rp, ci, v, n, residual_max_popc=-1)
+    torch.cuda.synchronize()
+    i = M.info
+    assert i.nnz == nnz and i.residual_max_popc == 4 and i.residual_parts == 2
+    g = torch.Generator(device="cuda")
+    g.manual_seed(7)
+    x = torch.rand(n, generator=g, device="cuda")
+    y = M.spmv(x)
+    torch.cuda.synchronize()
+    rph = rp.cpu().numpy().astype(np.int64)
+    lens = np.diff(rph)
+    rng = np.random.default_rng(3)
+    rows = np.unique(np.concatenate([rng.choice(n, 4064, replace=False), np.argsort(lens)[-32:]]))
+    sub_rp = np.zeros(rows.size + 1, np.int64)
+    sub_rp[1:] = np.cumsum(lens[rows])
+    idx = torch.from_numpy(np.concatenate([np.arange(rph[r], rph[r + 1]) for r in rows])).cuda()
+    cols = ci[idx].cpu().numpy()
+    vals = v[idx].cpu().numpy()
+    ys, s = oracle.spmv(sub_rp, cols, vals, x.cpu().numpy())
+    err = oracle.componentwise_error(y[torch.from_numpy(rows).cuda()].cpu().numpy(), ys, s)
+    assert err <= TOL32, err
+    M.free()
+
+
 def test_tile_row_cap_empty_block_rows(sp, torch):
     """Long runs of empty block-rows (more than the 128 block-rows a tile may
     hold) between a few populated ones: y is exact (small integers) and rows
