@@ -40,6 +40,10 @@ for fixup in ("8192", "0"):  # long-row fix-up fused into the chunk kernel / sep
     run(binned_rows_matrix(), "fp32", t=64)
     run(hub_matrix(m=40, n=70_001, hub_rows=(3, 30), hub_nnz=40_000), "fp32")
 os.environ.pop("SPADEN_FUSED_FIXUP_MAX")
+os.environ["SPADEN_XSEG_COLS"] = "3000"  # residual column parts (normally x > 64 MB)
+run(binned_rows_matrix(), "fp32", t=64)
+run(binned_rows_matrix(), "fp16", t=-1)
+os.environ.pop("SPADEN_XSEG_COLS")
 B = hub_matrix()
 MB = sp.convert(torch.from_numpy(B.rowptr).cuda(), torch.from_numpy(B.colidx).cuda(),
                 torch.from_numpy(B.values).cuda(), B.n, residual_max_popc=2)
