@@ -219,7 +219,8 @@ SPADEN_API spaden_status_t spaden_spmv_host(spaden_matrix_t A, float alpha, cons
  * spaden_spmv_host_batched -- nvec independent products y_k = alpha*A*x_k + beta*y_k
  * with HOST vectors, pipelined: the host->device copy of x_{k+1} and the
  * device->host copy of y_{k-1} overlap the SpMV of vector k (two internal copy
- * streams owned by the handle, triple-buffered device staging).
+ * streams owned by the handle, device staging in 3 slots by default;
+ * SPADEN_PIPE_SLOTS=2..8, read when the handle first builds its pipeline).
  *
  *   h_x     host float32, vector k at h_x + k*ldx (ldx >= n); pinned memory
  *           is required for the copies to overlap.

@@ -3,6 +3,7 @@
 // spmv.cu kernels.
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <new>
 #include <string>
 
@@ -44,12 +45,15 @@ static spaden_status_t check_device_ptr(const void *p, const char *name, int dev
 static void release(Matrix *A) {
     if (!A) return;
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap,   A->blk_offset, A->values,
-                    A->stage_x,     A->stage_y,  A->pipe_x[0], A->pipe_x[1], A->pipe_x[2],
-                    A->pipe_y[0],   A->pipe_y[1], A->pipe_y[2], A->tiles,
+                    A->stage_x,     A->stage_y,  A->tiles,
                     A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->chunk_done,
                     A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
     for (void *p : ptrs)
         if (p) cudaFree(p);
+    for (int j = 0; j < Matrix::kMaxPipe; ++j) {
+        if (A->pipe_x[j]) cudaFree(A->pipe_x[j]);
+        if (A->pipe_y[j]) cudaFree(A->pipe_y[j]);
+    }
     for (int q = 0; q < A->n_res_parts; ++q) {
         const spaden::ResPart &P = A->res[q];
         void *rp[] = {P.rowptr, P.colidx, P.values, P.long_rows, P.chunk_start, P.chunk_row, P.carry, P.done, P.perm};
@@ -63,10 +67,16 @@ static void release(Matrix *A) {
     delete A;
 }
 
+// slots of the batched host pipeline (SPADEN_PIPE_SLOTS overrides, 2..kMaxPipe)
+constexpr int kDefaultPipe = 3;
+
 // lazily create the batched host pipeline resources
 static spaden_status_t ensure_pipeline(Matrix *A) {
     if (A->s_h2d) return SPADEN_OK;
-    for (int j = 0; j < 3; ++j) {
+    int slots = kDefaultPipe;
+    if (const char *e = getenv("SPADEN_PIPE_SLOTS")) slots = atoi(e);
+    A->pipe_slots = slots < 2 ? 2 : (slots > Matrix::kMaxPipe ? Matrix::kMaxPipe : slots);
+    for (int j = 0; j < A->pipe_slots; ++j) {
         if (A->n > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->pipe_x[j], pad16(4 * A->n)));
         if (A->m > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->pipe_y[j], pad16(4 * A->m)));
     }
@@ -261,24 +271,26 @@ spaden_status_t spaden_spmv_host_batched(spaden_matrix_t A, float alpha, const f
     spaden_status_t s = ensure_pipeline(A);
     if (s != SPADEN_OK) return s;
     cudaStream_t cs = (cudaStream_t)stream;
-    cudaEvent_t *in_ready = A->ev, *computed = A->ev + 3, *drained = A->ev + 6;
-    // slot k%3: H2D(x_k[, y_k]) on s_h2d -> SpMV on cs -> D2H(y_k) on s_d2h.  A
-    // slot is refilled only after the SpMV of vector k-3 consumed it and its y
+    const int S = A->pipe_slots;
+    cudaEvent_t *in_ready = A->ev, *computed = A->ev + S, *drained = A->ev + 2 * S;
+    cudaEvent_t ev_start = A->ev[3 * S], ev_end = A->ev[3 * S + 1];
+    // slot k%S: H2D(x_k[, y_k]) on s_h2d -> SpMV on cs -> D2H(y_k) on s_d2h.  A
+    // slot is refilled only after the SpMV of vector k-S consumed it and its y
     // left the device, so H2D(k+1), SpMV(k) and D2H(k-1) run concurrently.
-    SPADEN_CUDA_TRY(cudaEventRecord(A->ev[9], cs));
-    SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_h2d, A->ev[9], 0));
-    SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_d2h, A->ev[9], 0));
+    SPADEN_CUDA_TRY(cudaEventRecord(ev_start, cs));
+    SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_h2d, ev_start, 0));
+    SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_d2h, ev_start, 0));
     for (int64_t k = 0; k < nvec; ++k) {
-        const int j = (int)(k % 3);
+        const int j = (int)(k % S);
         float *dx = A->pipe_x[j], *dy = A->pipe_y[j];
-        if (k >= 3) SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_h2d, drained[j], 0));
+        if (k >= S) SPADEN_CUDA_TRY(cudaStreamWaitEvent(A->s_h2d, drained[j], 0));
         if (A->n > 0)
             SPADEN_CUDA_TRY(cudaMemcpyAsync(dx, h_x + k * ldx, 4 * A->n, cudaMemcpyHostToDevice, A->s_h2d));
         if (beta != 0.f && A->m > 0)
             SPADEN_CUDA_TRY(cudaMemcpyAsync(dy, h_y + k * ldy, 4 * A->m, cudaMemcpyHostToDevice, A->s_h2d));
         SPADEN_CUDA_TRY(cudaEventRecord(in_ready[j], A->s_h2d));
         SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, in_ready[j], 0));
-        if (k >= 3 && beta == 0.f) SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, drained[j], 0));
+        if (k >= S && beta == 0.f) SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, drained[j], 0));
         s = spmv_launch(*A, alpha, dx, beta, dy, cs);
         if (s != SPADEN_OK) return s;
         SPADEN_CUDA_TRY(cudaEventRecord(computed[j], cs));
@@ -287,8 +299,8 @@ spaden_status_t spaden_spmv_host_batched(spaden_matrix_t A, float alpha, const f
             SPADEN_CUDA_TRY(cudaMemcpyAsync(h_y + k * ldy, dy, 4 * A->m, cudaMemcpyDeviceToHost, A->s_d2h));
         SPADEN_CUDA_TRY(cudaEventRecord(drained[j], A->s_d2h));
     }
-    SPADEN_CUDA_TRY(cudaEventRecord(A->ev[10], A->s_d2h));
-    SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, A->ev[10], 0));
+    SPADEN_CUDA_TRY(cudaEventRecord(ev_end, A->s_d2h));
+    SPADEN_CUDA_TRY(cudaStreamWaitEvent(cs, ev_end, 0));
     SPADEN_CUDA_TRY(cudaStreamSynchronize(cs));
     return SPADEN_OK;
 }

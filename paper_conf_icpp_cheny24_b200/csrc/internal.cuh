@@ -77,10 +77,12 @@ struct spaden_matrix_s {
     // host-API staging buffers (lazily allocated): [2] slots for the batched pipeline
     float *stage_x = nullptr;          // spaden_spmv_host
     float *stage_y = nullptr;
-    float *pipe_x[3] = {};             // spaden_spmv_host_batched: triple-buffered slots
-    float *pipe_y[3] = {};
+    static constexpr int kMaxPipe = 8;  // spaden_spmv_host_batched: up to kMaxPipe slots
+    int pipe_slots = 0;                 // slots in use (SPADEN_PIPE_SLOTS, default kDefaultPipe)
+    float *pipe_x[kMaxPipe] = {};
+    float *pipe_y[kMaxPipe] = {};
     cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
-    cudaEvent_t ev[11] = {};
+    cudaEvent_t ev[3 * kMaxPipe + 2] = {};
 };
 
 namespace spaden {
