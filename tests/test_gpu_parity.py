@@ -637,10 +637,13 @@ def test_every_tile_config_same_result(sp, torch, cfg, monkeypatch):
 
 
 @pytest.mark.parametrize("beta", [0.0, 0.5])
-def test_spmv_host_batched(sp, torch, beta):
+@pytest.mark.parametrize("slots", [None, 2, 8])
+def test_spmv_host_batched(sp, torch, beta, slots, monkeypatch):
+    if slots is not None:  # read when the handle first builds its pipeline
+        monkeypatch.setenv("SPADEN_PIPE_SLOTS", str(slots))
     A = W.make("fem62k")
     M = convert(sp, torch, A)
-    K = 5
+    K = 11  # > 8 slots: every slot is reused
     X = torch.from_numpy(np.stack([W.vector(A.n, 40 + k) for k in range(K)])).pin_memory()
     Y0 = np.stack([W.vector(A.m, 60 + k) for k in range(K)])
     Y = torch.from_numpy(Y0.copy()).pin_memory()
