@@ -347,45 +347,50 @@ def main():
     except Exception:
         pass
 
+    # ---- e2e through the C ABI with host buffers (H2D x (+y), SpMV, D2H y per step),
+    # every rank on its row slice (x replicated from host memory, no collective);
+    # time = max over ranks, value = all ranks' nonzeros / that time
+    beta = 0.0 if wl.c is None else 1.0
+    m_loc = wl.r1 - wl.r0
+    # spaden_spmv_host_batched: per step H2D of x_k (+ y_k if beta != 0), SpMV, D2H of y_k,
+    # pipelined across steps (copies of neighbouring steps overlap the SpMV)
+    K = int(max(2, min(args.steps, (512 << 20) // (4 * (wl.n + m_loc)))))
+    X = torch.empty((K, wl.n), dtype=torch.float32).pin_memory()
+    X.copy_(wl.x0.cpu().expand(K, wl.n))
+    Y = torch.full((K, m_loc), wl.c or 0.0, dtype=torch.float32).pin_memory()
+    # warm-up over the whole batch: the first pass over freshly pinned
+    # buffers runs ~20% slower (measured, tools/e2e_sweep.py)
+    M.spmv_host_batched(X, Y, alpha=wl.alpha, beta=beta, stream=stream)
+    # three timed passes of K steps each (PCIe throughput varies run to
+    # run); the reported value is the median pass
+    passes = []
+    for _ in range(3):
+        if beta:
+            Y.fill_(wl.c)
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        e0.record(stream)
+        M.spmv_host_batched(X, Y, alpha=wl.alpha, beta=beta, stream=stream)
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        tp = torch.tensor([e0.elapsed_time(e1) / K], device=dev)
+        if world > 1:
+            dist.all_reduce(tp, op=dist.ReduceOp.MAX)
+        passes.append(float(tp.item()))
+    e2e_ms = statistics.median(passes)
+    e2e = {"value": 2.0 * wl.nnz / (e2e_ms * 1e-3) / 1e9, "unit": UNIT,
+           "h2d_bytes_per_step": world * 4 * wl.n + (4 * wl.m if beta else 0), "d2h_bytes_per_step": 4 * wl.m,
+           "ms_per_step": e2e_ms, "steps": K, "passes_ms_per_step": passes,
+           "api": "spaden_spmv_host_batched (pinned host x_k/y_k, copies overlapped with SpMV; "
+                  "per rank: full x_k in, its row slice of y_k out; max over ranks)"}
+    del X, Y
+
     line = None
     if rank == 0:
         clocks = clk.summary()
-        beta = 0.0 if wl.c is None else 1.0
-        # ---- e2e through the C ABI with host buffers (H2D x (+y), SpMV, D2H y per step)
-        e2e = None
-        if world == 1:
-            # spaden_spmv_host_batched: per step H2D of x_k (+ y_k if beta != 0), SpMV, D2H of y_k,
-            # pipelined across steps (copies of neighbouring steps overlap the SpMV)
-            K = int(max(2, min(args.steps, (512 << 20) // (4 * (wl.n + wl.m)))))
-            X = torch.empty((K, wl.n), dtype=torch.float32).pin_memory()
-            X.copy_(wl.x0.cpu().expand(K, wl.n))
-            Y = torch.full((K, wl.m), wl.c or 0.0, dtype=torch.float32).pin_memory()
-            # warm-up over the whole batch: the first pass over freshly pinned
-            # buffers runs ~20% slower (measured, tools/e2e_sweep.py)
-            M.spmv_host_batched(X, Y, alpha=wl.alpha, beta=beta, stream=stream)
-            if beta:
-                Y.fill_(wl.c)
-            # three timed passes of K steps each (PCIe throughput varies run to
-            # run); the reported value is the median pass
-            passes = []
-            for _ in range(3):
-                if beta:
-                    Y.fill_(wl.c)
-                e0 = torch.cuda.Event(enable_timing=True)
-                e1 = torch.cuda.Event(enable_timing=True)
-                torch.cuda.synchronize(dev)
-                e0.record(stream)
-                M.spmv_host_batched(X, Y, alpha=wl.alpha, beta=beta, stream=stream)
-                e1.record(stream)
-                torch.cuda.synchronize(dev)
-                passes.append(e0.elapsed_time(e1) / K)
-            e2e_ms = statistics.median(passes)
-            e2e = {"value": 2.0 * wl.nnz / (e2e_ms * 1e-3) / 1e9, "unit": UNIT,
-                   "h2d_bytes_per_step": 4 * wl.n + (4 * wl.m if beta else 0), "d2h_bytes_per_step": 4 * wl.m,
-                   "ms_per_step": e2e_ms, "steps": K, "passes_ms_per_step": passes,
-                   "api": "spaden_spmv_host_batched (pinned host x_k/y_k, copies overlapped with SpMV)"}
-            del X, Y
-
         # ---- cuSPARSE CSR SpMV on the same matrix and GPU (north_star comparison)
         cus = None
         if not args.no_cusparse and world == 1:
