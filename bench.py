@@ -17,8 +17,8 @@ needed between steps (x, 6 MB, is L2-resident as in any iterative solver).
 A matrix that fits L2 (fem62k) is measured flushed by default (--l2 auto): a
 256 MB write before every step, the step timed by the SpMV's own events.
 
---impl reference times the CPU oracle (oracle/, fp64 CSR SpMV, single thread)
-on a bounded row sample per step -- this tier's reference arm.
+--impl reference times the CPU oracle (oracle/, fp64 CSR SpMV, Alg. 1, the row
+loop on all host cores) on a bounded row sample per step -- this tier's reference arm.
 """
 from __future__ import annotations
 
@@ -49,8 +49,11 @@ def parse():
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=2000)
     p.add_argument("--warmup", type=int, default=20)
-    p.add_argument("--workload", default="fem1p5m",
-                   help="one of %s, or rmatNN (PageRank on R-MAT scale NN, e.g. rmat25)" % sorted(W.CONFIGS))
+    p.add_argument("--workload", default=None,
+                   help="one of %s, or rmatNN (PageRank on R-MAT scale NN, e.g. rmat25); default fem1p5m "
+                        "at --gpus 1 (the single-GPU HBM-roofline config) and rmat25 for --gpus > 1 (the "
+                        "north_star multi-GPU config; take a scaling curve with an explicit --workload)"
+                        % sorted(W.CONFIGS))
     p.add_argument("--dtype", default="fp32", choices=["fp32", "fp16"])
     p.add_argument("--impl", default="spaden", choices=["spaden", "reference"])
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -67,7 +70,26 @@ def parse():
     p.add_argument("--l2", default="auto", choices=["auto", "flush", "warm"],
                    help="flush = write a 256 MB buffer before every timed step and take the step time from "
                         "the SpMV's own events; auto = flush when the matrix fits the 126 MB L2")
-    return p.parse_args()
+    a = p.parse_args()
+    if a.workload is None:
+        a.workload = "fem1p5m" if a.gpus <= 1 else "rmat25"
+    return a
+
+
+def spawn_ranks(args):
+    """--gpus N > 1 without a torchrun environment: re-launch this script as N
+    NCCL ranks (one process per GPU) with torch.distributed.run on 127.0.0.1."""
+    import socket
+    import subprocess
+
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")  # communicator lines (rank count, NVLS) on stderr
+    return subprocess.call(cmd, env=env)
 
 
 def peaks():
@@ -142,24 +164,39 @@ class Clocks:
                 "reasons": sorted(self.reasons - {"gpu_idle"}), "samples": len(self.samples)}
 
 
-def cpu_oracle_gflops(A, x, seconds):
-    """The oracle (fp64 CSR SpMV, single thread) on whole-matrix passes, bounded in time."""
+def cpu_oracle_gflops(A, x, seconds, all_cores=False):
+    """The oracle (fp64 CSR SpMV, Alg. 1) on whole-matrix passes, bounded in time:
+    one thread, or the row loop on all host cores (OpenMP static schedule)."""
     import oracle
     oracle.lib()
     rp = np.ascontiguousarray(A.rowptr, np.int64)
     v = np.ascontiguousarray(A.values.astype(np.float64))
     xx = np.ascontiguousarray(x.astype(np.float64))
+    fn = (lambda: oracle.spmv_omp(rp, A.colidx, v, xx)[2]) if all_cores else (lambda: oracle.spmv(rp, A.colidx, v, xx) and 1)
     t0 = time.perf_counter()
     passes = 0
+    threads = 1
     while True:
-        oracle.spmv(rp, A.colidx, v, xx)
+        threads = fn()
         passes += 1
         if time.perf_counter() - t0 >= seconds:
             break
     dt = time.perf_counter() - t0
-    return {"value": 2.0 * A.nnz * passes / dt / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+    return {"value": 2.0 * A.nnz * passes / dt / 1e9, "unit": UNIT, "cores": int(threads), "kind": "oracle",
+            "host_cpu": _cpu_model(), "os_cpu_count": os.cpu_count(),
             "sample": f"{passes} full passes over the {A.m}x{A.n} matrix ({A.nnz} nnz), fp64, "
-                      f"{dt:.1f} s wall"}
+                      f"{'OpenMP ' + str(threads) + ' threads' if all_cores else '1 thread'}, {dt:.1f} s wall"}
+
+
+def _cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 def reference_arm(args):
@@ -181,9 +218,9 @@ def reference_arm(args):
         x = W.vector(A.n, 2)
     vals = A.values if args.dtype == "fp32" else oracle.f32_to_f16(A.values)
     oracle.lib()
-    # per-step budget so that K+W steps take ~90 s of CPU time in total
+    # per-step budget so that K+W steps take ~90 s in total (all host cores)
     t0 = time.perf_counter()
-    oracle.spmv(A.rowptr, A.colidx, vals, x)
+    oracle.spmv_omp(A.rowptr, A.colidx, vals, x)
     full = time.perf_counter() - t0
     frac = min(1.0, 90.0 / max(1, args.steps + args.warmup) / max(full, 1e-6))
     r1 = max(8, int(A.m * frac) // 8 * 8)
@@ -192,11 +229,12 @@ def reference_arm(args):
     rp = np.ascontiguousarray(S.rowptr, np.int64)
     v = np.ascontiguousarray(sv.astype(np.float64))
     xx = np.ascontiguousarray(x.astype(np.float64))
+    threads = 1
     for _ in range(args.warmup):
-        oracle.spmv(rp, S.colidx, v, xx)
+        threads = oracle.spmv_omp(rp, S.colidx, v, xx)[2]
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        oracle.spmv(rp, S.colidx, v, xx)
+        threads = oracle.spmv_omp(rp, S.colidx, v, xx)[2]
     dt = time.perf_counter() - t0
     val = 2.0 * S.nnz * args.steps / dt / 1e9
     line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
@@ -205,8 +243,10 @@ def reference_arm(args):
             "impl": "reference",
             "config": {"workload": args.workload, "m": A.m, "n": A.n, "nnz": A.nnz, "values": args.dtype,
                        "sample_rows": r1, "sample_nnz": S.nnz},
-            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"rows [0,{r1}) of {args.workload} ({S.nnz} nnz) per step"},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle",
+                             "host_cpu": _cpu_model(), "os_cpu_count": os.cpu_count(),
+                             "sample": f"rows [0,{r1}) of {args.workload} ({S.nnz} nnz) per step, "
+                                       f"OpenMP {threads} threads"},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -259,9 +299,13 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_icpp_cheny24_b200 as sp
-    from paper_conf_icpp_cheny24_b200.dist import FusedIteratedSpMV, IteratedSpMV
+    from paper_conf_icpp_cheny24_b200.dist import FusedIteratedSpMV, IteratedSpMV, convert_slice
 
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return spawn_ranks(args)
     world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world} (launch one rank per GPU)")
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
@@ -276,12 +320,19 @@ def main():
     # warm-up conversion of the same matrix: loads every kernel the conversion
     # uses (lazy module loading) so the timed conversion below measures the
     # conversion only
-    sp.convert(*wl.local, wl.n, storage=args.dtype, residual_max_popc=args.hybrid).free()
+    convert_slice(*wl.local, wl.n, storage=args.dtype, residual_max_popc=args.hybrid).free()
     torch.cuda.synchronize(dev)
-    t0 = time.perf_counter()
-    M = sp.convert(*wl.local, wl.n, storage=args.dtype, residual_max_popc=args.hybrid)
-    torch.cuda.synchronize(dev)
-    convert_s = time.perf_counter() - t0
+    # conversion time: median of 5 warm repetitions (each includes the handle's
+    # allocations and the converter's host synchronisations)
+    conv_times = []
+    for rep in range(5):
+        t0 = time.perf_counter()
+        M = convert_slice(*wl.local, wl.n, storage=args.dtype, residual_max_popc=args.hybrid)
+        torch.cuda.synchronize(dev)
+        conv_times.append(time.perf_counter() - t0)
+        if rep < 4:
+            M.free()
+    convert_s = statistics.median(conv_times)
     info = M.info
     local_csr = wl.local
     wl.local = None
@@ -317,6 +368,8 @@ def main():
     flush = args.l2 == "flush" or (args.l2 == "auto" and info.format_bytes <= L2_BYTES)
     flush_buf = torch.empty(2 * L2_BYTES // 4, dtype=torch.float32, device=dev) if flush else None
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    gevs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)] \
+        if (world > 1 and args.exchange == "nccl") else None
     start = torch.cuda.Event(enable_timing=True)
     end = torch.cuda.Event(enable_timing=True)
     if world > 1:
@@ -328,8 +381,12 @@ def main():
             if flush:  # evict A, x and y from L2 (outside the step's events)
                 flush_buf.fill_(float(i))
             ev_pair[0] = evs[i]
+            if gevs is not None:
+                it.gather_events = gevs[i]
             it.step(wl.alpha, wl.c)
         ev_pair[0] = None
+        if gevs is not None:
+            it.gather_events = None
         end.record(stream)
         torch.cuda.synchronize(dev)
     if world > 1:
@@ -345,19 +402,38 @@ def main():
     ms_per_step = elapsed_ms / args.steps
     gflops = 2.0 * wl.nnz * args.steps / (elapsed_ms * 1e-3) / 1e9
 
-    # ---- roofline of the dominant kernel (the SpMV) on this rank
+    # per-iteration SpMV and all-gather times (max over ranks of each rank's mean)
     kavg_ms = float(np.mean(kernel_ms))
+    split = None
+    if world > 1:
+        tt = torch.tensor([kavg_ms, float(np.mean([a.elapsed_time(b) for a, b in gevs])) if gevs else 0.0],
+                          device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        nz = torch.tensor([float(wl.local_nnz)], device=dev)
+        dist.all_reduce(nz, op=dist.ReduceOp.MAX)
+        split = {"nnz_imbalance_max_over_mean": float(nz.item()) / (wl.nnz / world),
+                 "t_spmv_ms": float(tt[0]), "t_allgather_ms": float(tt[1]) if gevs else None,
+                 "t_iter_ms": ms_per_step,
+                 "note": ("NCCL all_gather_into_tensor after the SpMV" if gevs else
+                          "fused peer stores: the exchange runs inside the SpMV (+ one device barrier)")}
+
+    # ---- roofline of the dominant kernel (the SpMV) on this rank
     abytes = alg_bytes(wl.r1 - wl.r0, wl.n, wl.local_nnz, info.Bnrow, info.Bnnz, sv, beta_nonzero=wl.c is not None,
                        res_nnz=info.residual_nnz)
     peak, peak_kind = peaks()
     achieved = abytes / (kavg_ms * 1e-3) / 1e9
-    traffic = None
+    # roofline.traffic: dram__bytes_read.sum + dram__bytes_write.sum per launch from an
+    # `ncu --set full` capture of this kernel (not measurable inside a timed run);
+    # a STORED value, labelled with the capture it came from (profiles/ncu_traffic.json)
+    traffic, traffic_src = None, None
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
             tr = json.load(f)
         key = f"{args.workload}/{args.dtype}"
-        if key in tr and world == 1:
+        if key in tr and world == 1 and args.hybrid in (-1, 0):
             traffic = tr[key]["dram_bytes_per_launch"]
+            traffic_src = {k: v for k, v in tr[key].items() if k != "dram_bytes_per_launch"}
+            traffic_src["kind"] = "stored: ncu --set full capture (see source), not measured in this run"
     except Exception:
         pass
 
@@ -409,40 +485,40 @@ def main():
         cus = None
         if not args.no_cusparse and world == 1:
             try:
-                Ac = torch.sparse_csr_tensor(*local_csr, size=(wl.m, wl.n))
-                xv = wl.x0.contiguous()
-                for _ in range(5):
-                    yc = torch.mv(Ac, xv)
-                reps = max(20, min(args.steps, 500))
-                c0 = torch.cuda.Event(enable_timing=True)
-                c1 = torch.cuda.Event(enable_timing=True)
-                torch.cuda.synchronize(dev)
-                c0.record(stream)
-                for _ in range(reps):
-                    yc = torch.mv(Ac, xv)
-                c1.record(stream)
-                torch.cuda.synchronize(dev)
-                cms = c0.elapsed_time(c1) / reps
-                csr_bytes = 4 * (wl.m + 1) + 8 * wl.nnz
-                cus = {"impl": "torch.mv(sparse_csr fp32) -> cuSPARSE SpMV", "ms": cms,
-                       "gflops": 2.0 * wl.nnz / (cms * 1e-3) / 1e9,
-                       "footprint_bytes": csr_bytes, "bytes_per_nnz": csr_bytes / wl.nnz,
-                       "speedup_spaden_vs_cusparse": cms / kavg_ms,
-                       "footprint_saving": csr_bytes / info.format_bytes}
-                del Ac, yc
+                sys.path.insert(0, os.path.join(ROOT, "tools"))
+                import cusparse_csr
+                rp_d, ci_d, v_d = local_csr
+                v32 = v_d.float().contiguous()  # the paper's baseline: fp32 CSR
+                res = cusparse_csr.time_spmv(rp_d, ci_d, v32, wl.x0.contiguous(), wl.m, wl.n, stream,
+                                             reps=max(20, min(args.steps, 500)))
+                best = min(res, key=lambda k: res[k]["ms"])
+                cus = {"impl": "cusparseSpMV fp32 CSR, int32 indices (ctypes, same stream)",
+                       "algs": {k: {"ms": r["ms"], "buffer_bytes": r["buffer_bytes"],
+                                    "footprint_bytes": r["footprint_bytes"]} for k, r in res.items()},
+                       "best": best, "ms": res[best]["ms"],
+                       "gflops": 2.0 * wl.nnz / (res[best]["ms"] * 1e-3) / 1e9,
+                       "footprint_bytes": res[best]["footprint_bytes"],
+                       "bytes_per_nnz": res[best]["footprint_bytes"] / wl.nnz,
+                       "speedup_spaden_vs_cusparse": res[best]["ms"] / kavg_ms,
+                       "footprint_saving": res[best]["footprint_bytes"] / info.format_bytes,
+                       "note": ("back-to-back calls, no L2 flush" + (" (matrix fits L2: warm)"
+                                                                      if info.format_bytes <= L2_BYTES else ""))}
+                del res, v32
             except Exception as e:  # pragma: no cover
-                cus = {"error": repr(e)[:200]}
+                cus = {"error": repr(e)[:300]}
 
         cpu = None
         if not args.no_cpu_baseline and world == 1:
             if wl.host is not None:
-                cpu = cpu_oracle_gflops(wl.host, wl.x0.cpu().numpy(), args.cpu_seconds)
+                S = wl.host
             else:  # bounded row sample of the GPU-generated matrix
                 rp, ci, v = local_csr
                 k = max(8, min(wl.m, wl.m // 64))
                 hi = int(rp[k].item())
                 S = W.CSR(k, wl.n, rp[:k + 1].cpu().numpy(), ci[:hi].cpu().numpy(), v[:hi].cpu().numpy())
-                cpu = cpu_oracle_gflops(S, wl.x0.cpu().numpy(), args.cpu_seconds)
+            xs = wl.x0.cpu().numpy()
+            cpu = cpu_oracle_gflops(S, xs, args.cpu_seconds / 2, all_cores=True)
+            cpu["single_thread"] = cpu_oracle_gflops(S, xs, args.cpu_seconds / 2, all_cores=False)
 
         # ---- the other value precision on the same matrix (kernel time only)
         variants = {}
@@ -510,21 +586,26 @@ def main():
                        "parallelism": f"row-partition x{world}" + (
                            (" + NCCL all-gather" if args.exchange == "nccl" else " + fused peer-store all-gather")
                            if world > 1 else ""),
-                       "exchange": args.exchange,
                        "l2": ("256 MB L2 flush before every step; step time = spaden_spmv's CUDA events"
                               if flush else "inputs larger than L2 (A > 126 MB), no flush"
                               if info.format_bytes > L2_BYTES else "matrix fits L2, no flush (--l2 warm): warm-L2 number"),
-                       "step": wl.step_desc},
+                       "step": wl.step_desc,
+                       **({"exchange": args.exchange} if world > 1 else {})},
             "hbm_gbs": achieved,
             "bytes_per_nnz": {"stored": info.format_bytes / max(1, info.nnz),
                               "moved": abytes / max(1, wl.local_nnz)},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "frac_of_8tbps_spec": achieved / 8000.0,
+                         "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
+                         "frac_of_8tbps_spec": achieved / 8000.0,
                          "peak_kind": f"{peak_kind} copy bandwidth (MEASURED_PEAKS.json hbm_gbs)",
                          "kernel": "spaden_spmv (k_spmv_tiled [+ long-row chunks/fix-up])",
                          "kernel_ms": kavg_ms, "alg_bytes_per_launch": abytes,
                          "kernel_ms_p10_p50_p90": [float(np.percentile(kernel_ms, q)) for q in (10, 50, 90)]},
-            "convert": {"seconds": convert_s, "ns_per_nnz": convert_s * 1e9 / max(1, wl.local_nnz)},
+            "convert": {"seconds": convert_s, "ns_per_nnz": convert_s * 1e9 / max(1, wl.local_nnz),
+                        "reps_seconds": conv_times,
+                        "what": "median of 5 warm spaden_convert_csr_to_bitmap_ex calls (host wall clock incl. "
+                                "allocation and the converter's host synchronisations)"},
+            "multi_gpu": split,
             "cusparse_csr": cus,
             "variants": variants,
             "spmm": spmm,

@@ -106,7 +106,12 @@ typedef struct {
                                    instead of bitBSR blocks (0 = pure bitBSR, max 64;
                                    -1 = automatic: 4 when the mean block fill nnz/Bnnz
                                    is below 8, else 0)                                     */
-    int32_t reserved[6];
+    float   auto_mean_fill;     /* > 0: the mean block fill nnz/Bnnz the automatic choice
+                                   (residual_max_popc = -1) uses instead of this matrix's
+                                   own.  A row-partitioned caller passes the WHOLE matrix's
+                                   fill (spaden_count_blocks + a sum over ranks) so every
+                                   slice takes the same t (partition invariance).  0 = own. */
+    int32_t reserved[5];
 } spaden_convert_opts_t;
 
 /*
@@ -123,8 +128,13 @@ typedef struct {
  *   stream          cudaStream_t (void*).
  *   out             receives the new handle (NULL on error).
  *
- * Stream-ordered; performs exactly one host synchronisation of `stream` (to
- * learn Bnnz and the validation result before allocating).  A stored 0.0 keeps
+ * Stream-ordered.  The host synchronises `stream` a few times, each to read a
+ * size before allocating: the block count Bnnz and the validation result, the
+ * SpMV schedule's tile / long-row counts, the long-row chunk count (only when
+ * long block-rows exist); the hybrid split (_ex, t > 0) adds its own (kept
+ * counts, residual column parts).  Other streams and the device are never
+ * synchronised.  Row rotations for the decode's shared-memory banks are chosen
+ * here as well (a schedule pass; they never change y).  A stored 0.0 keeps
  * its bit (the round trip bitBSR -> CSR is the identity).  Invalid CSR is
  * reported as INVALID_ARGUMENT / INDEX_OUT_OF_RANGE / UNSORTED_OR_DUPLICATE;
  * nothing is leaked on error.  m == 0, n == 0 or nnz == 0 give a valid handle.
@@ -134,6 +144,18 @@ SPADEN_API spaden_status_t spaden_convert_csr_to_bitmap(int64_t m, int64_t n, in
                                              const void *d_values, spaden_dtype_t values_dtype,
                                              spaden_dtype_t storage_dtype, void *stream,
                                              spaden_matrix_t *out);
+
+/*
+ * spaden_count_blocks -- the converter's validation + block-count pass only
+ * (C1 of the conversion): *Bnnz receives the number of non-empty
+ * 8x8 blocks of the CSR matrix, without building the format.  Same argument
+ * rules and error codes as spaden_convert_csr_to_bitmap; one host
+ * synchronisation; allocates only stream-ordered temporaries.  Bnnz is additive
+ * over 8-row-aligned row slices, so ranks of a row partition sum it to get the
+ * whole matrix's mean fill (spaden_convert_opts_t.auto_mean_fill).
+ */
+SPADEN_API spaden_status_t spaden_count_blocks(int64_t m, int64_t n, int64_t nnz, const int32_t *d_rowptr,
+                                               const int32_t *d_colidx, void *stream, int64_t *Bnnz);
 
 /*
  * spaden_convert_csr_to_bitmap_ex -- as spaden_convert_csr_to_bitmap, with options
@@ -156,9 +178,9 @@ SPADEN_API spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n,
  * and a dense vector x as input and produces a dense vector y").
  *
  *   A         handle from spaden_convert_csr_to_bitmap.  The bitBSR arrays are
- *             immutable, but block-rows too large for a pipeline stage use a
- *             per-handle scratch buffer: calls on one handle must be ordered
- *             (same stream, or synchronised across streams).
+ *             immutable; block-rows too large for a pipeline stage use one of 4
+ *             per-handle scratch sets, taken round robin per call, so up to 4
+ *             calls on one handle may run concurrently on different streams.
  *   d_x       float32[n] (read-only; only entries referenced by a set bit are read,
  *             structural zeros are never multiplied).
  *   d_y       float32[m]; with beta == 0 it is write-only (its old contents, even
@@ -166,8 +188,12 @@ SPADEN_API spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n,
  *   stream    cudaStream_t (void*).
  *
  * Accumulation is fp32 in a fixed order that depends only on each block-row's own
- * blocks (deterministic; identical for any row partition aligned to 8 rows).
- * Never allocates and never synchronises: CUDA-graph capturable.
+ * blocks: deterministic, and bitwise identical for any row partition aligned to
+ * 8 rows (whether a block-row takes the tile path or the long-row path is a
+ * constant cost threshold, kLongRowBytes; the hybrid's automatic threshold is
+ * the same on every slice when spaden_convert_opts_t.auto_mean_fill carries the
+ * whole matrix's fill).  Never allocates and never synchronises: CUDA-graph
+ * capturable.
  */
 SPADEN_API spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const float *d_x, float beta,
                             float *d_y, void *stream);
@@ -186,7 +212,9 @@ SPADEN_API spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const flo
  * identical to spaden_spmv.
  *   h_out_ptrs  HOST array of npeers device pointers (1 <= npeers <= 8).
  *   d_y         local y (read if beta != 0, also written if non-NULL; may be NULL).
- * Requires a pure bitBSR handle (no hybrid residual).
+ * Requires a pure bitBSR handle (converted with residual_max_popc = 0, or an
+ * automatic choice that took t = 0); a hybrid handle returns
+ * SPADEN_ERR_UNSUPPORTED.
  */
 SPADEN_API spaden_status_t spaden_spmv_scatter(spaden_matrix_t A, float alpha, const float *d_x, float beta,
                                                float *d_y, float *const *h_out_ptrs, int32_t npeers,

@@ -26,7 +26,7 @@ def build(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(["gcc", "-O2", "-std=gnu11", "-fPIC", "-shared",
-                               "-ffp-contract=off", "-fno-fast-math", _SRC, "-o", tmp, "-lm"])
+                               "-ffp-contract=off", "-fno-fast-math", "-fopenmp", _SRC, "-o", tmp, "-lm"])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -41,6 +41,8 @@ def lib():
         P = ctypes.c_void_p
         I64 = ctypes.c_int64
         _lib.oracle_csr_spmv_f64.argtypes = [I64, P, P, P, P, P, P]
+        _lib.oracle_csr_spmv_f64_omp.argtypes = [I64, P, P, P, P, P, P]
+        _lib.oracle_csr_spmv_f64_omp.restype = ctypes.c_int
         _lib.oracle_bitbsr_count.argtypes = [I64, I64, I64, P, P, P]
         _lib.oracle_bitbsr_count.restype = ctypes.c_int
         _lib.oracle_csr_to_bitbsr.argtypes = [I64, I64, I64, P, P, P, ctypes.c_int, P, P, P, P, P]
@@ -72,6 +74,20 @@ def spmv(rowptr, colidx, values, x):
     s = np.zeros(m, np.float64)
     lib().oracle_csr_spmv_f64(m, _p(rowptr), _p(colidx), _p(v), _p(xx), _p(y), _p(s))
     return y, s
+
+
+def spmv_omp(rowptr, colidx, values, x):
+    """spmv() with the row loop on all host cores (OpenMP, static schedule);
+    bitwise equal to spmv().  Returns (y, s, threads)."""
+    rowptr = _c(rowptr, np.int64)
+    colidx = _c(colidx, np.int32)
+    v = _c(np.asarray(values).astype(np.float64), np.float64)
+    xx = _c(np.asarray(x).astype(np.float64), np.float64)
+    m = rowptr.shape[0] - 1
+    y = np.zeros(m, np.float64)
+    s = np.zeros(m, np.float64)
+    t = lib().oracle_csr_spmv_f64_omp(m, _p(rowptr), _p(colidx), _p(v), _p(xx), _p(y), _p(s))
+    return y, s, int(t)
 
 
 def f32_to_f16(values) -> np.ndarray:

@@ -12,6 +12,10 @@
  *
  * Functions and the passage each follows:
  *   oracle_csr_spmv_f64      Algorithm 1, standard CSR SpMV (§2.1), fp64.
+ *   oracle_csr_spmv_f64_omp  The same Algorithm 1 with the row loop split over OpenMP
+ *                            threads (schedule(static)); every row is still one
+ *                            sequential-k sum, so y and s are bitwise equal to the
+ *                            serial function (bench.py's all-cores cpu_baseline).
  *   oracle_bitbsr_count      §4.2 bitBSR, block positions "encoded as CSR".
  *   oracle_csr_to_bitbsr     §4.2 / Fig. 4 bitBSR conversion: 8x8 blocks
  *                            (P:L132), bit = 8*(r%8)+(c%8) with LSB = top-left,
@@ -35,6 +39,7 @@
 #include <stdlib.h>
 #include <string.h>
 #include <math.h>
+#include <omp.h>
 
 /* status codes of the oracle's own input checks (independent of include/spaden.h) */
 enum { ORC_OK = 0, ORC_BAD_ROWPTR = 1, ORC_COL_RANGE = 2, ORC_UNSORTED = 3, ORC_NOMEM = 4 };
@@ -56,6 +61,31 @@ void oracle_csr_spmv_f64(int64_t m, const int64_t *rowptr, const int32_t *colidx
         y[i] = acc;
         if (s) s[i] = abs_acc;
     }
+}
+
+/* Alg. 1 over all host cores: rows split statically over OpenMP threads, each
+ * row the same sequential sum as above.  Returns the number of threads used. */
+int oracle_csr_spmv_f64_omp(int64_t m, const int64_t *rowptr, const int32_t *colidx,
+                            const double *val, const double *x, double *y, double *s)
+{
+    int threads = 1;
+#pragma omp parallel
+    {
+#pragma omp single
+        threads = omp_get_num_threads();
+#pragma omp for schedule(static)
+        for (int64_t i = 0; i < m; ++i) {
+            double acc = 0.0, abs_acc = 0.0;
+            for (int64_t k = rowptr[i]; k < rowptr[i + 1]; ++k) {
+                double p = val[k] * x[colidx[k]];
+                acc += p;
+                abs_acc += fabs(p);
+            }
+            y[i] = acc;
+            if (s) s[i] = abs_acc;
+        }
+    }
+    return threads;
 }
 
 /* ---------------------------------------------------------- input checks */

@@ -5,7 +5,7 @@ in the library's CUDA kernels.  PyTorch supplies device memory and streams.
 There is no CPU fallback: importing this package on a machine without the
 built library raises ImportError, and every call on a missing device fails.
 
-Raw entry points keep the C names (spaden_convert_csr_to_bitmap, spaden_spmv,
+Raw entry points keep the C names (spaden_convert_csr_to_bitmap, spaden_count_blocks, spaden_spmv,
 spaden_spmv_host, spaden_free, spaden_get_info, spaden_get_arrays, spaden_spmv_launch_count,
 spaden_status_string, spaden_last_error_message, spaden_version); `convert`
 and `Matrix` wrap them for torch tensors.
@@ -53,7 +53,7 @@ class spaden_arrays_t(ctypes.Structure):
 
 class spaden_convert_opts_t(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_int32), ("residual_max_popc", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 6)]
+                ("auto_mean_fill", ctypes.c_float), ("reserved", ctypes.c_int32 * 5)]
 
 
 _P = ctypes.c_void_p
@@ -69,6 +69,9 @@ spaden_convert_csr_to_bitmap_ex = _lib.spaden_convert_csr_to_bitmap_ex
 spaden_convert_csr_to_bitmap_ex.argtypes = [_I64, _I64, _I64, _P, _P, _P, ctypes.c_int, ctypes.c_int,
                                             ctypes.POINTER(spaden_convert_opts_t), _P, ctypes.POINTER(_P)]
 spaden_convert_csr_to_bitmap_ex.restype = _ST
+spaden_count_blocks = _lib.spaden_count_blocks
+spaden_count_blocks.argtypes = [_I64, _I64, _I64, _P, _P, _P, ctypes.POINTER(_I64)]
+spaden_count_blocks.restype = _ST
 spaden_spmv = _lib.spaden_spmv
 spaden_spmv.argtypes = [_P, _F, _P, _F, _P, _P]
 spaden_spmv.restype = _ST
@@ -106,7 +109,7 @@ spaden_version = _lib.spaden_version
 spaden_version.argtypes = []
 spaden_version.restype = ctypes.c_char_p
 
-EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_spmv", "spaden_spmm",
+EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_count_blocks", "spaden_spmv", "spaden_spmm",
             "spaden_spmv_scatter", "spaden_spmv_host", "spaden_spmv_host_batched",
             "spaden_free",
             "spaden_get_info", "spaden_get_arrays", "spaden_spmv_launch_count", "spaden_status_string",
@@ -282,10 +285,24 @@ class Matrix:
             pass
 
 
-def convert(rowptr, colidx, values, n: int, storage=None, stream=None, residual_max_popc: int = 0) -> Matrix:
+def count_blocks(rowptr, colidx, n: int, stream=None) -> int:
+    """Non-empty 8x8 blocks (Bnnz) of a CSR matrix: the converter's validation and
+    count pass only (spaden_count_blocks)."""
+    torch = _torch()
+    assert rowptr.dtype == torch.int32 and colidx.dtype == torch.int32 and rowptr.is_cuda and colidx.is_cuda
+    out = ctypes.c_int64()
+    _check(spaden_count_blocks(rowptr.numel() - 1, n, colidx.numel(), ctypes.c_void_p(rowptr.data_ptr()),
+                               ctypes.c_void_p(colidx.data_ptr()), _stream_ptr(stream), ctypes.byref(out)),
+           "spaden_count_blocks")
+    return out.value
+
+
+def convert(rowptr, colidx, values, n: int, storage=None, stream=None, residual_max_popc: int = 0,
+            auto_mean_fill: float = 0.0) -> Matrix:
     """CSR (int32 CUDA tensors + fp32/fp16 values) -> bitBSR Matrix (hybrid with a CSR
     residual for blocks of <= residual_max_popc entries when that is > 0; -1 = automatic:
-    4 when the mean block fill is below 8, else pure bitBSR)."""
+    4 when the mean block fill is below 8, else pure bitBSR; the fill used is
+    auto_mean_fill when > 0 -- a row slice passes the whole matrix's)."""
     torch = _torch()
     assert rowptr.dtype == torch.int32 and colidx.dtype == torch.int32
     assert rowptr.is_cuda and colidx.is_cuda and values.is_cuda
@@ -293,7 +310,8 @@ def convert(rowptr, colidx, values, n: int, storage=None, stream=None, residual_
     sdt = vdt if storage is None else _dtype_code(storage)
     m = rowptr.numel() - 1
     h = ctypes.c_void_p()
-    opts = spaden_convert_opts_t(ctypes.sizeof(spaden_convert_opts_t), int(residual_max_popc))
+    opts = spaden_convert_opts_t(ctypes.sizeof(spaden_convert_opts_t), int(residual_max_popc),
+                                 float(auto_mean_fill))
     st = spaden_convert_csr_to_bitmap_ex(m, n, colidx.numel(), ctypes.c_void_p(rowptr.data_ptr()),
                                          ctypes.c_void_p(colidx.data_ptr()),
                                          ctypes.c_void_p(values.data_ptr()), vdt, sdt, ctypes.byref(opts),

@@ -45,7 +45,7 @@ static spaden_status_t check_device_ptr(const void *p, const char *name, int dev
 static void release(Matrix *A) {
     if (!A) return;
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap,   A->blk_offset, A->values,
-                    A->stage_x,     A->stage_y,  A->tiles,
+                    A->stage_x,     A->stage_y,  A->tiles, A->rot,
                     A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->chunk_done,
                     A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
     for (void *p : ptrs)
@@ -124,6 +124,7 @@ spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n, int64_t nn
                                                 spaden_matrix_t *out) {
     g_last_error.clear();
     int res_t = 0;
+    float auto_fill = 0.f;
     if (opts) {
         if (opts->struct_size != (int32_t)sizeof(spaden_convert_opts_t) || opts->residual_max_popc < -1 ||
             opts->residual_max_popc > 64) {
@@ -132,6 +133,12 @@ spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n, int64_t nn
             return SPADEN_ERR_INVALID_ARGUMENT;
         }
         res_t = opts->residual_max_popc;
+        auto_fill = opts->auto_mean_fill;
+        if (!(auto_fill >= 0.f && auto_fill <= 64.f)) {
+            if (out) *out = nullptr;
+            set_error("bad spaden_convert_opts_t.auto_mean_fill (must be in [0, 64])");
+            return SPADEN_ERR_INVALID_ARGUMENT;
+        }
     }
     if (!out) {
         set_error("out must not be NULL");
@@ -169,7 +176,7 @@ spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n, int64_t nn
         return SPADEN_ERR_OUT_OF_MEMORY;
     }
     A->device = dev;
-    s = convert_csr(m, n, nnz, d_rowptr, d_colidx, d_values, values_dtype, storage_dtype, res_t,
+    s = convert_csr(m, n, nnz, d_rowptr, d_colidx, d_values, values_dtype, storage_dtype, res_t, auto_fill,
                     (cudaStream_t)stream, A);
     if (s != SPADEN_OK) {
         cudaStreamSynchronize((cudaStream_t)stream);
@@ -178,6 +185,40 @@ spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n, int64_t nn
     }
     *out = A;
     return SPADEN_OK;
+}
+
+spaden_status_t spaden_count_blocks(int64_t m, int64_t n, int64_t nnz, const int32_t *d_rowptr,
+                                    const int32_t *d_colidx, void *stream, int64_t *Bnnz) {
+    g_last_error.clear();
+    if (!Bnnz) {
+        set_error("Bnnz must not be NULL");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    *Bnnz = 0;
+    if (m < 0 || n < 0 || nnz < 0) {
+        set_error("m, n, nnz must be >= 0");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (m >= (1LL << 31) - 8 || n >= (1LL << 31) - 8 || nnz >= (1LL << 31) - 1) {
+        set_error("m, n, nnz must be < 2^31 (int32 indices)");
+        return SPADEN_ERR_UNSUPPORTED;
+    }
+    if (!d_rowptr || (nnz > 0 && !d_colidx)) {
+        set_error("NULL rowptr (or colidx with nnz > 0)");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_status(e, "cudaGetDevice");
+    spaden_status_t s = check_device_ptr(d_rowptr, "rowptr", dev);
+    if (s == SPADEN_OK && nnz > 0) s = check_device_ptr(d_colidx, "colidx", dev);
+    if (s != SPADEN_OK) return s;
+    Matrix tmp;
+    tmp.device = dev;
+    s = convert_csr(m, n, nnz, d_rowptr, d_colidx, nullptr, SPADEN_R_32F, SPADEN_R_32F, 0, 0.f,
+                    (cudaStream_t)stream, &tmp, /*count_only=*/true);
+    if (s == SPADEN_OK) *Bnnz = tmp.Bnnz;
+    return s;
 }
 
 spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const float *d_x, float beta, float *d_y,

@@ -303,7 +303,8 @@ void launch_fill(int64_t m, int64_t n, int64_t NBC, const int32_t *rowptr, const
 
 spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *rowptr,
                             const int32_t *colidx, const void *values, spaden_dtype_t vdt,
-                            spaden_dtype_t sdt, int residual_max_popc, cudaStream_t st, Matrix *A) {
+                            spaden_dtype_t sdt, int residual_max_popc, float auto_mean_fill,
+                            cudaStream_t st, Matrix *A, bool count_only) {
     const int64_t Bnrow = (m + 7) / 8;
     const int64_t NBC = (n + 7) / 8;
     const int64_t max_chunks = Bnrow + nnz / kChunkNnz + 1;
@@ -369,6 +370,11 @@ spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *ro
         return SPADEN_ERR_CUDA;
     }
 
+    if (count_only) {  // spaden_count_blocks: validation + C1 only
+        A->m = m; A->n = n; A->nnz = nnz; A->Bnrow = Bnrow; A->Bnnz = h[2];
+        return SPADEN_OK;
+    }
+
     // ---- owned arrays
     A->m = m; A->n = n; A->nnz = nnz; A->Bnrow = Bnrow; A->Bnnz = Bnnz; A->storage = sdt;
     auto alloc = [&](void **ptr, size_t bytes) -> cudaError_t {
@@ -406,8 +412,13 @@ spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *ro
     // -1 = automatic: t = kAutoResidualPopc when the mean block fill is below
     // kSlotsMinFill (the low-degree regime of P:L236, where the measured best t
     // on powerlaw1m / rmat22 / rmat25 is 3-4), else pure bitBSR
-    if (residual_max_popc < 0)
-        residual_max_popc = (Bnnz > 0 && nnz < (int64_t)kSlotsMinFill * Bnnz) ? kAutoResidualPopc : 0;
+    // (auto_mean_fill > 0: the caller's whole-matrix fill, so that every row
+    // slice of a partition takes the same t)
+    if (residual_max_popc < 0) {
+        const double fill = auto_mean_fill > 0.f ? (double)auto_mean_fill
+                                                 : (Bnnz > 0 ? (double)nnz / (double)Bnnz : 64.0);
+        residual_max_popc = fill < (double)kSlotsMinFill ? kAutoResidualPopc : 0;
+    }
     if (residual_max_popc > 0) {
         spaden_status_t hs = split_residual(A, residual_max_popc, st);
         if (hs != SPADEN_OK) return hs;

@@ -423,9 +423,10 @@ spaden_status_t residual_schedule(Matrix *A, ResPart &P, cudaStream_t st) {
             P.n_chunks = nc;
             e = cudaMalloc(&P.chunk_row, 4 * (size_t)std::max(1, nc));
         }
-        if (e == cudaSuccess) e = cudaMalloc(&P.carry, 4 * (size_t)std::max(1, nc));
-        if (e == cudaSuccess) e = cudaMalloc(&P.done, 4 * (size_t)nl);
-        if (e == cudaSuccess) e = cudaMemsetAsync(P.done, 0, 4 * (size_t)nl, st);
+        constexpr int SL = Matrix::kScratchSlots;
+        if (e == cudaSuccess) e = cudaMalloc(&P.carry, 4 * (size_t)std::max(1, nc) * SL);
+        if (e == cudaSuccess) e = cudaMalloc(&P.done, 4 * (size_t)nl * SL);
+        if (e == cudaSuccess) e = cudaMemsetAsync(P.done, 0, 4 * (size_t)nl * SL, st);
         if (e == cudaSuccess) {
             k_res_chunk_rows<<<(unsigned)((nl + 255) / 256), 256, 0, st>>>(nl, P.chunk_start, P.chunk_row);
             e = cudaGetLastError();
@@ -683,13 +684,17 @@ __global__ void k_scale(int64_t m, float beta, float *__restrict__ y) {
 // accumulate their chunks (PDL launches).  Per row the parts are added in
 // column order (a function of the row and of n: partition invariant).
 // SPADEN_RES=fixed: beta pass (memset / scale) + the 16-lane kernel (ablation).
+// `any`: whether a kernel of this SpMV call has been launched already; a
+// kernel may use programmatic dependent launch only after one (the first
+// kernel of a call must wait for everything before it on the stream).
 static cudaError_t residual_part(const Matrix &A, const ResPart &P, bool binned, float alpha, const float *x,
-                                 float beta, float *y, cudaStream_t st) {
+                                 float beta, float *y, cudaStream_t st, int slot, bool &any) {
     cudaError_t e = cudaSuccess;
     if (binned) {
         // the last class (empty / long rows) only scales y: skipped when beta = 1
         const int64_t nc = P.bins.cta_start[beta == 1.f ? kResClasses : kResClasses + 1];
         if (nc > 0) {
+            any = true;
             if (A.storage == SPADEN_R_16F)
                 e = launch_k(false, k_residual_binned<__half>, dim3((unsigned)nc), dim3(256), 0, st, P.bins,
                              (const int32_t *)P.perm, (const int32_t *)P.rowptr, (const int32_t *)P.colidx,
@@ -700,6 +705,7 @@ static cudaError_t residual_part(const Matrix &A, const ResPart &P, bool binned,
                              (const float *)P.values, x, alpha, beta, y);
         }
     } else {
+        any = any || beta != 1.f || P.nnz > 0;
         if (beta == 0.f) e = cudaMemsetAsync(y, 0, sizeof(float) * (size_t)A.m, st);
         else if (beta != 1.f)
             k_scale<<<(unsigned)std::min<int64_t>((A.m + 255) / 256, 148 * 16), 256, 0, st>>>(A.m, beta, y);
@@ -716,20 +722,24 @@ static cudaError_t residual_part(const Matrix &A, const ResPart &P, bool binned,
     if (e == cudaSuccess && P.n_long > 0) {
         const unsigned gc = (unsigned)((32 * P.n_chunks + 255) / 256);
         const bool fused = P.n_chunks <= fused_fixup_max();
+        const bool dep = any;  // PDL only behind a kernel of this call
+        any = true;
+        float *carry = P.carry + (size_t)slot * (size_t)std::max<int64_t>(1, P.n_chunks);
+        int32_t *done = P.done + (size_t)slot * (size_t)P.n_long;
         if (A.storage == SPADEN_R_16F)
-            e = launch_k(true, fused ? k_res_chunks<__half, true> : k_res_chunks<__half, false>, dim3(gc), dim3(256),
+            e = launch_k(dep, fused ? k_res_chunks<__half, true> : k_res_chunks<__half, false>, dim3(gc), dim3(256),
                          0, st, (int64_t)P.n_chunks, (const int32_t *)P.long_rows, (const int32_t *)P.chunk_start,
                          (const int32_t *)P.chunk_row, (const int32_t *)P.rowptr, (const int32_t *)P.colidx,
-                         (const __half *)P.values, x, P.carry, P.done, alpha, y);
+                         (const __half *)P.values, x, carry, done, alpha, y);
         else
-            e = launch_k(true, fused ? k_res_chunks<float, true> : k_res_chunks<float, false>, dim3(gc), dim3(256),
+            e = launch_k(dep, fused ? k_res_chunks<float, true> : k_res_chunks<float, false>, dim3(gc), dim3(256),
                          0, st, (int64_t)P.n_chunks, (const int32_t *)P.long_rows, (const int32_t *)P.chunk_start,
                          (const int32_t *)P.chunk_row, (const int32_t *)P.rowptr, (const int32_t *)P.colidx,
-                         (const float *)P.values, x, P.carry, P.done, alpha, y);
+                         (const float *)P.values, x, carry, done, alpha, y);
         if (e == cudaSuccess && !fused)
             e = launch_k(true, k_res_fixup, dim3((unsigned)((32 * P.n_long + 255) / 256)), dim3(256), 0, st,
                          (int64_t)P.n_long, (const int32_t *)P.long_rows, (const int32_t *)P.chunk_start,
-                         (const float *)P.carry, alpha, y);
+                         (const float *)carry, alpha, y);
     }
     return e;
 }
@@ -739,12 +749,16 @@ bool residual_binned_enabled(const Matrix &A) {
     return A.n_res_parts > 0 && A.res[0].perm && !(env && env[0] == 'f');
 }
 
-cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st) {
+cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st,
+                           int slot, bool *launched) {
+    *launched = false;
     if (A.m == 0 || A.n_res_parts == 0) return cudaSuccess;
     const bool binned = residual_binned_enabled(A);
     cudaError_t e = cudaSuccess;
+    bool any = false;
     for (int q = 0; q < A.n_res_parts && e == cudaSuccess; ++q)
-        e = residual_part(A, A.res[q], binned, alpha, x, q == 0 ? beta : 1.f, y, st);
+        e = residual_part(A, A.res[q], binned, alpha, x, q == 0 ? beta : 1.f, y, st, slot, any);
+    *launched = any;
     if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }

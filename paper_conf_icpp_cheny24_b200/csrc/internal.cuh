@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 #include <cuda_fp16.h>
 #include <stdint.h>
+#include <atomic>
 #include <string>
 
 #include "spaden.h"
@@ -34,12 +35,18 @@ struct spaden_matrix_s {
     int64_t n_long = 0;                        // block-rows too large for a tile
     int tile_cfg = 0;                          // spaden::tile_cfg index the schedule was built for
     struct spaden_tile_desc_s *tiles = nullptr; // [n_tiles] (spaden::TileDesc)
+    uint8_t *rot = nullptr;                    // [Bnnz] per-block row rotation of the slot decode (bank
+                                               // conflicts, schedule.cu) or NULL (no rotation)
     int32_t *long_rows = nullptr;              // [n_long]
     int64_t n_chunks = 0;                      // kLongChunk-block chunks of the long rows
     int32_t *chunk_start = nullptr;            // [n_long+1] first chunk of each long row
     int32_t *chunk_row = nullptr;              // [n_chunks] index into long_rows
-    float *carry = nullptr;                    // [n_chunks*8] per-chunk row partials
-    int32_t *chunk_done = nullptr;             // [n_long] chunks finished per long row (0 between calls)
+    float *carry = nullptr;                    // [kScratchSlots][n_chunks*8] per-chunk row partials
+    int32_t *chunk_done = nullptr;             // [kScratchSlots][n_long] chunks finished per long row (0 between calls)
+    // long-row scratch: one of kScratchSlots sets per spmv call (round robin), so
+    // up to kScratchSlots calls on one handle may run concurrently on different streams
+    static constexpr int kScratchSlots = 4;
+    mutable std::atomic<uint32_t> scratch_next{0};
 
     // SpMM schedules for K = 2, 4 right-hand sides (index 0, 1; built lazily by spaden_spmm)
     struct spaden_tile_desc_s *spmm_tiles[3] = {};
@@ -64,8 +71,8 @@ struct spaden_matrix_s {
         int32_t *long_rows = nullptr;        // [n_long]
         int32_t *chunk_start = nullptr;      // [n_long+1]
         int32_t *chunk_row = nullptr;        // [n_chunks] index into long_rows
-        float *carry = nullptr;              // [n_chunks]
-        int32_t *done = nullptr;             // [n_long] chunks finished per long row (0 between calls)
+        float *carry = nullptr;              // [kScratchSlots][n_chunks]
+        int32_t *done = nullptr;             // [kScratchSlots][n_long] chunks finished per long row (0 between calls)
         int32_t *perm = nullptr;             // all rows, grouped by length class (then empty / long rows)
         ResBins bins = {};
     };
@@ -112,32 +119,30 @@ enum : uint32_t {
 // stage including the 16-byte alignment slack of its regions.
 struct TileCfg {
     int ctas_per_sm, consumers, stages, stage_bytes;
-    int warp_mode;  // 0: CTA pipeline (producer warp + consumers share stages)
-                    // 1: warp pipelines (each warp streams its own tiles; consumers = warps/CTA)
 };
 constexpr int kMaxStages = 8;
-constexpr int kNumTileCfgs = 17;
+// the launch shapes k_spmv_tiled is instantiated for (SPADEN_TILE_CFG selects one;
+// every stage holds a block-row of kLongRowBytes plus kStageSlack)
+inline bool tile_cfg_valid(int i) {
+    switch (i) {
+    case 1: case 2: case 3: case 5: case 6: case 7: case 10: case 14: case 15: case 16: return true;
+    default: return false;
+    }
+}
 __host__ __device__ inline TileCfg tile_cfg(int i) {
     switch (i) {
-    case 1: return TileCfg{2, 16, 3, 36 * 1024, 0};
-    case 2: return TileCfg{3, 8, 3, 24 * 1024, 0};
-    case 3: return TileCfg{4, 8, 2, 27 * 1024, 0};
-    case 4: return TileCfg{3, 4, 2, 9 * 1024, 1};
-    case 5: return TileCfg{3, 8, 4, 18 * 1024, 0};
-    case 6: return TileCfg{2, 16, 6, 18 * 1024, 0};
-    case 7: return TileCfg{4, 8, 3, 18 * 1024, 0};
-    case 8: return TileCfg{4, 8, 3, 9 * 1024, 0};
-    case 9: return TileCfg{4, 8, 4, 6 * 1024, 0};
+    case 1: return TileCfg{2, 16, 3, 36 * 1024};
+    case 3: return TileCfg{4, 8, 2, 27 * 1024};
+    case 5: return TileCfg{3, 8, 4, 18 * 1024};
+    case 6: return TileCfg{2, 16, 6, 18 * 1024};
+    case 7: return TileCfg{4, 8, 3, 18 * 1024};
     // 4 consumer warps per CTA: half the warps share (and wait on) each tile
-    case 10: return TileCfg{6, 4, 2, 18 * 1024, 0};
-    case 11: return TileCfg{5, 4, 3, 14 * 1024, 0};
-    case 12: return TileCfg{4, 4, 3, 18 * 1024, 0};
-    case 13: return TileCfg{6, 4, 3, 12 * 1024, 0};
+    case 10: return TileCfg{6, 4, 2, 18 * 1024};
     // 2 CTAs per SM, deeper rings (4 stages)
-    case 14: return TileCfg{2, 12, 4, 24 * 1024, 0};
-    case 15: return TileCfg{2, 16, 4, 27 * 1024, 0};
-    case 16: return TileCfg{2, 8, 4, 27 * 1024, 0};
-    default: return TileCfg{1, 16, 3, 64 * 1024, 0};
+    case 14: return TileCfg{2, 12, 4, 24 * 1024};
+    case 15: return TileCfg{2, 16, 4, 27 * 1024};
+    case 16: return TileCfg{2, 8, 4, 27 * 1024};
+    default: return TileCfg{3, 8, 3, 24 * 1024};  // cfg 2
     }
 }
 int default_tile_cfg(int64_t format_bytes, int value_bytes);  // SPADEN_TILE_CFG override, else by matrix size
@@ -147,6 +152,16 @@ constexpr int kSmallTileCfg = 5;  // measured L2-flushed: fem62k
 // shared-memory bytes a block occupies in a stage: bitmap 8 + blk_col 4 +
 // blk_offset 4 (copied) + 8 fp32 row partials at a 9-word stride (scratch)
 constexpr int kBlockStageBytes = 16 + 36;
+// + 1 byte per block when the schedule carries row rotations (the rotation region);
+// the long-row cost (kLongRowBytes) is computed with kBlockStageBytes alone
+constexpr int kBlockRotBytes = 1;
+// A block-row whose stage cost (kBlockStageBytes per block + its values + 4)
+// exceeds kLongRowBytes is "long" (chunk path) whatever the tile config: the
+// split between the tile path and the chunk path -- two different summation
+// orders -- is then a function of the block-row alone, so y is bitwise the
+// same for every 8-row-aligned partition (slices of different sizes pick
+// different tile configs).  Every tile config holds such a row in one stage.
+constexpr int64_t kLongRowBytes = 9 * 1024;
 // long block-rows are split into chunks of this many blocks (relative to the
 // block-row start, so the split depends only on the row itself)
 #ifndef SPADEN_LONG_CHUNK
@@ -219,13 +234,21 @@ struct PeerOut {
 // converter (convert.cu)
 spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *rowptr,
                             const int32_t *colidx, const void *values, spaden_dtype_t vdt,
-                            spaden_dtype_t sdt, int residual_max_popc, cudaStream_t stream, Matrix *A);
+                            spaden_dtype_t sdt, int residual_max_popc, float auto_mean_fill,
+                            cudaStream_t stream, Matrix *A, bool count_only = false);
 
 // hybrid split (hybrid.cu): move blocks with popc <= t into a CSR residual
 spaden_status_t split_residual(Matrix *A, int t, cudaStream_t stream);
 // hybrid SpMV, first part: y = beta*y + alpha*A_res*x on every row (y not read
 // when beta = 0); the bitBSR kernels follow with beta = 1
-cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t stream);
+// (*launched: whether it launched any kernel -- later kernels of the call use
+// programmatic dependent launch only then)
+cudaError_t residual_first(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t stream,
+                           int slot, bool *launched);
+// scratch set of one spmv call (Matrix::kScratchSlots round robin)
+inline int pick_scratch(const Matrix &A) {
+    return (int)(A.scratch_next.fetch_add(1u, std::memory_order_relaxed) % (uint32_t)Matrix::kScratchSlots);
+}
 bool residual_binned_enabled(const Matrix &A);  // binned residual kernel (not the SPADEN_RES=fixed ablation)
 
 // SpMV (spmv.cu)

@@ -94,6 +94,101 @@ __global__ void k_pack(int64_t Bnrow, const int32_t *__restrict__ brp, const int
     }
 }
 
+// ---------------------------------------------------------------------------
+// Row rotations of the slot decode (bank conflicts).  The tiled kernel decodes a
+// 32-block unit with one lane per block and one predicated shared-memory load
+// per bit slot: instruction i = 8t + c reads, in every lane whose block has that
+// bit, the block's value at its popcount rank.  Lanes whose values sit in the
+// same bank at different words serialise (one wavefront per distinct word).  A
+// lane may walk its block's rows in any cyclic order -- row (t + rho) & 7 at
+// step t -- without changing any row's own fma order, so y is bitwise the same
+// for every rho.  This pass picks rho per block greedily, lanes in order: for
+// each lane the rotation that adds the fewest wavefronts given the lanes before
+// it (a warp per tile; lanes evaluate the 8 rotations x 64 slots in parallel,
+// per-(instruction, bank) word counts in shared memory).  Banks are taken
+// relative to the tile's value region, which the kernel copies from a 16-byte
+// aligned start (a constant bank shift per tile, invisible to the conflicts).
+constexpr int kRotWarps = 8;
+
+template <int SV>
+__global__ void __launch_bounds__(32 * kRotWarps)
+k_rot_greedy(const TileDesc *__restrict__ tiles, int ntiles, const uint64_t *__restrict__ bitmap,
+             const int32_t *__restrict__ blk_offset, uint8_t *__restrict__ rot) {
+    __shared__ uint8_t load[kRotWarps][64][32];  // words per (slot instruction, bank) so far
+    __shared__ uint8_t mx[kRotWarps][64];        // max over banks = wavefronts of the instruction
+    __shared__ uint8_t sload[kRotWarps][8][32];  // the 8 partial stores (step t -> row (t+rho)&7)
+    __shared__ uint8_t smx[kRotWarps][8];
+    const int w = threadIdx.x >> 5, j = threadIdx.x & 31;
+    const int t = blockIdx.x * kRotWarps + w;
+    if (t >= ntiles) return;
+    const int b0 = tiles[t].b0, b1 = tiles[t].b1;
+    uint32_t *lw = reinterpret_cast<uint32_t *>(&load[w][0][0]);
+    const int r = j & 7;
+    for (int ub = b0; ub < b1; ub += 32) {
+        for (int q = j; q < 64 * 32 / 4; q += 32) lw[q] = 0u;
+        for (int q = j; q < 8 * 32 / 4; q += 32) reinterpret_cast<uint32_t *>(&sload[w][0][0])[q] = 0u;
+        if (j < 16) reinterpret_cast<uint32_t *>(&mx[w][0])[j] = 0u;
+        if (j < 2) reinterpret_cast<uint32_t *>(&smx[w][0])[j] = 0u;
+        __syncwarp();
+        const int nbu = min(32, b1 - ub);
+        for (int l = 0; l < nbu; ++l) {
+            const uint64_t bm = __ldg(bitmap + ub + l);
+            const int off = __ldg(blk_offset + ub + l);
+            int delta = 0;
+#pragma unroll 4
+            for (int k = 0; k < 16; ++k) {
+                const int sl = (j >> 3) + 4 * k;
+                if ((bm >> sl) & 1ull) {
+                    const int rank = __popcll(bm & ((1ull << sl) - 1ull));
+                    const int bank = (int)((((int64_t)off + rank) * SV) >> 2) & 31;
+                    const int ins = 8 * (((sl >> 3) - r) & 7) + (sl & 7);
+                    delta += (load[w][ins][bank] + 1 > mx[w][ins]) ? 1 : 0;
+                }
+            }
+            // the block's partial stores: step t writes row (t + r) & 7 at word
+            // 9 * lane + row of the unit's scratch (kPartStride = 36 bytes)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int tt = 2 * (j >> 3) + h;
+                const int bank = (9 * l + ((tt + r) & 7)) & 31;
+                delta += (sload[w][tt][bank] + 1 > smx[w][tt]) ? 1 : 0;
+            }
+            delta += __shfl_xor_sync(0xffffffffu, delta, 8);
+            delta += __shfl_xor_sync(0xffffffffu, delta, 16);
+            int key = delta * 8 + r;  // fewest added wavefronts, then the smallest rotation
+            key = min(key, __shfl_xor_sync(0xffffffffu, key, 1));
+            key = min(key, __shfl_xor_sync(0xffffffffu, key, 2));
+            key = min(key, __shfl_xor_sync(0xffffffffu, key, 4));
+            const int best = key & 7;
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {  // lane j commits slots j and j + 32 (distinct instructions)
+                const int sl = j + 32 * h;
+                if ((bm >> sl) & 1ull) {
+                    const int rank = __popcll(bm & ((1ull << sl) - 1ull));
+                    const int bank = (int)((((int64_t)off + rank) * SV) >> 2) & 31;
+                    const int ins = 8 * (((sl >> 3) - best) & 7) + (sl & 7);
+                    const int nl = load[w][ins][bank] + 1;
+                    load[w][ins][bank] = (uint8_t)nl;
+                    if (nl > mx[w][ins]) mx[w][ins] = (uint8_t)nl;
+                }
+            }
+            if (j < 8) {
+                const int bank = (9 * l + ((j + best) & 7)) & 31;
+                const int nl = sload[w][j][bank] + 1;
+                sload[w][j][bank] = (uint8_t)nl;
+                if (nl > smx[w][j]) smx[w][j] = (uint8_t)nl;
+            }
+            if (j == 0) rot[ub + l] = (uint8_t)best;
+            __syncwarp();
+        }
+    }
+}
+
+bool rotation_enabled() {  // SPADEN_ROT=0 disables (A/B, tests), read per conversion
+    const char *e = getenv("SPADEN_ROT");
+    return !(e && e[0] == '0');
+}
+
 __global__ void k_long_chunks(int nlong, const int32_t *__restrict__ long_rows, const int32_t *__restrict__ brp,
                               int32_t *__restrict__ cnt) {
     const int j = blockIdx.x * blockDim.x + threadIdx.x;
@@ -120,7 +215,7 @@ int default_tile_cfg(int64_t format_bytes, int value_bytes) {
     const char *e = getenv("SPADEN_TILE_CFG");
     if (e && e[0] >= '0' && e[0] <= '9') {
         const int c = atoi(e);
-        if (c >= 0 && c < kNumTileCfgs) return c;
+        if (tile_cfg_valid(c)) return c;
     }
     // measured best on fem1p5m: fp32 values 3 CTAs/SM x 8 consumers
     // x 3 x 24 KB, fp16 values 2 x 16 x 4 x 27 KB; small matrices need smaller stages to
@@ -136,12 +231,22 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     const int sv_b = A->storage == SPADEN_R_16F ? 2 : 4;
     A->tile_cfg = default_tile_cfg(4 * (A->Bnrow + 1) + 16 * A->Bnnz + (int64_t)sv_b * A->nnz, sv_b);
     const TileCfg cfg = tile_cfg(A->tile_cfg);
-    const int64_t cap = cfg.stage_bytes - kStageSlack;
-    // CTA pipelines: rows above half a stage are long (keeps tiles well packed);
-    // warp pipelines: any row that fits a stage alone stays in the tiles
-    const int64_t long_cost = cfg.warp_mode ? cap : cfg.stage_bytes / 2;
+    const int64_t stage_cap = cfg.stage_bytes - kStageSlack;
+    // long rows: one constant for every config (partition invariance, internal.cuh);
+    const int64_t long_cost = kLongRowBytes;
+    const int64_t cap = stage_cap;
+    if (stage_cap < long_cost) {
+        set_error("tile config stage smaller than the long-row threshold");
+        return SPADEN_ERR_UNSUPPORTED;
+    }
     const bool hyb = A->res_max_popc > 0;  // hybrid: tiles skip block-rows without blocks
     if (Bnrow == 0) return SPADEN_OK;
+    // row rotations: CTA-pipeline configs with the predicated-slot decode (mean
+    // block fill >= kSlotsMinFill, spmv.cu); one byte per block in the stage
+    const int64_t bit_nnz = A->nnz - A->res_nnz;
+    const bool use_rot = rotation_enabled() && A->Bnnz > 0 &&
+                         bit_nnz >= (int64_t)kSlotsMinFill * A->Bnnz;
+    const int pack_blk = kBlockStageBytes + (use_rot ? kBlockRotBytes : 0);
 
     const size_t n_tmp = scan_tmp_ints(nseg + 1);
     const size_t ints = 2 * (size_t)(nseg + 1) + n_tmp + 4;
@@ -150,7 +255,7 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     int32_t *seg_tiles = tmp, *seg_long = tmp + (nseg + 1), *scan_tmp = tmp + 2 * (nseg + 1);
     int32_t *summary = scan_tmp + n_tmp;
     const unsigned grid = (unsigned)((nseg + 127) / 128);
-    k_pack<false><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, kBlockStageBytes,
+    k_pack<false><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, pack_blk,
                                         hyb, nullptr, seg_tiles, seg_long, nullptr, nullptr, nullptr, nullptr);
     cudaError_t e = exclusive_scan_i32(seg_tiles, seg_tiles, nseg, scan_tmp, st);
     if (e == cudaSuccess) e = exclusive_scan_i32(seg_long, seg_long, nseg, scan_tmp, st);
@@ -175,11 +280,25 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
         return cuda_status(e, "allocating SpMV schedule");
     }
     A->aux_bytes = (int64_t)(tile_bytes + long_bytes);
-    k_pack<true><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, kBlockStageBytes,
+    k_pack<true><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, pack_blk,
                                        hyb, nullptr, nullptr, nullptr, seg_tiles, seg_long, A->tiles, A->long_rows);
     e = cudaGetLastError();
     cudaFreeAsync(tmp, st);
     if (e != cudaSuccess) return cuda_status(e, "packing SpMV schedule");
+    if (use_rot && A->n_tiles > 0 && A->Bnnz > 0) {  // bank-conflict row rotations (slot decode)
+        e = cudaMalloc(&A->rot, pad16((size_t)A->Bnnz));
+        if (e == cudaSuccess) e = cudaMemsetAsync(A->rot, 0, pad16((size_t)A->Bnnz), st);
+        if (e == cudaSuccess) {
+            const unsigned g = (unsigned)((A->n_tiles + kRotWarps - 1) / kRotWarps);
+            if (sv == 2)
+                k_rot_greedy<2><<<g, 32 * kRotWarps, 0, st>>>(A->tiles, (int)A->n_tiles, A->bitmap, A->blk_offset, A->rot);
+            else
+                k_rot_greedy<4><<<g, 32 * kRotWarps, 0, st>>>(A->tiles, (int)A->n_tiles, A->bitmap, A->blk_offset, A->rot);
+            e = cudaGetLastError();
+        }
+        if (e != cudaSuccess) return cuda_status(e, "row-rotation schedule");
+        A->aux_bytes += (int64_t)pad16((size_t)A->Bnnz);
+    }
     if (A->n_long == 0) return SPADEN_OK;
 
     // long block-rows -> fixed kLongChunk-block chunks (+ carry slots)
@@ -200,15 +319,16 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
         A->n_chunks = nch;
         e = cudaMalloc(&A->chunk_row, sizeof(int32_t) * std::max(1, nch));
     }
-    if (e == cudaSuccess) e = cudaMalloc(&A->carry, sizeof(float) * 8 * std::max(1, nch));
-    if (e == cudaSuccess) e = cudaMalloc(&A->chunk_done, sizeof(int32_t) * nl);
-    if (e == cudaSuccess) e = cudaMemsetAsync(A->chunk_done, 0, sizeof(int32_t) * nl, st);
+    constexpr int SL = Matrix::kScratchSlots;
+    if (e == cudaSuccess) e = cudaMalloc(&A->carry, sizeof(float) * 8 * std::max(1, nch) * SL);
+    if (e == cudaSuccess) e = cudaMalloc(&A->chunk_done, sizeof(int32_t) * nl * SL);
+    if (e == cudaSuccess) e = cudaMemsetAsync(A->chunk_done, 0, sizeof(int32_t) * nl * SL, st);
     if (e == cudaSuccess) {
         k_chunk_rows<<<(nl + 255) / 256, 256, 0, st>>>(nl, A->chunk_start, A->chunk_row);
         e = cudaGetLastError();
     }
     if (e != cudaSuccess) return cuda_status(e, "long-row chunk schedule");
-    A->aux_bytes += (int64_t)sizeof(int32_t) * (2 * nl + 1 + nch) + (int64_t)sizeof(float) * 8 * nch;
+    A->aux_bytes += (int64_t)sizeof(int32_t) * (2 * nl + 1 + nch) + (int64_t)(sizeof(float) * 8 * nch + 4 * nl) * SL;
     return SPADEN_OK;
 }
 
@@ -221,12 +341,12 @@ spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t st)
     const int sv = A->storage == SPADEN_R_16F ? 2 : 4;
     const TileCfg cfg = tile_cfg(A->tile_cfg);
     const int64_t cap = cfg.stage_bytes - kStageSlack;
-    const int64_t long_cost = cfg.warp_mode ? cap : cfg.stage_bytes / 2;
+    const int64_t long_cost = kLongRowBytes;  // same long-row set as the SpMV schedule
     const int pack_bytes = 16 + 4 * (8 * K + 1);
     const bool hyb = A->res_max_popc > 0;
     const int64_t nseg = (Bnrow + kSeg - 1) / kSeg;
     A->spmm_state[kidx] = -1;
-    if (Bnrow == 0 || cfg.warp_mode) return SPADEN_ERR_UNSUPPORTED;
+    if (Bnrow == 0) return SPADEN_ERR_UNSUPPORTED;
     const size_t n_tmp = scan_tmp_ints(nseg + 1);
     int32_t *tmp = nullptr;
     SPADEN_CUDA_TRY(cudaMallocAsync(&tmp, (2 * (size_t)(nseg + 1) + n_tmp + 8) * sizeof(int32_t), st));

@@ -1,11 +1,8 @@
 // spmv.cu -- y = alpha*A*x + beta*y over bitBSR on sm_100a CUDA cores
 // (§4.3).
 //
-// Two kernels:
-//   k_spmv_tiled  (default)  persistent CTAs fed by a TMA bulk-copy pipeline;
-//   k_spmv_v0     (SPADEN_KERNEL=v0) the first, simple row-byte kernel, kept as
-//                 the measured baseline of DESIGN.md.
-// and k_spmv_long_chunks (chunks + fused fix-up) for block-rows too large for a
+// k_spmv_tiled: persistent CTAs fed by a TMA bulk-copy pipeline, and
+// k_spmv_long_chunks (chunks + fused fix-up) for block-rows too large for a
 // pipeline stage.
 //
 // Decode (both kernels follow PAPER.md §4.3.1 / Alg. 2 semantics):
@@ -32,59 +29,6 @@ template <typename V> __device__ __forceinline__ float ldv(const V *p);
 template <> __device__ __forceinline__ float ldv<float>(const float *p) { return __ldg(p); }
 template <> __device__ __forceinline__ float ldv<__half>(const __half *p) {
     return __half2float(__ldg(p));
-}
-
-// ==========================================================================
-// v0: one warp per block-row; 8 lanes per block (lane r = row r = bitmap byte
-// r), four blocks per warp step; 8 predicated bit slots per lane.
-// ==========================================================================
-template <typename V>
-__global__ void __launch_bounds__(256)
-k_spmv_v0(int64_t m, int64_t n, int64_t Bnrow, const int32_t *__restrict__ blk_rowptr,
-          const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
-          const int32_t *__restrict__ blk_offset, const V *__restrict__ vals,
-          const float *__restrict__ x, bool x_vec, float alpha, float beta, float *__restrict__ y) {
-    const int lane = threadIdx.x & 31;
-    const int g = lane >> 3, r = lane & 7;
-    const int64_t nwarps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t br = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); br < Bnrow;
-         br += nwarps) {
-        const int b0 = __ldg(blk_rowptr + br), b1 = __ldg(blk_rowptr + br + 1);
-        float acc = 0.f;
-        for (int b = b0 + g; b < b1; b += 4) {
-            const uint64_t bmp = __ldg(bitmap + b);
-            const int bc = __ldg(blk_col + b);
-            const int off = __ldg(blk_offset + b);
-            const uint32_t byte = (uint32_t)(bmp >> (8 * r)) & 0xffu;
-            int p = off + __popcll(bmp & ((1ull << (8 * r)) - 1ull));
-            const float *xs = x + 8 * (int64_t)bc;
-            float xv[8];
-            if (x_vec && 8 * (int64_t)bc + 8 <= n) {
-                const float4 lo = __ldg(reinterpret_cast<const float4 *>(xs));
-                const float4 hi = __ldg(reinterpret_cast<const float4 *>(xs) + 1);
-                xv[0] = lo.x; xv[1] = lo.y; xv[2] = lo.z; xv[3] = lo.w;
-                xv[4] = hi.x; xv[5] = hi.y; xv[6] = hi.z; xv[7] = hi.w;
-            } else {  // ragged last block column / unaligned x: read only referenced entries
-#pragma unroll
-                for (int c = 0; c < 8; ++c) xv[c] = ((byte >> c) & 1u) ? __ldg(xs + c) : 0.f;
-            }
-#pragma unroll
-            for (int c = 0; c < 8; ++c) {
-                if ((byte >> c) & 1u) {
-                    acc = fmaf(ldv<V>(vals + p), xv[c], acc);
-                    ++p;
-                }
-            }
-        }
-        acc += __shfl_xor_sync(kFull, acc, 8);
-        acc += __shfl_xor_sync(kFull, acc, 16);
-        const int64_t row = 8 * br + r;
-        if (g == 0 && row < m) {
-            float o = alpha * acc;
-            if (beta != 0.f) o = fmaf(beta, y[row], o);
-            y[row] = o;
-        }
-    }
 }
 
 // ==========================================================================
@@ -165,6 +109,11 @@ __device__ __forceinline__ int lds_i32(uint32_t a) {
 __device__ __forceinline__ float lds_f32(uint32_t a) {
     float v;
     asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u8(uint32_t a) {
+    unsigned short v;
+    asm("ld.shared.u8 %0, [%1];" : "=h"(v) : "r"(a));
     return v;
 }
 __device__ __forceinline__ float lds_f16(uint32_t a) {
@@ -260,18 +209,47 @@ __device__ __forceinline__ void block_slots_at(uint2 bm, typename VS::P pA, type
 #pragma unroll
         for (int c = 0; c < 8; ++c) {
             if ((byte >> c) & 1u) {
-#ifdef SPADEN_EXP_NOCONFLICT  // timing experiment only: conflict-free (wrong) addresses
-                if constexpr (sizeof(typename VS::P) == 4)
-                    a = fmaf(VS::get((pA & ~127u) + 4u * ((threadIdx.x + 8 * r + c) & 31u)), xs.v[c], a);
-                else
-                    a = fmaf(VS::get(p), xs.v[c], a);
-#else
                 a = fmaf(VS::get(p), xs.v[c], a);
-#endif
                 p += VS::step;
             }
         }
         acc[r] = a;
+    }
+}
+
+// Slot decode of one block walking its rows in the cyclic order rho, rho+1, ...
+// (rho from the schedule's bank-conflict pass, schedule.cu): step t decodes
+// original row (t + rho) & 7, whose values start at popcount rank
+// below(row) = (below_rot(t) + below(rho)) mod popc(bm).  Each row is still one
+// fma chain over its columns in ascending order, stored to its own partial
+// slot, so the result does not depend on rho.  Partials go to q + 4*row.
+template <class VS>
+__device__ __forceinline__ void block_slots_rot(uint2 bm, uint32_t rho, typename VS::P p0, const XSeg &xs,
+                                                uint32_t q) {
+    const uint64_t b = ((uint64_t)bm.y << 32) | bm.x;
+    const uint32_t sh = 8u * rho;
+    const uint64_t rb = sh ? ((b >> sh) | (b << (64u - sh))) : b;  // row t of rb = row (t+rho)&7 of b
+    const int P = __popcll(b);
+    const int B = __popcll(b & ((1ull << sh) - 1ull));             // values of rows < rho
+    const uint32_t rlo = (uint32_t)rb, rhi = (uint32_t)(rb >> 32);
+#pragma unroll
+    for (int t = 0; t < 8; ++t) {
+        const uint32_t w = t < 4 ? rlo : rhi;
+        const uint32_t byte = (w >> (8 * (t & 3))) & 0xffu;
+        int below = (t & 3) == 0 ? 0 : __popc(w & ((1u << (8 * (t & 3))) - 1u));
+        if (t >= 4) below += __popc(rlo);
+        int start = below + B;
+        start = start >= P ? start - P : start;  // rows of the wrapped part
+        typename VS::P p = p0 + start * VS::step;
+        float a = 0.f;
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+            if ((byte >> c) & 1u) {
+                a = fmaf(VS::get(p), xs.v[c], a);
+                p += VS::step;
+            }
+        }
+        sts_f32(q + 4u * ((uint32_t)(t + rho) & 7u), a);
     }
 }
 
@@ -523,34 +501,56 @@ __device__ __forceinline__ void mma_unit(int lb0, int nb, int lane, uint32_t a_b
 // per-stage tile header; the first 32 bytes are what every consumer warp needs
 // to decode (two 16-byte loads), the next 16 only the phase-2 warp
 struct alignas(16) StageHdr {
-    int v0, nb, units;                         // first value, blocks, 32-block units
+    int v0, nb;                                // first value, blocks
+    uint32_t a_rot;                            // shared address of the row-rotation bytes (ROT)
     uint32_t a_val;                            // shared address of the value slice
     uint32_t a_bmp, a_col, a_off, a_part;      // ... of bitmap / blk_col / blk_offset; row-partial scratch
     int br0, nbr, b0;                          // tile block-rows, first block (phase 2)
     uint32_t a_rp;                             // ... of the blk_rowptr slice
-    int u_next, done, pad0, pad1;              // next unit to grab, units done
 };
 
-// DEC: 0 = set-bit loop, 1 = 64 predicated slots per lane (lane = block),
-//      2 = 8 predicated slots per lane (lane = one row of a block, 4 blocks per
-//          warp step: value loads of a step stay inside 4 consecutive runs).
-template <typename V, int DEC, int CONSUMERS, int MINB, int K = 1>
+// DEC: 0 = set-bit loop, 1 = 64 predicated slots per lane (lane = block; with
+// ROT the rows in the schedule's bank-conflict rotation), 4 = tensor-core
+// ablation (fp16).
+//
+// Work split inside a CTA: the producer lane stages the CTA's tiles through an
+// S-stage ring; their 32-block units form one queue (numbered in tile order).
+// A consumer warp takes the next unit number from a shared counter, waits
+// until the producer has published the tile holding it (units_avail), finds
+// its stage by unit range, waits for the data (full mbarrier), decodes the
+// unit and counts it done on the stage; the warp that completes a tile runs
+// its phase 2 and alone releases the stage (empty mbarrier, one arrival).  A
+// warp therefore only touches the tiles it works on, and idle warps take the
+// units of tiles whose other warps are still busy.
+struct alignas(16) StageRange {
+    int ustart, uend;  // the stage's tile holds queue units [ustart, uend)
+    int parity, pad;   // full-barrier phase parity of that fill
+};
+
+template <typename V, int DEC, int CONSUMERS, int MINB, int K = 1, bool ROT = false>
 __global__ void __launch_bounds__(32 * (CONSUMERS + 1), MINB)
 k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int ntiles, const int32_t *__restrict__ blk_rowptr,
              const int32_t *__restrict__ blk_col, const uint64_t *__restrict__ bitmap,
              const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
              int nbc_vec, float alpha, float beta, float *__restrict__ y, int64_t ldx, int64_t ldy,
-             const PeerOut po, unsigned long long texx, int wait_y) {
+             const PeerOut po, unsigned long long texx, int wait_y, const uint8_t *__restrict__ rot) {
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t full_bar[kMaxStages], empty_bar[kMaxStages];
     __shared__ StageHdr hdr[kMaxStages];
+    __shared__ StageRange range[kMaxStages];
+    __shared__ int unit_done[kMaxStages];
+    __shared__ int unit_next, units_avail;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     pdl_trigger();
     if (threadIdx.x == 0) {
         for (int s = 0; s < stages; ++s) {
             mbar_init(smem_u32(&full_bar[s]), 1);
-            mbar_init(smem_u32(&empty_bar[s]), CONSUMERS);
+            mbar_init(smem_u32(&empty_bar[s]), 1);
+            range[s] = StageRange{0, 0, 0, 0};
+            unit_done[s] = 0;
         }
+        unit_next = 0;
+        units_avail = 0;
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -559,21 +559,25 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
     if (warp == 0) {  // ---------------------------------------------- producer
         if (lane == 0) {
             const uint64_t pol = policy_evict_first();
-            int i = 0, s = 0;
+            int i = 0, s = 0, U = 0;
             uint32_t ph = 0;
+            // tile descriptors are loaded one tile ahead (the load latency then
+            // overlaps the wait for a free stage)
+            int4 nd0 = make_int4(0, 0, 0, 0);
+            int2 nd1 = make_int2(0, 0);
+            if (blockIdx.x < ntiles) {
+                nd0 = __ldg(reinterpret_cast<const int4 *>(tiles + blockIdx.x));
+                nd1 = __ldg(reinterpret_cast<const int2 *>(tiles + blockIdx.x) + 2);
+            }
             for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++i, s = (s + 1 == stages) ? (ph ^= 1u, 0) : s + 1) {
-                const int4 d0 = __ldg(reinterpret_cast<const int4 *>(tiles + t));
-                const int4 d1 = __ldg(reinterpret_cast<const int4 *>(tiles + t) + 1);
+                const int4 d0 = nd0;
+                const int2 d1 = nd1;
+                if (t + (int)gridDim.x < ntiles) {
+                    nd0 = __ldg(reinterpret_cast<const int4 *>(tiles + t + gridDim.x));
+                    nd1 = __ldg(reinterpret_cast<const int2 *>(tiles + t + gridDim.x) + 2);
+                }
                 const int br0 = d0.x, br1 = d0.y, b0 = d0.z, b1 = d0.w, v0 = d1.x, v1 = d1.y;
                 if (i >= stages) mbar_wait(smem_u32(&empty_bar[s]), ph ^ 1u);
-#ifdef SPADEN_EXP_NOLOAD  // timing experiment: re-process the stage's first tile, no copies
-                if (i >= stages) {
-                    hdr[s].u_next = 0;
-                    hdr[s].done = 0;
-                    mbar_arrive(smem_u32(&full_bar[s]));
-                    continue;
-                }
-#endif
                 const uint32_t stage = sbase + (uint32_t)s * (uint32_t)stage_bytes;
                 uint32_t cur = stage;
                 struct Reg {
@@ -594,26 +598,34 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                 h.b0 = b0;
                 h.v0 = v0;
                 h.nb = b1 - b0;
-                h.units = max(1, (h.nb + 31) >> 5);
-                h.u_next = 0;
-                h.done = 0;
-                h.pad0 = h.pad1 = 0;
-                const Reg rs[5] = {region(bitmap + b0, 8u * (b1 - b0), &h.a_bmp),
+                h.a_rot = 0;
+                // the value slice first: its bank layout is the one the rotation
+                // pass assumed (16-byte aligned start of the stage)
+                const Reg rs[6] = {region(vals + v0, sizeof(V) * (size_t)(v1 - v0), &h.a_val),
+                                   region(bitmap + b0, 8u * (b1 - b0), &h.a_bmp),
                                    region(blk_col + b0, 4u * (b1 - b0), &h.a_col),
                                    region(blk_offset + b0, 4u * (b1 - b0), &h.a_off),
                                    region(blk_rowptr + br0, 4u * (br1 - br0 + 1), &h.a_rp),
-                                   region(vals + v0, sizeof(V) * (size_t)(v1 - v0), &h.a_val)};
+                                   ROT ? region(rot + b0, (size_t)(b1 - b0), &h.a_rot) : Reg{0, 0u}};
                 const uint32_t bytes = cur - stage;
                 h.a_part = cur;  // kPartStride bytes of row partials per block (not copied)
                 hdr[s] = h;
+                const int units = max(1, (h.nb + 31) >> 5);
+                asm volatile("st.shared.v4.s32 [%0], {%1, %2, %3, %4};" ::"r"(smem_u32(&range[s])), "r"(U),
+                             "r"(U + units), "r"((int)ph), "r"(0)
+                             : "memory");  // one 16-byte store: consumers never see a torn range
+                unit_done[s] = 0;
+                U += units;
                 const uint32_t fb = smem_u32(&full_bar[s]);
                 mbar_arrive_expect_tx(fb, bytes);
                 uint32_t dst = stage;
 #pragma unroll
-                for (int k = 0; k < 5; ++k) {
+                for (int k = 0; k < 6; ++k) {
                     if (rs[k].sz) bulk_g2s(dst, (const void *)rs[k].src, rs[k].sz, fb, pol);
                     dst += rs[k].sz;
                 }
+                // publish the tile's units (after its header, range and counter)
+                asm volatile("st.release.cta.shared.s32 [%0], %1;" ::"r"(smem_u32(&units_avail)), "r"(U) : "memory");
             }
         }
         pdl_wait();  // a PDL-launched grid completes only after its predecessor
@@ -621,279 +633,110 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
     }
 
     // ------------------------------------------------------------ consumers
-    int s = 0;
-    uint32_t ph = 0;
-    // shared addresses of stage 0's barriers / header, hoisted out of the tile loop
-    const uint32_t a_full0 = smem_u32(&full_bar[0]), a_empty0 = smem_u32(&empty_bar[0]);
-    const uint32_t a_hdr0 = smem_u32(&hdr[0]);
-    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, s = (s + 1 == stages) ? (ph ^= 1u, 0) : s + 1) {
+    // the CTA's unit count (its tiles t = blockIdx.x + k*gridDim.x)
+    int total = 0;
+    for (int t = blockIdx.x + lane * gridDim.x; t < ntiles; t += 32 * gridDim.x) {
+        const int2 bb = __ldg(reinterpret_cast<const int2 *>(tiles + t) + 1);  // b0, b1
+        total += max(1, (bb.y - bb.x + 31) >> 5);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) total += __shfl_xor_sync(kFull, total, o);
+    const uint32_t a_avail = smem_u32(&units_avail), a_unext = smem_u32(&unit_next);
+    const uint32_t a_range0 = smem_u32(&range[0]), a_full0 = smem_u32(&full_bar[0]);
+    const uint32_t a_hdr0 = smem_u32(&hdr[0]), a_done0 = smem_u32(&unit_done[0]);
+    int avail = 0;
+    while (true) {
+        int g = 0;
+        if (lane == 0) g = atom_add_shared(a_unext, 1);
+        g = __shfl_sync(kFull, g, 0);
+        if (g >= total) break;
+        while (avail <= g) {  // the producer has not published the tile yet
+            asm volatile("ld.acquire.cta.shared.s32 %0, [%1];" : "=r"(avail) : "r"(a_avail) : "memory");
+            if (avail <= g) __nanosleep(64);
+        }
+        int s = 0, us = 0, par = 0;
+        for (; s < stages; ++s) {  // the stage whose tile holds unit g (its current fill:
+            const int4 rg = lds_i4_volatile(a_range0 + 16u * s);  // a stage is refilled
+            if (rg.x <= g && g < rg.y) {                          // only after its tile is done)
+                us = rg.x;
+                par = rg.z;
+                break;
+            }
+        }
         const uint32_t a_hdr = a_hdr0 + (uint32_t)(s * sizeof(StageHdr));
-        mbar_wait(a_full0 + 8u * s, ph);
+        mbar_wait(a_full0 + 8u * s, (uint32_t)par);
         const int4 h0 = lds_i4_volatile(a_hdr);
         const int4 h1 = lds_i4_volatile(a_hdr + 16u);
-        const int v0 = h0.x, nb = h0.y, units = h0.z;
-        const uint32_t a_val = h0.w, a_bmp = h1.x, a_col = h1.y, a_off = h1.z, a_part = h1.w;
-        // units of 32 blocks are grabbed dynamically (shared counter per stage)
-        const uint32_t a_next = a_hdr + (uint32_t)offsetof(StageHdr, u_next);
-        int mine = 0;
-#ifdef SPADEN_EXP_NOCOMPUTE  // timing experiment: stream only
-        __syncwarp();
-        if (lane == 0) mbar_arrive(a_empty0 + 8u * s);
-        continue;
-#endif
-
-        while (true) {
-            int ul = 0;
-            if (lane == 0) ul = atom_add_shared(a_next, 1);
-            ul = __shfl_sync(kFull, ul, 0);
-            if (ul >= units) break;
-            ++mine;
-            if constexpr (K > 1) {  // SpMM: K right-hand sides
-                const int lb = ul * 32 + lane;
-                if (lb < nb) {
-                    const uint2 bm = lds_u2(a_bmp + 8u * lb);
-                    const int bc = lds_i32(a_col + 4u * lb);
-                    const uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
-                    const uint32_t cols = used_cols(bm);
-                    XSeg xs[K];
-#pragma unroll
-                    for (int j = 0; j < K; ++j) load_x(xs[j], x + j * ldx, bc, nbc_vec, cols, texx, (int)(j * ldx / 4));
-                    block_slots_k<SmemVals<V>, K>(bm, p, xs, a_part + 4u * (8 * K + 1) * lb);
-                }
-            } else if constexpr (DEC == 5 || DEC == 6) {
-                // LPB lanes per block (5: 4 lanes x 2 rows, 6: 2 lanes x 4 rows), 32/LPB
-                // consecutive blocks per step: a step's value loads stay inside fewer,
-                // contiguous runs (fewer bank conflicts, esp. for fp16)
-                constexpr int LPB = DEC == 5 ? 4 : 2, RPL = 8 / LPB, BPS = 32 / LPB;
-                const int g = lane / LPB, q = lane % LPB;
-                const int r0 = q * RPL;  // first row of this lane
-#pragma unroll 1
-                for (int st = 0; st < LPB; ++st) {
-                    const int lb = ul * 32 + st * BPS + g;
-                    if (lb < nb) {
-                        const uint2 bm = lds_u2(a_bmp + 8u * lb);
-                        const int bc = lds_i32(a_col + 4u * lb);
-                        const uint32_t p0 = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
-                        XSeg xs;
-                        load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
-                        const int plo = __popc(bm.x);
-#pragma unroll
-                        for (int rr = 0; rr < RPL; ++rr) {
-                            const int r = r0 + rr;  // not a compile-time constant: select by q
-                            const uint32_t w = r < 4 ? bm.x : bm.y;
-                            const int sh = 8 * (r & 3);
-                            const uint32_t byte = (w >> sh) & 0xffu;
-                            const int below = ((r & 3) == 0 ? 0 : __popc(w & ((1u << sh) - 1u))) + (r < 4 ? 0 : plo);
-                            uint32_t p = p0 + (uint32_t)below * (uint32_t)sizeof(V);
-                            float a = 0.f;
-#pragma unroll
-                            for (int c = 0; c < 8; ++c) {
-                                if ((byte >> c) & 1u) {
-                                    a = fmaf(SmemVals<V>::get(p), xs.v[c], a);
-                                    p += SmemVals<V>::step;
-                                }
-                            }
-                            sts_f32(a_part + kPartStride * lb + 4u * r, a);
-                        }
-                    }
-                }
-            } else if constexpr (DEC == 4) {
-                // tensor-core ablation (SURVEY.md §8(f) NEXT-3, fp16 values): the
-                // paper's fragment trick on mma.sync.m16n8k16 -- four
-                // blocks per MMA, block P/Q/R/S in the TL/TR/BL/BR quadrants, lane l
-                // owns bits 2l, 2l+1 of each (Alg. 2 mapping); x split
-                // into fp16 hi + lo parts (two MMAs) to keep ~22 bits of x.
-                mma_unit(ul * 32, nb, lane, a_bmp, a_col, a_off, a_val, v0, a_part, x, nbc_vec);
-            } else if constexpr (DEC == 2) {
-                const int g = lane >> 3, r = lane & 7;
-                const uint32_t mlo = r == 0 ? 0u : (r < 4 ? (1u << (8 * r)) - 1u : 0xffffffffu);
-                const uint32_t mhi = r <= 4 ? 0u : (1u << (8 * (r - 4))) - 1u;
-                const int sh = 8 * (r & 3);
-#pragma unroll 2
-                for (int st = 0; st < 8; ++st) {
-                    const int lb = ul * 32 + st * 4 + g;
-                    if (lb < nb) {
-                        const uint2 bm = lds_u2(a_bmp + 8u * lb);
-                        const int bc = lds_i32(a_col + 4u * lb);
-                        const uint32_t byte = ((r < 4 ? bm.x : bm.y) >> sh) & 0xffu;
-                        uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0 + __popc(bm.x & mlo) +
-                                                        __popc(bm.y & mhi)) *
-                                                 (uint32_t)sizeof(V);
-                        XSeg xs;
-                        load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
-                        float a = 0.f;
-#pragma unroll
-                        for (int c = 0; c < 8; ++c) {
-                            if ((byte >> c) & 1u) {
-                                a = fmaf(SmemVals<V>::get(p), xs.v[c], a);
-                                p += SmemVals<V>::step;
-                            }
-                        }
-                        sts_f32(a_part + kPartStride * lb + 4u * r, a);
-                    }
-                }
-            } else {
-                const int lb = ul * 32 + lane;
-                if (lb < nb) {  // phase 1: one block per lane
-                    const uint2 bm = lds_u2(a_bmp + 8u * lb);
-                    const int bc = lds_i32(a_col + 4u * lb);
-                    const uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
-                    float acc[8];
-                    const uint32_t q = a_part + kPartStride * lb;
-                    if constexpr (DEC == 1) {
-                        XSeg xs;
-                        load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
-                        const SwapHalves sw{sizeof(V) == 2 && ((lane >> 1) & 1)};
-                        const uint32_t plo = (uint32_t)__popc(bm.x) * (uint32_t)sizeof(V);
-                        block_slots_at<SmemVals<V>>(sw.bitmap(bm), sw.on ? p + plo : p, sw.on ? p : p + plo, xs, acc);
-#pragma unroll
-                        for (int r = 0; r < 8; ++r) sts_f32(q + sw.part_off(r), acc[r]);
-                    } else {
-                        block_bits<SmemVals<V>>(bm, p, x + 8 * (int64_t)bc, acc);
-#pragma unroll
-                        for (int r = 0; r < 8; ++r) sts_f32(q + 4u * r, acc[r]);
-                    }
-                }
-            }
-        }
-        if (mine) {
-            __syncwarp();
-            int last = 0;
-            if (lane == 0) {
-                __threadfence_block();
-                last = (atom_add_shared(a_hdr + (uint32_t)offsetof(StageHdr, done), mine) + mine == units);
-            }
-            if (__shfl_sync(kFull, last, 0)) {  // phase 2: this warp completed the tile
-                __threadfence_block();
-                if (wait_y) pdl_wait();  // y of the previous kernels (hybrid residual pass)
-                const int4 h2 = lds_i4_volatile(a_hdr + 32u);  // br0, nbr, b0, a_rp
-                if constexpr (K > 1)
-                    reduce_tile_k<K>((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, ldy);
-                else
-                    reduce_tile((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, po);
-            }
-        }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(a_empty0 + 8u * s);
-    }
-    pdl_wait();  // a PDL-launched grid completes only after its predecessor
-}
-
-// ==========================================================================
-// Warp-pipelined variant (TileCfg::warp_mode): every warp streams its own tiles
-// (tile t -> global warp t % total_warps) through a private S-stage ring of
-// shared memory: lane 0 issues the cp.async.bulk copies of tile k+S-1 into the
-// slot freed by tile k-1 and the warp waits on its own "full" mbarrier; phase 1
-// (lane per block, same decode) and phase 2 (same fixed-order block-row sums)
-// run inside the warp.  No cross-warp synchronisation at all.
-// ==========================================================================
-struct alignas(16) WarpHdr {
-    int br0, nbr, b0, v0, nb, pad0;
-    uint32_t a_bmp, a_col, a_off, a_rp, a_val, a_part;
-};
-
-template <typename V, int DEC, int WARPS, int S>
-__global__ void __launch_bounds__(32 * WARPS)
-k_spmv_warp(int stage_bytes, int64_t m, const TileDesc *__restrict__ tiles, int ntiles,
-            const int32_t *__restrict__ blk_rowptr, const int32_t *__restrict__ blk_col,
-            const uint64_t *__restrict__ bitmap, const int32_t *__restrict__ blk_offset,
-            const V *__restrict__ vals, const float *__restrict__ x, int nbc_vec, float alpha, float beta,
-            float *__restrict__ y) {
-    extern __shared__ __align__(128) unsigned char smem[];
-    __shared__ uint64_t full_bar[WARPS][S];
-    __shared__ WarpHdr hdr[WARPS][S];
-    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    if (lane == 0) {
-        for (int s = 0; s < S; ++s) mbar_init(smem_u32(&full_bar[w][s]), 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncwarp();
-    const uint32_t wbase = smem_u32(smem) + (uint32_t)(w * S) * (uint32_t)stage_bytes;
-    const int gw = blockIdx.x * WARPS + w, GW = gridDim.x * WARPS;
-    const uint64_t pol = policy_evict_first();
-
-    auto issue = [&](int k) {  // lane 0: tile gw + k*GW into slot k % S
-        const int t = gw + k * GW;
-        const int s = k % S;
-        const int4 d0 = __ldg(reinterpret_cast<const int4 *>(tiles + t));
-        const int4 d1 = __ldg(reinterpret_cast<const int4 *>(tiles + t) + 1);
-        const int br0 = d0.x, br1 = d0.y, b0 = d0.z, b1 = d0.w, v0 = d1.x, v1 = d1.y;
-        uint32_t cur = wbase + (uint32_t)s * (uint32_t)stage_bytes;
-        const uint32_t stage = cur;
-        struct Reg {
-            uintptr_t src;
-            uint32_t sz;
-        };
-        auto region = [&](const void *lo_p, size_t len, uint32_t *addr_out) {
-            const uintptr_t lo = (uintptr_t)lo_p, hi = lo + len;
-            const uintptr_t alo = lo & ~(uintptr_t)15, ahi = (hi + 15) & ~(uintptr_t)15;
-            *addr_out = cur + (uint32_t)(lo - alo);
-            const Reg r{alo, len > 0 ? (uint32_t)(ahi - alo) : 0u};
-            cur += r.sz;
-            return r;
-        };
-        WarpHdr h;
-        h.br0 = br0;
-        h.nbr = br1 - br0;
-        h.b0 = b0;
-        h.v0 = v0;
-        h.nb = b1 - b0;
-        h.pad0 = 0;
-        const Reg rs[5] = {region(bitmap + b0, 8u * (b1 - b0), &h.a_bmp),
-                           region(blk_col + b0, 4u * (b1 - b0), &h.a_col),
-                           region(blk_offset + b0, 4u * (b1 - b0), &h.a_off),
-                           region(blk_rowptr + br0, 4u * (br1 - br0 + 1), &h.a_rp),
-                           region(vals + v0, sizeof(V) * (size_t)(v1 - v0), &h.a_val)};
-        h.a_part = cur;
-        hdr[w][s] = h;
-        const uint32_t fb = smem_u32(&full_bar[w][s]);
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // prior generic reads of the slot
-        mbar_arrive_expect_tx(fb, cur - stage);
-        uint32_t dst = stage;
-#pragma unroll
-        for (int q = 0; q < 5; ++q) {
-            if (rs[q].sz) bulk_g2s(dst, (const void *)rs[q].src, rs[q].sz, fb, pol);
-            dst += rs[q].sz;
-        }
-    };
-
-    const int my_tiles = gw < ntiles ? (ntiles - gw + GW - 1) / GW : 0;
-    if (lane == 0)
-        for (int k = 0; k < S - 1 && k < my_tiles; ++k) issue(k);
-    for (int k = 0; k < my_tiles; ++k) {
-        if (lane == 0 && k + S - 1 < my_tiles) issue(k + S - 1);
-        const int s = k % S;
-        mbar_wait(smem_u32(&full_bar[w][s]), (uint32_t)(k / S) & 1u);
-        __syncwarp();
-        const int4 h0 = lds_i4_volatile(smem_u32(&hdr[w][s].br0));
-        const int4 h1 = lds_i4_volatile(smem_u32(&hdr[w][s].nb));
-        const int4 h2 = lds_i4_volatile(smem_u32(&hdr[w][s].a_off));
-        const int br0 = h0.x, nbr = h0.y, b0 = h0.z, v0 = h0.w, nb = h1.x;
-        const uint32_t a_bmp = (uint32_t)h1.z, a_col = (uint32_t)h1.w, a_off = (uint32_t)h2.x;
-        const uint32_t a_rp = (uint32_t)h2.y, a_val = (uint32_t)h2.z, a_part = (uint32_t)h2.w;
-        for (int lb = lane; lb < ((nb + 31) & ~31); lb += 32) {  // phase 1: one block per lane
+        const int v0 = h0.x, nb = h0.y;
+        const int units = max(1, (nb + 31) >> 5);
+        const uint32_t a_rot = (uint32_t)h0.z, a_val = (uint32_t)h0.w;
+        const uint32_t a_bmp = h1.x, a_col = h1.y, a_off = h1.z, a_part = h1.w;
+        const int ul = g - us;
+        if constexpr (K > 1) {  // SpMM: K right-hand sides
+            const int lb = ul * 32 + lane;
             if (lb < nb) {
                 const uint2 bm = lds_u2(a_bmp + 8u * lb);
                 const int bc = lds_i32(a_col + 4u * lb);
                 const uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
+                const uint32_t cols = used_cols(bm);
+                XSeg xs[K];
+#pragma unroll
+                for (int j = 0; j < K; ++j) load_x(xs[j], x + j * ldx, bc, nbc_vec, cols, texx, (int)(j * ldx / 4));
+                block_slots_k<SmemVals<V>, K>(bm, p, xs, a_part + 4u * (8 * K + 1) * lb);
+            }
+        } else if constexpr (DEC == 4) {
+            // tensor-core ablation (SURVEY.md §8(f) NEXT-3, fp16 values): the
+            // paper's fragment trick on mma.sync.m16n8k16 -- four
+            // blocks per MMA, block P/Q/R/S in the TL/TR/BL/BR quadrants, lane l
+            // owns bits 2l, 2l+1 of each (Alg. 2 mapping); x split
+            // into fp16 hi + lo parts (two MMAs) to keep ~22 bits of x.
+            mma_unit(ul * 32, nb, lane, a_bmp, a_col, a_off, a_val, v0, a_part, x, nbc_vec);
+        } else {
+            const int lb = ul * 32 + lane;
+            if (lb < nb) {  // phase 1: one block per lane
+                const uint2 bm = lds_u2(a_bmp + 8u * lb);
+                const int bc = lds_i32(a_col + 4u * lb);
+                const uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
                 float acc[8];
-                if constexpr (DEC != 0) {
+                const uint32_t q = a_part + kPartStride * lb;
+                if constexpr (DEC == 1 && ROT) {
                     XSeg xs;
-                    load_x(xs, x, bc, nbc_vec, used_cols(bm));
-                    block_slots<SmemVals<V>>(bm, p, xs, acc);
+                    load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
+                    block_slots_rot<SmemVals<V>>(bm, lds_u8(a_rot + (uint32_t)lb), p, xs, q);
+                } else if constexpr (DEC == 1) {
+                    XSeg xs;
+                    load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
+                    const SwapHalves sw{sizeof(V) == 2 && ((lane >> 1) & 1)};
+                    const uint32_t plo = (uint32_t)__popc(bm.x) * (uint32_t)sizeof(V);
+                    block_slots_at<SmemVals<V>>(sw.bitmap(bm), sw.on ? p + plo : p, sw.on ? p : p + plo, xs, acc);
+#pragma unroll
+                    for (int r = 0; r < 8; ++r) sts_f32(q + sw.part_off(r), acc[r]);
                 } else {
                     block_bits<SmemVals<V>>(bm, p, x + 8 * (int64_t)bc, acc);
-                }
-                const uint32_t q = a_part + kPartStride * lb;
 #pragma unroll
-                for (int r = 0; r < 8; ++r) sts_f32(q + 4u * r, acc[r]);
+                    for (int r = 0; r < 8; ++r) sts_f32(q + 4u * r, acc[r]);
+                }
             }
         }
         __syncwarp();
-        pdl_wait();
-        reduce_tile(a_rp, a_part, nbr, b0, br0, lane, m, alpha, beta, y, PeerOut{});  // phase 2
-        __syncwarp();
+        int last = 0;
+        if (lane == 0) {
+            __threadfence_block();
+            last = (atom_add_shared(a_done0 + 4u * s, 1) + 1 == units);
+        }
+        if (__shfl_sync(kFull, last, 0)) {  // phase 2: this warp completed the tile
+            __threadfence_block();
+            if (wait_y) pdl_wait();  // y of the previous kernels (hybrid residual pass)
+            const int4 h2 = lds_i4_volatile(a_hdr + 32u);  // br0, nbr, b0, a_rp
+            if constexpr (K > 1)
+                reduce_tile_k<K>((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, ldy);
+            else
+                reduce_tile((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, po);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(smem_u32(&empty_bar[s]));  // release the stage
+        }
     }
+    pdl_wait();  // a PDL-launched grid completes only after its predecessor
 }
 
 // fix-up of long block-row j by one warp: lane l adds the 8-float partials of
@@ -1008,15 +851,6 @@ k_spmv_long_chunks(int nchunks, const int32_t *__restrict__ long_rows, const int
     }
 }
 
-int kernel_variant() {
-    static int v = [] {
-        const char *e = getenv("SPADEN_KERNEL");
-        if (e && e[0] == 'v' && e[1] == '0') return 0;
-        return 1;
-    }();
-    return v;
-}
-
 int sm_count() {
     static int c = [] {
         int dev = 0, n = 148;
@@ -1029,10 +863,10 @@ int sm_count() {
 
 // Texture objects binding x (n4 float4 elements from x) for load_x, cached per
 // (device, pointer, length); SPADEN_XTEX=0 disables (LDG path, ablation).
-// Entries are never destroyed while the library is loaded, so a CUDA graph that
-// captured one stays valid; at most kTexCache distinct vectors are bound (the
-// least recently created is replaced beyond that).
-constexpr int kTexCache = 64;
+// Entries are never destroyed while the library is loaded (a CUDA graph or an
+// in-flight kernel may hold one); once kTexCache distinct vectors are bound,
+// further vectors use the LDG path (same values, load_x's other branch).
+constexpr int kTexCache = 256;
 unsigned long long x_texture(const float *x, int64_t n4) {
     const char *env = getenv("SPADEN_XTEX");  // read per call (tests toggle it)
     if ((env && env[0] == '0') || n4 <= 0) return 0ull;
@@ -1044,16 +878,18 @@ unsigned long long x_texture(const float *x, int64_t n4) {
         cudaTextureObject_t obj;
     };
     static Entry cache[kTexCache] = {};
-    static int next = 0;
-    static int max_width = -1;
+    static int used = 0;
+    static int max_width[64] = {};
     int dev = 0;
     cudaGetDevice(&dev);
     std::lock_guard<std::mutex> lock(mu);
-    for (const Entry &e : cache)
-        if (e.obj && e.x == x && e.dev == dev && e.n4 == n4) return e.obj;
-    if (max_width < 0 && cudaDeviceGetAttribute(&max_width, cudaDevAttrMaxTexture1DLinearWidth, dev) != cudaSuccess)
-        max_width = 0;
-    if (n4 > (int64_t)max_width) return 0ull;
+    for (int i = 0; i < used; ++i)
+        if (cache[i].x == x && cache[i].dev == dev && cache[i].n4 == n4) return cache[i].obj;
+    if (used == kTexCache || dev < 0 || dev >= 64) return 0ull;
+    if (max_width[dev] == 0 &&
+        cudaDeviceGetAttribute(&max_width[dev], cudaDevAttrMaxTexture1DLinearWidth, dev) != cudaSuccess)
+        max_width[dev] = -1;
+    if (n4 > (int64_t)max_width[dev]) return 0ull;
     cudaResourceDesc rd{};
     rd.resType = cudaResourceTypeLinear;
     rd.res.linear.devPtr = const_cast<float *>(x);
@@ -1066,40 +902,72 @@ unsigned long long x_texture(const float *x, int64_t n4) {
         cudaGetLastError();
         return 0ull;
     }
-    Entry &slot = cache[next];
-    next = (next + 1) % kTexCache;
-    if (slot.obj) cudaDestroyTextureObject(slot.obj);
-    slot = Entry{x, dev, n4, o};
+    cache[used++] = Entry{x, dev, n4, o};
     return o;
 }
 
-template <typename V, int DEC, int CONSUMERS, int MINB>
-cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, const float *x, float beta,
+// Resident CTAs per SM of a kernel at a dynamic shared-memory size, capped at
+// `cap`; sets the kernel's max dynamic smem attribute first.  Cached per
+// (kernel, smem, device) behind a mutex (thread-safe; several handles and
+// streams may launch concurrently).
+int occupancy(const void *kern, int threads, size_t smem, int cap, cudaError_t *err) {
+    static std::mutex mu;
+    struct Key {
+        const void *k;
+        size_t smem;
+        int dev;
+        int occ;
+    };
+    static Key cache[64];
+    static int used = 0;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lock(mu);
+    for (int i = 0; i < used; ++i)
+        if (cache[i].k == kern && cache[i].smem == smem && cache[i].dev == dev) return cache[i].occ;
+    int occ = 0;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, threads, smem);
+    if (e != cudaSuccess) {
+        *err = e;
+        return 0;
+    }
+    occ = std::max(1, std::min(occ, cap));
+    if (used < 64) cache[used++] = Key{kern, smem, dev, occ};
+    return occ;
+}
+
+// long block-rows after (or, few chunks, before and beside) the tile kernel
+template <typename V, bool SLOTS>
+cudaError_t launch_long_rows(const Matrix &A, int slot, float alpha, const float *x, int nbc_vec, float beta,
+                             float *y, cudaStream_t st, const PeerOut &po, bool dep, bool fused) {
+    float *carry = A.carry + (size_t)slot * 8 * (size_t)std::max<int64_t>(1, A.n_chunks);
+    int32_t *done = A.chunk_done + (size_t)slot * (size_t)A.n_long;
+    const unsigned g = (unsigned)((32 * A.n_chunks + 255) / 256);
+    cudaError_t e = launch_k(dep, fused ? k_spmv_long_chunks<V, SLOTS, true> : k_spmv_long_chunks<V, SLOTS, false>,
+                             dim3(g), dim3(256), 0, st, (int)A.n_chunks, (const int32_t *)A.long_rows,
+                             (const int32_t *)A.chunk_start, (const int32_t *)A.chunk_row,
+                             (const int32_t *)A.blk_rowptr, (const int32_t *)A.blk_col, (const uint64_t *)A.bitmap,
+                             (const int32_t *)A.blk_offset, (const V *)A.values, x, nbc_vec, carry, done,
+                             (int64_t)A.m, alpha, beta, y, po);
+    if (e == cudaSuccess && !fused)
+        e = launch_k(true, k_spmv_long_fixup, dim3((unsigned)((32 * A.n_long + 255) / 256)), dim3(256), 0, st,
+                     (int64_t)A.m, (int)A.n_long, (const int32_t *)A.long_rows, (const int32_t *)A.chunk_start,
+                     (const float *)carry, alpha, beta, y, po);
+    return e;
+}
+
+template <typename V, int DEC, int CONSUMERS, int MINB, bool ROT>
+cudaError_t launch_tiled_rot(const Matrix &A, int slot, const TileCfg &cfg, float alpha, const float *x, float beta,
                              float *y, cudaStream_t st, const PeerOut &po, bool dep) {
     const int nbc_vec = ((uintptr_t)x & 31u) == 0 ? (int)(A.n / 8) : 0;
     const size_t smem = (size_t)cfg.stages * cfg.stage_bytes;
-    static size_t occ_smem = 0;  // resident CTAs per SM (registers, smem), cached per smem size
-    static int occ = 0;
-    if (occ_smem != smem) {
-        auto kern = k_spmv_tiled<V, DEC, CONSUMERS, MINB>;
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e == cudaSuccess)
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * (CONSUMERS + 1), smem);
-        if (e != cudaSuccess) return e;
-        occ = std::max(1, std::min(occ, MINB));
-        occ_smem = smem;
-    }
+    auto kern = k_spmv_tiled<V, DEC, CONSUMERS, MINB, 1, ROT>;
     cudaError_t e = cudaSuccess;
+    const int occ = occupancy((const void *)kern, 32 * (CONSUMERS + 1), smem, MINB, &e);
+    if (e != cudaSuccess) return e;
     const bool hyb = A.res_max_popc > 0;  // the residual pass wrote y before these kernels
     const bool fused = A.n_long > 0 && A.n_chunks <= fused_fixup_max();
-    auto launch_long = [&](bool d) {
-        const unsigned g = (unsigned)((32 * A.n_chunks + 255) / 256);
-        return launch_k(d, fused ? k_spmv_long_chunks<V, (DEC != 0), true> : k_spmv_long_chunks<V, (DEC != 0), false>,
-                        dim3(g), dim3(256), 0, st, (int)A.n_chunks, (const int32_t *)A.long_rows,
-                        (const int32_t *)A.chunk_start, (const int32_t *)A.chunk_row, (const int32_t *)A.blk_rowptr,
-                        (const int32_t *)A.blk_col, (const uint64_t *)A.bitmap, (const int32_t *)A.blk_offset,
-                        (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, (int64_t)A.m, alpha, beta, y, po);
-    };
     // few long-row chunks (one wave): launch them first, the tiled kernel then
     // starts (PDL) while they run -- their rows are disjoint, so it waits for
     // them only before exiting.  Many chunks: tiled kernel, then the chunks as a
@@ -1107,150 +975,92 @@ cudaError_t launch_tiled_cfg(const Matrix &A, const TileCfg &cfg, float alpha, c
     // CTAs in pdl_wait next to the tiled kernel: rmat22 pure 1.33 -> 2.20 ms),
     // then the separate fix-up.
     if (fused) {
-        e = launch_long(dep);
+        e = launch_long_rows<V, (DEC != 0)>(A, slot, alpha, x, nbc_vec, beta, y, st, po, dep, true);
         dep = true;
     }
     if (A.n_tiles > 0 && e == cudaSuccess) {
         const int grid = (int)std::min<int64_t>(A.n_tiles, (int64_t)sm_count() * occ);
         const unsigned long long texx = x_texture(x, 2 * (int64_t)nbc_vec);
-        e = launch_k(dep, k_spmv_tiled<V, DEC, CONSUMERS, MINB>, dim3(grid), dim3(32 * (CONSUMERS + 1)), smem, st,
+        e = launch_k(dep, kern, dim3(grid), dim3(32 * (CONSUMERS + 1)), smem, st,
                      cfg.stages, cfg.stage_bytes, (int64_t)A.m, (const TileDesc *)A.tiles, (int)A.n_tiles,
                      (const int32_t *)A.blk_rowptr, (const int32_t *)A.blk_col, (const uint64_t *)A.bitmap,
                      (const int32_t *)A.blk_offset, (const V *)A.values, x, nbc_vec, alpha, beta, y, (int64_t)0,
-                     (int64_t)0, po, texx, (int)hyb);
+                     (int64_t)0, po, texx, (int)hyb, (const uint8_t *)A.rot);
         dep = true;
     }
-    if (A.n_long > 0 && !fused && e == cudaSuccess) {
-        e = launch_long(false);
-        if (e == cudaSuccess)
-            e = launch_k(true, k_spmv_long_fixup, dim3((unsigned)((32 * A.n_long + 255) / 256)), dim3(256), 0, st,
-                         (int64_t)A.m, (int)A.n_long, (const int32_t *)A.long_rows, (const int32_t *)A.chunk_start,
-                         (const float *)A.carry, alpha, beta, y, po);
-    }
+    if (A.n_long > 0 && !fused && e == cudaSuccess)
+        e = launch_long_rows<V, (DEC != 0)>(A, slot, alpha, x, nbc_vec, beta, y, st, po, false, false);
     if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }
 
-template <typename V, int DEC, int WARPS, int S>
-cudaError_t launch_warp_cfg(const Matrix &A, const TileCfg &cfg, float alpha, const float *x, float beta,
-                            float *y, cudaStream_t st) {
-    const int nbc_vec = ((uintptr_t)x & 31u) == 0 ? (int)(A.n / 8) : 0;
-    const size_t smem = (size_t)WARPS * S * cfg.stage_bytes;
-    static size_t occ_smem = 0;  // occupancy cached per dynamic-smem size
-    static int occ = 0;
-    if (occ_smem != smem) {
-        auto kern = k_spmv_warp<V, DEC, WARPS, S>;
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * WARPS, smem);
-        if (e != cudaSuccess) return e;
-        occ = std::max(1, std::min(occ, cfg.ctas_per_sm));
-        occ_smem = smem;
+template <typename V, int DEC, int CONSUMERS, int MINB>
+cudaError_t launch_tiled_cfg(const Matrix &A, int slot, const TileCfg &cfg, float alpha, const float *x, float beta,
+                             float *y, cudaStream_t st, const PeerOut &po, bool dep) {
+    if constexpr (DEC == 1) {
+        if (A.rot) return launch_tiled_rot<V, DEC, CONSUMERS, MINB, true>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
     }
-    if (A.n_tiles > 0) {
-        const int64_t need = (A.n_tiles + WARPS - 1) / WARPS;
-        const int grid = (int)std::min<int64_t>(need, (int64_t)sm_count() * occ);
-        k_spmv_warp<V, DEC, WARPS, S><<<grid, 32 * WARPS, smem, st>>>(
-            cfg.stage_bytes, A.m, A.tiles, (int)A.n_tiles, A.blk_rowptr, A.blk_col, A.bitmap, A.blk_offset,
-            (const V *)A.values, x, nbc_vec, alpha, beta, y);
-    }
-    if (A.n_long > 0) {
-        const int64_t threads = 32 * A.n_chunks;
-        if (A.n_chunks <= fused_fixup_max())
-            k_spmv_long_chunks<V, (DEC != 0), true><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
-            (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, A.m, alpha, beta, y, PeerOut{});
-        else
-            k_spmv_long_chunks<V, (DEC != 0), false><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
-            (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, x, nbc_vec, A.carry, A.chunk_done, A.m, alpha, beta, y, PeerOut{});
-        if (A.n_chunks > fused_fixup_max())
-            k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
-                A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, y, PeerOut{});
-    }
-    return cudaGetLastError();
+    return launch_tiled_rot<V, DEC, CONSUMERS, MINB, false>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
 }
 
 template <typename V, int DEC>
-cudaError_t launch_tiled(const Matrix &A, float alpha, const float *x, float beta, float *y, cudaStream_t st,
-                         const PeerOut &po, bool dep) {
+cudaError_t launch_tiled(const Matrix &A, int slot, float alpha, const float *x, float beta, float *y,
+                         cudaStream_t st, const PeerOut &po, bool dep) {
     const TileCfg cfg = tile_cfg(A.tile_cfg);
     switch (A.tile_cfg) {
-    case 4: return launch_warp_cfg<V, DEC, 4, 2>(A, cfg, alpha, x, beta, y, st);
-    case 5: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 6: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 7: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 8: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 9: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 10: return launch_tiled_cfg<V, DEC, 4, 6>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 11: return launch_tiled_cfg<V, DEC, 4, 5>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 12: return launch_tiled_cfg<V, DEC, 4, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 13: return launch_tiled_cfg<V, DEC, 4, 6>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 14: return launch_tiled_cfg<V, DEC, 12, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 15: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 16: return launch_tiled_cfg<V, DEC, 8, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 2: return launch_tiled_cfg<V, DEC, 8, 3>(A, cfg, alpha, x, beta, y, st, po, dep);
-    case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, cfg, alpha, x, beta, y, st, po, dep);
-    default: return launch_tiled_cfg<V, DEC, 16, 1>(A, cfg, alpha, x, beta, y, st, po, dep);
+    case 5: return launch_tiled_cfg<V, DEC, 8, 3>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
+    case 6: return launch_tiled_cfg<V, DEC, 16, 2>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
+    case 7: return launch_tiled_cfg<V, DEC, 8, 4>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
+    case 10: return launch_tiled_cfg<V, DEC, 4, 6>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
+    case 14: return launch_tiled_cfg<V, DEC, 12, 2>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
+    case 15: return launch_tiled_cfg<V, DEC, 16, 2>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
+    case 16: return launch_tiled_cfg<V, DEC, 8, 2>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
+    case 1: return launch_tiled_cfg<V, DEC, 16, 2>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
+    case 3: return launch_tiled_cfg<V, DEC, 8, 4>(A, slot, cfg, alpha, x, beta, y, st, po, dep);
+    default: return launch_tiled_cfg<V, DEC, 8, 3>(A, slot, cfg, alpha, x, beta, y, st, po, dep);  // cfg 2
     }
 }
 
 template <typename V, int K, int CONSUMERS, int MINB>
-cudaError_t launch_spmm_cfg(const Matrix &A, const TileCfg &cfg, const TileDesc *tiles, int64_t ntiles, float alpha,
+cudaError_t launch_spmm_cfg(const Matrix &A, int slot, const TileCfg &cfg, const TileDesc *tiles, int64_t ntiles, float alpha,
                             const float *X, int64_t ldx, float beta, float *Y, int64_t ldy, cudaStream_t st) {
     const bool aligned = ((uintptr_t)X & 31u) == 0 && ((ldx * 4) % 32) == 0;
     const int nbc_vec = aligned ? (int)(A.n / 8) : 0;
     const size_t smem = (size_t)cfg.stages * cfg.stage_bytes;
-    static size_t occ_smem = 0;
-    static int occ = 0;
-    if (occ_smem != smem) {
-        auto kern = k_spmv_tiled<V, 1, CONSUMERS, MINB, K>;
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e == cudaSuccess)
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * (CONSUMERS + 1), smem);
-        if (e != cudaSuccess) return e;
-        occ = std::max(1, std::min(occ, MINB));
-        occ_smem = smem;
-    }
+    cudaError_t oe = cudaSuccess;
+    const int occ = occupancy((const void *)k_spmv_tiled<V, 1, CONSUMERS, MINB, K>, 32 * (CONSUMERS + 1), smem,
+                              MINB, &oe);
+    if (oe != cudaSuccess) return oe;
     if (ntiles > 0) {
         const int grid = (int)std::min<int64_t>(ntiles, (int64_t)sm_count() * occ);
         const unsigned long long texx = nbc_vec ? x_texture(X, 2 * (int64_t)nbc_vec + (K - 1) * (ldx / 4)) : 0ull;
         k_spmv_tiled<V, 1, CONSUMERS, MINB, K><<<grid, 32 * (CONSUMERS + 1), smem, st>>>(
             cfg.stages, cfg.stage_bytes, A.m, tiles, (int)ntiles, A.blk_rowptr, A.blk_col, A.bitmap,
-            A.blk_offset, (const V *)A.values, X, nbc_vec, alpha, beta, Y, ldx, ldy, PeerOut{}, texx, 1);
+            A.blk_offset, (const V *)A.values, X, nbc_vec, alpha, beta, Y, ldx, ldy, PeerOut{}, texx, 1,
+            (const uint8_t *)nullptr);
     }
     if (A.n_long > 0) {  // long block-rows: the SpMV chunk path, once per vector (same arithmetic)
         const int nbc1 = ((uintptr_t)X & 31u) == 0 && ((ldx * 4) % 32) == 0 ? (int)(A.n / 8) : 0;
+        const bool fused = A.n_chunks <= fused_fixup_max();
         for (int j = 0; j < K; ++j) {
-            const int64_t threads = 32 * A.n_chunks;
-            if (A.n_chunks <= fused_fixup_max())
-                k_spmv_long_chunks<V, true, true><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
-                (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
-                A.blk_offset, (const V *)A.values, X + j * ldx, nbc1, A.carry, A.chunk_done, A.m, alpha, beta,
-                Y + j * ldy, PeerOut{});
-            else
-                k_spmv_long_chunks<V, true, false><<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(
-                (int)A.n_chunks, A.long_rows, A.chunk_start, A.chunk_row, A.blk_rowptr, A.blk_col, A.bitmap,
-                A.blk_offset, (const V *)A.values, X + j * ldx, nbc1, A.carry, A.chunk_done, A.m, alpha, beta,
-                Y + j * ldy, PeerOut{});
-            if (A.n_chunks > fused_fixup_max())
-                k_spmv_long_fixup<<<(unsigned)((32 * A.n_long + 255) / 256), 256, 0, st>>>(
-                    A.m, (int)A.n_long, A.long_rows, A.chunk_start, A.carry, alpha, beta, Y + j * ldy, PeerOut{});
+            cudaError_t e = launch_long_rows<V, true>(A, slot, alpha, X + j * ldx, nbc1, beta, Y + j * ldy, st,
+                                                      PeerOut{}, false, fused);
+            if (e != cudaSuccess) return e;
         }
     }
     return cudaGetLastError();
 }
 
 template <typename V, int K>
-cudaError_t launch_spmm(const Matrix &A, const TileDesc *tiles, int64_t ntiles, float alpha, const float *X,
+cudaError_t launch_spmm(const Matrix &A, int slot, const TileDesc *tiles, int64_t ntiles, float alpha, const float *X,
                         int64_t ldx, float beta, float *Y, int64_t ldy, cudaStream_t st) {
     const TileCfg cfg = tile_cfg(A.tile_cfg);
     // same stage geometry as the SpMV schedule; fewer CTAs per SM so the K
     // accumulators and x segments fit in registers without spilling
     switch (A.tile_cfg) {
     case 0: case 1: case 6:
-        return launch_spmm_cfg<V, K, 16, 1>(A, cfg, tiles, ntiles, alpha, X, ldx, beta, Y, ldy, st);
-    default: return launch_spmm_cfg<V, K, 8, 2>(A, cfg, tiles, ntiles, alpha, X, ldx, beta, Y, ldy, st);
+        return launch_spmm_cfg<V, K, 16, 1>(A, slot, cfg, tiles, ntiles, alpha, X, ldx, beta, Y, ldy, st);
+    default: return launch_spmm_cfg<V, K, 8, 2>(A, slot, cfg, tiles, ntiles, alpha, X, ldx, beta, Y, ldy, st);
     }
 }
 
@@ -1289,18 +1099,20 @@ spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx,
             float *Yj = Y + j * ldy;
             cudaError_t e = cudaSuccess;
             float beta_bit = beta;  // hybrid: residual pass first (y = beta*y + alpha*A_res*x), then accumulate
+            const int slot = pick_scratch(A);
             if (A.res_max_popc > 0) {
+                bool launched = false;
                 for (int q = 0; q < K && e == cudaSuccess; ++q)
-                    e = residual_first(A, alpha, Xj + q * ldx, beta, Yj + q * ldy, st);
+                    e = residual_first(A, alpha, Xj + q * ldx, beta, Yj + q * ldy, st, slot, &launched);
                 beta_bit = 1.f;
             }
             if (e != cudaSuccess) return cuda_status(e, "launching the residual pass");
             if (A.storage == SPADEN_R_16F)
-                e = K == 4 ? launch_spmm<__half, 4>(A, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st)
-                           : launch_spmm<__half, 2>(A, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st);
+                e = K == 4 ? launch_spmm<__half, 4>(A, slot, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st)
+                           : launch_spmm<__half, 2>(A, slot, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st);
             else
-                e = K == 4 ? launch_spmm<float, 4>(A, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st)
-                           : launch_spmm<float, 2>(A, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st);
+                e = K == 4 ? launch_spmm<float, 4>(A, slot, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st)
+                           : launch_spmm<float, 2>(A, slot, tiles, nt, alpha, Xj, ldx, beta_bit, Yj, ldy, st);
             if (e != cudaSuccess) return cuda_status(e, "launching SpMM");
         }
         j += K;
@@ -1322,7 +1134,6 @@ int spmv_launch_count(const Matrix &A, float beta) {
             if (P.n_long > 0) n += 1 + (P.n_chunks > fused_fixup_max() ? 1 : 0);
         }
     }
-    if (kernel_variant() == 0) return n + 1;
     n += A.n_tiles > 0 ? 1 : 0;
     if (A.n_long > 0) n += 1 + (A.n_chunks > fused_fixup_max() ? 1 : 0);
     return n;
@@ -1331,44 +1142,26 @@ int spmv_launch_count(const Matrix &A, float beta) {
 spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float beta, float *y,
                             cudaStream_t st, const PeerOut *peers) {
     if (A.m == 0) return SPADEN_OK;
-    const bool x_vec = ((uintptr_t)x & 15u) == 0;
     const PeerOut po = peers ? *peers : PeerOut{};
-    if (po.n > 0 && (A.res_nnz > 0 || tile_cfg(A.tile_cfg).warp_mode)) {
-        set_error("the fused all-gather store needs pure bitBSR and a CTA-pipeline tile config");
+    if (po.n > 0 && A.res_max_popc > 0) {
+        set_error("the fused all-gather store needs a pure bitBSR handle (no hybrid residual)");
         return SPADEN_ERR_UNSUPPORTED;
     }
     // hybrid (NEXT-1): the residual pass runs first and applies beta to every row
     // (y = beta*y + alpha*A_res*x); the bitBSR kernels then accumulate (beta = 1)
     // over the block-rows that hold blocks (the schedule skips the others)
-    const bool dep = A.res_max_popc > 0;  // bitBSR kernels follow the residual pass (PDL)
+    bool dep = false;  // bitBSR kernels follow a residual kernel of this call (PDL)
+    const int slot = pick_scratch(A);
     if (A.res_max_popc > 0) {
-        SPADEN_CUDA_TRY(residual_first(A, alpha, x, beta, y, st));
+        SPADEN_CUDA_TRY(residual_first(A, alpha, x, beta, y, st, slot, &dep));
         beta = 1.f;
-    }
-    if (kernel_variant() == 0 && po.n == 0) {
-        const int threads = 256;
-        const int64_t want = (A.Bnrow + 7) / 8;
-        const unsigned grid = (unsigned)std::min<int64_t>(want, 148LL * 64);
-        if (A.storage == SPADEN_R_16F)
-            k_spmv_v0<__half><<<grid, threads, 0, st>>>(A.m, A.n, A.Bnrow, A.blk_rowptr, A.blk_col, A.bitmap,
-                                                       A.blk_offset, (const __half *)A.values, x, x_vec, alpha,
-                                                       beta, y);
-        else
-            k_spmv_v0<float><<<grid, threads, 0, st>>>(A.m, A.n, A.Bnrow, A.blk_rowptr, A.blk_col, A.bitmap,
-                                                      A.blk_offset, (const float *)A.values, x, x_vec, alpha,
-                                                      beta, y);
-        SPADEN_CUDA_TRY(cudaGetLastError());
-        return SPADEN_OK;
     }
     // decode style from the mean block fill (predicated slots for dense-ish blocks)
     const int decode_env = [] {  // SPADEN_DECODE=bits|slots|rows|mma overrides (ablation), read per call
         const char *e = getenv("SPADEN_DECODE");
         if (e && e[0] == 'b') return 0;
         if (e && e[0] == 's') return 1;
-        if (e && e[0] == 'r') return 2;
         if (e && e[0] == 'm') return 4;
-        if (e && e[0] == 'q') return 5;  // "quad": 4 lanes per block
-        if (e && e[0] == 'p') return 6;  // "pair": 2 lanes per block
         return -1;
     }();
     const int dec = decode_env >= 0 ? decode_env
@@ -1376,20 +1169,14 @@ spaden_status_t spmv_launch(const Matrix &A, float alpha, const float *x, float 
     cudaError_t e;
     if (A.storage == SPADEN_R_16F) {
         switch (dec) {
-        case 0: e = launch_tiled<__half, 0>(A, alpha, x, beta, y, st, po, dep); break;
-        case 2: e = launch_tiled<__half, 2>(A, alpha, x, beta, y, st, po, dep); break;
-        case 4: e = launch_tiled<__half, 4>(A, alpha, x, beta, y, st, po, dep); break;
-        case 5: e = launch_tiled<__half, 5>(A, alpha, x, beta, y, st, po, dep); break;
-        case 6: e = launch_tiled<__half, 6>(A, alpha, x, beta, y, st, po, dep); break;
-        default: e = launch_tiled<__half, 1>(A, alpha, x, beta, y, st, po, dep);
+        case 0: e = launch_tiled<__half, 0>(A, slot, alpha, x, beta, y, st, po, dep); break;
+        case 4: e = launch_tiled<__half, 4>(A, slot, alpha, x, beta, y, st, po, dep); break;
+        default: e = launch_tiled<__half, 1>(A, slot, alpha, x, beta, y, st, po, dep);
         }
     } else {  // (the tensor-core ablation exists for fp16 values only)
         switch (dec) {
-        case 0: e = launch_tiled<float, 0>(A, alpha, x, beta, y, st, po, dep); break;
-        case 2: e = launch_tiled<float, 2>(A, alpha, x, beta, y, st, po, dep); break;
-        case 5: e = launch_tiled<float, 5>(A, alpha, x, beta, y, st, po, dep); break;
-        case 6: e = launch_tiled<float, 6>(A, alpha, x, beta, y, st, po, dep); break;
-        default: e = launch_tiled<float, 1>(A, alpha, x, beta, y, st, po, dep);
+        case 0: e = launch_tiled<float, 0>(A, slot, alpha, x, beta, y, st, po, dep); break;
+        default: e = launch_tiled<float, 1>(A, slot, alpha, x, beta, y, st, po, dep);
         }
     }
     if (e != cudaSuccess) return cuda_status(e, "launching k_spmv_tiled");

@@ -43,6 +43,30 @@ class RowPartition:
         return r0, r1
 
 
+def convert_slice(rowptr, colidx, values, n: int, storage=None, residual_max_popc: int = 0, group=None,
+                  stream=None):
+    """Convert this rank's row slice (local rows, global columns).  With the
+    automatic hybrid choice (residual_max_popc = -1) and several ranks, the
+    choice is taken from the WHOLE matrix's mean block fill: each rank counts
+    its slice's blocks (spaden_count_blocks; Bnnz is additive over 8-row-aligned
+    slices), one all-reduce sums (nnz, Bnnz), and every rank converts with that
+    fill -- so all slices take the same t and y stays partition invariant."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_cheny24_b200 as sp
+
+    fill = 0.0
+    if residual_max_popc < 0 and dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+        cnt = torch.tensor([float(colidx.numel()), float(sp.count_blocks(rowptr, colidx, n, stream=stream))],
+                           dtype=torch.float64, device=rowptr.device)
+        dist.all_reduce(cnt, group=group)
+        nnz, bnnz = float(cnt[0]), float(cnt[1])
+        fill = min(64.0, nnz / bnnz) if bnnz > 0 else 64.0
+    return sp.convert(rowptr, colidx, values, n, storage=storage, stream=stream,
+                      residual_max_popc=residual_max_popc, auto_mean_fill=fill)
+
+
 def gather_slices(full, local, group=None):
     """full[world*slice] <- concat over ranks of local[slice] (in rank order)."""
     import torch.distributed as dist
@@ -77,6 +101,7 @@ class IteratedSpMV:
         self.x[: x0.numel()].copy_(x0)
         self.x_next = torch.zeros_like(self.x)
         self.r0, self.r1 = part.range(rank)
+        self.gather_events = None  # (start, end) CUDA events around the all-gather (bench timing)
 
     def local_slot(self, buf):
         s = self.part.slice_rows
@@ -88,7 +113,12 @@ class IteratedSpMV:
         if c is not None:
             y.fill_(c)
         self.local_spmv(self.x[: self.n], y, alpha, 0.0 if c is None else 1.0)
+        ev = self.gather_events
+        if ev is not None:
+            ev[0].record()
         gather_slices(self.x_next[: self.part.padded], slot, self.group)
+        if ev is not None:
+            ev[1].record()
         self.x, self.x_next = self.x_next, self.x
         return self.x
 

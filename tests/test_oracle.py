@@ -80,6 +80,20 @@ def test_spmv_vs_dense_bruteforce(m, n, dens, seed):
     np.testing.assert_allclose(s, ref_s, rtol=1e-13, atol=1e-13)
 
 
+@pytest.mark.parametrize("m,n,dens,seed", [(0, 5, 0.1, 0), (255, 129, 0.01, 3), (256, 256, 0.3, 4)])
+def test_spmv_omp_vs_dense_and_serial(m, n, dens, seed):
+    """The all-cores oracle (bench cpu_baseline arm) against the dense product,
+    and bitwise against the serial Alg. 1 (same per-row order)."""
+    A = W.random_sparse(m, n, dens, seed)
+    x = W.vector(n, seed + 10)
+    y, s, threads = oracle.spmv_omp(A.rowptr, A.colidx, A.values, x)
+    assert threads >= 1
+    ref = dense_of(A) @ x.astype(np.float64)
+    np.testing.assert_allclose(y, ref, rtol=1e-13, atol=1e-13)
+    y1, s1 = oracle.spmv(A.rowptr, A.colidx, A.values, x)
+    assert np.array_equal(y, y1) and np.array_equal(s, s1)
+
+
 def tiles_bruteforce(A):
     """Independent bitBSR builder from the dense view: walk every 8x8 tile of
     the dense pattern in (tile-row, tile-col) order, bit = 8r + c."""
