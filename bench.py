@@ -60,6 +60,8 @@ def parse():
     p.add_argument("--no-cusparse", action="store_true")
     p.add_argument("--no-variants", action="store_true", help="skip the other-precision kernel timing")
     p.add_argument("--spmm", default="4", help="comma list of right-hand-side counts for the SpMM extra ('' = skip)")
+    p.add_argument("--spmm-tc", default="128", help="comma list of right-hand-side counts for the tensor-core "
+                                                   "SpMM extra (fp16 storage, tcgen05; '' = skip)")
     p.add_argument("--hybrid", type=int, default=-1,
                    help="hybrid format: blocks with <= HYBRID entries go to a CSR residual (0 = pure bitBSR, "
                         "-1 = automatic by mean block fill)")
@@ -572,6 +574,55 @@ def main():
                                 "per_vector_speedup_vs_spmv": kavg_ms * K / sms}
                 del X, Yk
 
+        # ---- NEXT-4: tensor-core SpMM (tcgen05, fp16 storage and fp16 x slabs)
+        spmm_tc = {}
+        if world == 1 and args.spmm_tc and info.residual_max_popc == 0:
+            Mh = M if args.dtype == "fp16" else sp.convert(*local_csr, wl.n, storage="fp16", residual_max_popc=0)
+            # the same matrix's fp16 SpMV kernel time (per-vector reference)
+            yv = torch.empty(wl.m, dtype=torch.float32, device=dev)
+            for _ in range(5):
+                Mh.spmv(wl.x0, yv, stream=stream)
+            s0e, s1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize(dev)
+            s0e.record(stream)
+            for _ in range(50):
+                Mh.spmv(wl.x0, yv, stream=stream)
+            s1e.record(stream)
+            torch.cuda.synchronize(dev)
+            spmv16_ms = s0e.elapsed_time(s1e) / 50
+            for K in [int(v) for v in args.spmm_tc.split(",") if v]:
+                gen = torch.Generator(device=dev).manual_seed(7)
+                X = torch.rand((K, wl.n), generator=gen, device=dev, dtype=torch.float32) * 2 - 1
+                Yk = torch.empty((K, wl.m), dtype=torch.float32, device=dev)
+                Xb = Mh.pack_x_tc(X, stream=stream)
+                for _ in range(3):
+                    Mh.spmm_tc(Xb, K, Yk, alpha=wl.alpha, stream=stream)
+                reps = max(5, min(args.steps, 50))
+                p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                s0e, s1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                torch.cuda.synchronize(dev)
+                p0.record(stream)
+                for _ in range(reps):
+                    Mh.pack_x_tc(X, Xb, stream=stream)
+                p1.record(stream)
+                s0e.record(stream)
+                for _ in range(reps):
+                    Mh.spmm_tc(Xb, K, Yk, alpha=wl.alpha, stream=stream)
+                s1e.record(stream)
+                torch.cuda.synchronize(dev)
+                tms = s0e.elapsed_time(s1e) / reps
+                pms = p0.elapsed_time(p1) / reps
+                spmm_tc[str(K)] = {"ms": tms, "pack_x_ms": pms,
+                                   "gflops": 2.0 * wl.nnz * K / (tms * 1e-3) / 1e9,
+                                   "gflops_incl_pack": 2.0 * wl.nnz * K / ((tms + pms) * 1e-3) / 1e9,
+                                   "per_vector_speedup_vs_fp16_spmv": spmv16_ms * K / tms,
+                                   "fp16_spmv_ms": spmv16_ms,
+                                   "precision": "fp16 A (stored), fp16 x (RNE), fp32 accumulation in TMEM"}
+                del X, Yk, Xb
+            if Mh is not M:
+                Mh.free()
+            del yv
+
         n_launch = M.launch_count(1.0 if wl.c is not None else 0.0)  # kernels + memsets of one spaden_spmv
         line = {
             "metric": METRIC, "value": gflops, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -609,6 +660,7 @@ def main():
             "cusparse_csr": cus,
             "variants": variants,
             "spmm": spmm,
+            "spmm_tc": spmm_tc,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": args.steps * n_launch,

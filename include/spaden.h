@@ -236,6 +236,32 @@ SPADEN_API spaden_status_t spaden_spmm(spaden_matrix_t A, float alpha, const flo
                                        int32_t k, float beta, float *d_Y, int64_t ldy, void *stream);
 
 /*
+ * spaden_spmm_tc_pack_x -- x slabs for spaden_spmm_tc: d_Xb[bc][j][c] =
+ * fp16(d_X[j*ldx + 8*bc + c]) for block columns bc < ceil(n/8), vectors j < k,
+ * c < 8 (round to nearest even; entries past n are 0).  d_X: float32,
+ * column-major (vector j at d_X + j*ldx, ldx >= n).  d_Xb: DEVICE buffer of
+ * 16 * ceil(n/8) * k bytes, 16-byte aligned, owned by the caller.  Stream-ordered.
+ */
+SPADEN_API spaden_status_t spaden_spmm_tc_pack_x(int64_t n, int32_t k, const float *d_X, int64_t ldx, void *d_Xb,
+                                                 void *stream);
+
+/*
+ * spaden_spmm_tc -- Y[:, j] = alpha * A X[:, j] + beta * Y[:, j], j < k, on the
+ * tcgen05 tensor cores (the paper's SpMM future work,
+ * P:L336).  X enters as fp16 slabs from spaden_spmm_tc_pack_x (fp16 inputs and
+ * fp32 accumulation: the paper's tensor-core precision); Y is float32,
+ * column-major (ldy >= m).  Per block-row, every pair of consecutive blocks is
+ * one tcgen05.mma (M = 128 vectors, N = 8 rows, K = 16) accumulating in TMEM
+ * in block order: deterministic.  Unlike the CUDA-core paths, structural zeros
+ * of a stored block are multiplied (as in the paper's MMA), so X must be finite.
+ *   A       pure bitBSR handle with fp16 storage (else SPADEN_ERR_UNSUPPORTED).
+ *   d_Xb    slabs of the k vectors (see above); d_Y must not overlap it.
+ * Never allocates or synchronises.
+ */
+SPADEN_API spaden_status_t spaden_spmm_tc(spaden_matrix_t A, float alpha, const void *d_Xb, int32_t k, float beta,
+                                          float *d_Y, int64_t ldy, void *stream);
+
+/*
  * spaden_spmv_host -- the same operation with HOST vectors: copies h_x (and h_y if
  * beta != 0) to device staging buffers owned by the handle, runs spaden_spmv,
  * copies y back to h_y and synchronises `stream`.  Not thread-safe per handle.

@@ -81,6 +81,12 @@ spaden_spmv_scatter.restype = _ST
 spaden_spmm = _lib.spaden_spmm
 spaden_spmm.argtypes = [_P, _F, _P, _I64, ctypes.c_int32, _F, _P, _I64, _P]
 spaden_spmm.restype = _ST
+spaden_spmm_tc_pack_x = _lib.spaden_spmm_tc_pack_x
+spaden_spmm_tc_pack_x.argtypes = [_I64, ctypes.c_int32, _P, _I64, _P, _P]
+spaden_spmm_tc_pack_x.restype = _ST
+spaden_spmm_tc = _lib.spaden_spmm_tc
+spaden_spmm_tc.argtypes = [_P, _F, _P, ctypes.c_int32, _F, _P, _I64, _P]
+spaden_spmm_tc.restype = _ST
 spaden_spmv_host = _lib.spaden_spmv_host
 spaden_spmv_host.argtypes = [_P, _F, _P, _F, _P, _P]
 spaden_spmv_host.restype = _ST
@@ -110,7 +116,7 @@ spaden_version.argtypes = []
 spaden_version.restype = ctypes.c_char_p
 
 EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_count_blocks", "spaden_spmv", "spaden_spmm",
-            "spaden_spmv_scatter", "spaden_spmv_host", "spaden_spmv_host_batched",
+            "spaden_spmv_scatter", "spaden_spmm_tc_pack_x", "spaden_spmm_tc", "spaden_spmv_host", "spaden_spmv_host_batched",
             "spaden_free",
             "spaden_get_info", "spaden_get_arrays", "spaden_spmv_launch_count", "spaden_status_string",
             "spaden_last_error_message", "spaden_version"]
@@ -254,6 +260,31 @@ class Matrix:
         assert X.shape[1] == self.n and Y.shape == (k, self.m) and X.stride(1) == 1 and Y.stride(1) == 1
         _check(spaden_spmm(self._h, alpha, ctypes.c_void_p(X.data_ptr()), X.stride(0), k, beta,
                            ctypes.c_void_p(Y.data_ptr()), Y.stride(0), _stream_ptr(stream)), "spaden_spmm")
+        return Y
+
+    def pack_x_tc(self, X, Xb=None, stream=None):
+        """fp16 x slabs for spmm_tc (spaden_spmm_tc_pack_x): X is k x n (CUDA float32, rows
+        contiguous); returns a uint8 CUDA tensor of 16 * ceil(n/8) * k bytes."""
+        torch = _torch()
+        k = X.shape[0]
+        assert X.dtype == torch.float32 and X.is_cuda and X.shape[1] == self.n and X.stride(1) == 1
+        nbytes = 16 * ((self.n + 7) // 8) * k
+        if Xb is None:
+            Xb = torch.empty(max(16, nbytes), dtype=torch.uint8, device=X.device)
+        assert Xb.numel() >= nbytes and Xb.is_cuda
+        _check(spaden_spmm_tc_pack_x(self.n, k, ctypes.c_void_p(X.data_ptr()), X.stride(0),
+                                     ctypes.c_void_p(Xb.data_ptr()), _stream_ptr(stream)), "spaden_spmm_tc_pack_x")
+        return Xb
+
+    def spmm_tc(self, Xb, k: int, Y=None, alpha: float = 1.0, beta: float = 0.0, stream=None):
+        """Y[j] = alpha * A x_j + beta * Y[j] on the tensor cores (spaden_spmm_tc) from the
+        fp16 slabs of pack_x_tc; Y is k x m (CUDA float32, rows contiguous)."""
+        torch = _torch()
+        if Y is None:
+            Y = torch.empty((k, self.m), dtype=torch.float32, device=Xb.device)
+        assert Y.dtype == torch.float32 and Y.is_cuda and Y.shape == (k, self.m) and Y.stride(1) == 1
+        _check(spaden_spmm_tc(self._h, alpha, ctypes.c_void_p(Xb.data_ptr()), k, beta,
+                              ctypes.c_void_p(Y.data_ptr()), Y.stride(0), _stream_ptr(stream)), "spaden_spmm_tc")
         return Y
 
     def spmv_host(self, x_host, y_host, alpha: float = 1.0, beta: float = 0.0, stream=None):

@@ -47,7 +47,7 @@ static void release(Matrix *A) {
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap,   A->blk_offset, A->values,
                     A->stage_x,     A->stage_y,  A->tiles, A->rot,
                     A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->chunk_done,
-                    A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2]};
+                    A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2], A->tc_chunks, A->tc_cta_start};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     for (int j = 0; j < Matrix::kMaxPipe; ++j) {
@@ -278,6 +278,38 @@ spaden_status_t spaden_spmm(spaden_matrix_t A, float alpha, const float *d_X, in
     }
     if (k == 0) return SPADEN_OK;
     return spmm_launch(*A, alpha, d_X, ldx, k, beta, d_Y, ldy, (cudaStream_t)stream);
+}
+
+spaden_status_t spaden_spmm_tc_pack_x(int64_t n, int32_t k, const float *d_X, int64_t ldx, void *d_Xb,
+                                      void *stream) {
+    g_last_error.clear();
+    if (n < 0 || k < 0 || ldx < n || (n > 0 && k > 0 && (!d_X || !d_Xb)) || ((uintptr_t)d_Xb & 15u)) {
+        set_error("bad arguments (n, k >= 0, ldx >= n, non-NULL 16-byte aligned d_Xb)");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    return spmm_tc_pack_x(n, k, d_X, ldx, d_Xb, (cudaStream_t)stream);
+}
+
+spaden_status_t spaden_spmm_tc(spaden_matrix_t A, float alpha, const void *d_Xb, int32_t k, float beta, float *d_Y,
+                               int64_t ldy, void *stream) {
+    g_last_error.clear();
+    if (!A || k < 0 || ldy < A->m || (k > 0 && A->m > 0 && (!d_Y || !d_Xb)) || ((uintptr_t)d_Xb & 15u)) {
+        set_error("NULL handle/matrices, k < 0, ldy < m, or d_Xb not 16-byte aligned");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (A->storage != SPADEN_R_16F || A->res_max_popc > 0) {
+        set_error("spaden_spmm_tc needs a pure bitBSR handle with fp16 storage");
+        return SPADEN_ERR_UNSUPPORTED;
+    }
+    if (k > 0 && A->m > 0 && A->n > 0) {
+        const char *xb = (const char *)d_Xb, *xe = xb + 16 * ((A->n + 7) / 8) * (int64_t)k;
+        const char *yb = (const char *)d_Y, *ye = (const char *)(d_Y + (int64_t)(k - 1) * ldy + A->m);
+        if (xb < ye && yb < xe) {
+            set_error("X slabs and Y must not overlap");
+            return SPADEN_ERR_INVALID_ARGUMENT;
+        }
+    }
+    return spmm_tc_launch(*A, alpha, d_Xb, k, beta, d_Y, ldy, (cudaStream_t)stream);
 }
 
 spaden_status_t spaden_spmv_host(spaden_matrix_t A, float alpha, const float *h_x, float beta, float *h_y,

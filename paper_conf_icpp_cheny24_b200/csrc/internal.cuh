@@ -52,6 +52,11 @@ struct spaden_matrix_s {
     struct spaden_tile_desc_s *spmm_tiles[3] = {};
     int64_t spmm_ntiles[3] = {};
     int spmm_state[3] = {};                    // 0 not built, 1 built, -1 unsupported
+    // tensor-core SpMM chunk schedule (spmm_tc.cu, built by the first spaden_spmm_tc call)
+    void *tc_chunks = nullptr;                 // [tc_nchunks] chunk descriptors
+    int32_t *tc_cta_start = nullptr;           // [tc_grid + 1] first chunk of each CTA
+    int tc_grid = 0;                           // CTAs the schedule was built for (0 = not built)
+    int64_t tc_nchunks = 0;
 
     // hybrid residual (csrc/hybrid.cu), empty in pure bitBSR mode: a CSR with
     // global columns, split into column segments (parts) when x is larger than
@@ -258,6 +263,11 @@ int spmv_launch_count(const Matrix &A, float beta);  // launches of one spmv_lau
 // SpMM: k column-major vectors (spmv.cu)
 spaden_status_t spmm_launch(Matrix &A, float alpha, const float *X, int64_t ldx, int k, float beta, float *Y,
                             int64_t ldy, cudaStream_t stream);
+
+// tensor-core SpMM (spmm_tc.cu)
+spaden_status_t spmm_tc_pack_x(int64_t n, int32_t k, const float *X, int64_t ldx, void *Xb, cudaStream_t stream);
+spaden_status_t spmm_tc_launch(Matrix &A, float alpha, const void *Xb, int32_t k, float beta, float *Y,
+                               int64_t ldy, cudaStream_t stream);  // builds the chunk schedule at the first call
 
 // exclusive scan of int32 (scan.cu): out[i] = sum_{j<i} in[j], out[count] = total.
 // `in` and `out` may alias.  tmp must hold scan_tmp_ints(count) int32.

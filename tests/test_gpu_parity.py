@@ -1152,3 +1152,53 @@ def test_hybrid_empty_residual_chained_calls(sp, torch):
         ys, s = oracle.spmv(A.rowptr, A.colidx, A.values, h1)
         ref = ys + y2_0.cpu().numpy().astype(np.float64)
         assert oracle.componentwise_error(y2.cpu().numpy(), ref, s + np.abs(y2_0.cpu().numpy())) <= TOL32
+
+
+# ------------------------------------------------- NEXT-4 tensor-core SpMM
+def _spmm_tc_case(name):
+    return {"fem": lambda: W.fem(7, 8, 9, seed=6), "hub": hub_matrix, "tiny": lambda: W.tiny(2),
+            "h2": W.h2, "ragged": lambda: W.random_sparse(333, 517, 0.02, 5),
+            "empty_rows": lambda: W.from_coo(90, 70, [0, 41, 89], [5, 69, 0], [1.5, -2.0, 3.0]),
+            "dense64": lambda: W.dense_block(64, 64, 2)}[name]()
+
+
+@pytest.mark.parametrize("k", [1, 64, 128, 200])
+@pytest.mark.parametrize("name", ["fem", "hub", "tiny", "h2", "ragged", "empty_rows", "dense64"])
+def test_spmm_tc_vs_oracle(sp, torch, name, k):
+    """tcgen05 SpMM (UTCHMMA, TMEM accumulators) against the fp64 oracle on the
+    stored fp16 values and fp16-rounded x (the paper's tensor-core input
+    precision): every column componentwise <= 1e-5, alpha/beta honoured,
+    rows of empty block-rows = beta*y."""
+    A = _spmm_tc_case(name)
+    M = convert(sp, torch, A, storage="fp16")
+    rng = np.random.default_rng(k)
+    X = rng.uniform(-1, 1, (k, A.n)).astype(np.float32)
+    Y0 = rng.uniform(-1, 1, (k, A.m)).astype(np.float32)
+    Xd = torch.from_numpy(X).cuda()
+    Xb = M.pack_x_tc(Xd)
+    Yd = torch.from_numpy(Y0).cuda()
+    M.spmm_tc(Xb, k, Yd, alpha=0.5, beta=0.25)
+    torch.cuda.synchronize()
+    Y = Yd.cpu().numpy()
+    vals = oracle.f32_to_f16(A.values)
+    for j in range(k):
+        xr = oracle.f32_to_f16(X[j]).astype(np.float64)
+        ys, s = oracle.spmv(A.rowptr, A.colidx, vals, xr)
+        ref = 0.5 * ys + 0.25 * Y0[j].astype(np.float64)
+        sc = 0.5 * s + 0.25 * np.abs(Y0[j].astype(np.float64))
+        err = oracle.componentwise_error(Y[j], ref, sc)
+        assert err <= TOL32, (j, err)
+
+
+def test_spmm_tc_deterministic_and_rejects(sp, torch):
+    A = W.fem(6, 7, 8, seed=2)
+    M = convert(sp, torch, A, storage="fp16")
+    X = torch.from_numpy(np.random.default_rng(1).uniform(-1, 1, (96, A.n)).astype(np.float32)).cuda()
+    Xb = M.pack_x_tc(X)
+    y1 = M.spmm_tc(Xb, 96)
+    y2 = M.spmm_tc(Xb, 96)
+    torch.cuda.synchronize()
+    assert torch.equal(y1, y2)
+    M32 = convert(sp, torch, A, storage="fp32")
+    with pytest.raises(sp.SpadenError):
+        M32.spmm_tc(Xb, 96)
