@@ -221,7 +221,7 @@ int default_tile_cfg(int64_t format_bytes, int value_bytes) {
     // x 3 x 24 KB, fp16 values 2 x 16 x 4 x 27 KB; small matrices need smaller stages to
     // give every CTA several tiles
     if (format_bytes < kSmallMatrixBytes) return kSmallTileCfg;
-    return value_bytes == 4 ? 2 : 15;
+    return 15;  // fp32 and fp16 values (fp32: cfg2 0.1151 ms, cfg15 0.1131 ms on fem1p5m)
 }
 
 spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {

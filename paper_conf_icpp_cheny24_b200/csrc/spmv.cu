@@ -534,6 +534,10 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
              const int32_t *__restrict__ blk_offset, const V *__restrict__ vals, const float *__restrict__ x,
              int nbc_vec, float alpha, float beta, float *__restrict__ y, int64_t ldx, int64_t ldy,
              const PeerOut po, unsigned long long texx, int wait_y, const uint8_t *__restrict__ rot) {
+    // a unit is BPL * 32 consecutive blocks: the slot decode handles two blocks per
+    // lane (the second block's x fetch is issued before the first is decoded)
+    constexpr int BPL = 1;  // 2 measured slower (fewer units per tile: fem1p5m fp32 0.1146 -> 0.1227 ms)
+    constexpr int UB = 32 * BPL;
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t full_bar[kMaxStages], empty_bar[kMaxStages];
     __shared__ StageHdr hdr[kMaxStages];
@@ -610,7 +614,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                 const uint32_t bytes = cur - stage;
                 h.a_part = cur;  // kPartStride bytes of row partials per block (not copied)
                 hdr[s] = h;
-                const int units = max(1, (h.nb + 31) >> 5);
+                const int units = max(1, (h.nb + UB - 1) / UB);
                 asm volatile("st.shared.v4.s32 [%0], {%1, %2, %3, %4};" ::"r"(smem_u32(&range[s])), "r"(U),
                              "r"(U + units), "r"((int)ph), "r"(0)
                              : "memory");  // one 16-byte store: consumers never see a torn range
@@ -637,7 +641,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
     int total = 0;
     for (int t = blockIdx.x + lane * gridDim.x; t < ntiles; t += 32 * gridDim.x) {
         const int2 bb = __ldg(reinterpret_cast<const int2 *>(tiles + t) + 1);  // b0, b1
-        total += max(1, (bb.y - bb.x + 31) >> 5);
+        total += max(1, (bb.y - bb.x + UB - 1) / UB);
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) total += __shfl_xor_sync(kFull, total, o);
@@ -668,7 +672,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
         const int4 h0 = lds_i4_volatile(a_hdr);
         const int4 h1 = lds_i4_volatile(a_hdr + 16u);
         const int v0 = h0.x, nb = h0.y;
-        const int units = max(1, (nb + 31) >> 5);
+        const int units = max(1, (nb + UB - 1) / UB);
         const uint32_t a_rot = (uint32_t)h0.z, a_val = (uint32_t)h0.w;
         const uint32_t a_bmp = h1.x, a_col = h1.y, a_off = h1.z, a_part = h1.w;
         const int ul = g - us;
@@ -692,6 +696,42 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             // into fp16 hi + lo parts (two MMAs) to keep ~22 bits of x.
             mma_unit(ul * 32, nb, lane, a_bmp, a_col, a_off, a_val, v0, a_part, x, nbc_vec);
         } else {
+            if constexpr (DEC == 1) {  // phase 1: BPL blocks per lane, all loads first
+                int lbs[BPL];
+                uint2 bms[BPL];
+                uint32_t ps[BPL], rhos[BPL];
+                XSeg xss[BPL];
+#pragma unroll
+                for (int h = 0; h < BPL; ++h) {
+                    const int lb = ul * UB + 32 * h + lane;
+                    lbs[h] = lb;
+                    if (lb < nb) {
+                        bms[h] = lds_u2(a_bmp + 8u * lb);
+                        const int bc = lds_i32(a_col + 4u * lb);
+                        ps[h] = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
+                        rhos[h] = ROT ? lds_u8(a_rot + (uint32_t)lb) : 0u;
+                        load_x(xss[h], x, bc, nbc_vec, used_cols(bms[h]), texx);
+                    }
+                }
+#pragma unroll
+                for (int h = 0; h < BPL; ++h) {
+                    const int lb = lbs[h];
+                    if (lb >= nb) continue;
+                    const uint32_t q = a_part + kPartStride * lb;
+                    if constexpr (ROT) {
+                        block_slots_rot<SmemVals<V>>(bms[h], rhos[h], ps[h], xss[h], q);
+                    } else {
+                        float acc[8];
+                        const uint2 bm = bms[h];
+                        const SwapHalves sw{sizeof(V) == 2 && ((lane >> 1) & 1)};
+                        const uint32_t plo = (uint32_t)__popc(bm.x) * (uint32_t)sizeof(V);
+                        block_slots_at<SmemVals<V>>(sw.bitmap(bm), sw.on ? ps[h] + plo : ps[h], sw.on ? ps[h] : ps[h] + plo,
+                                                    xss[h], acc);
+#pragma unroll
+                        for (int r = 0; r < 8; ++r) sts_f32(q + sw.part_off(r), acc[r]);
+                    }
+                }
+            } else {
             const int lb = ul * 32 + lane;
             if (lb < nb) {  // phase 1: one block per lane
                 const uint2 bm = lds_u2(a_bmp + 8u * lb);
@@ -699,10 +739,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                 const uint32_t p = a_val + (uint32_t)(lds_i32(a_off + 4u * lb) - v0) * (uint32_t)sizeof(V);
                 float acc[8];
                 const uint32_t q = a_part + kPartStride * lb;
-                if constexpr (DEC == 1 && ROT) {
-                    XSeg xs;
-                    load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
-                    block_slots_rot<SmemVals<V>>(bm, lds_u8(a_rot + (uint32_t)lb), p, xs, q);
+                if constexpr (false) {
                 } else if constexpr (DEC == 1) {
                     XSeg xs;
                     load_x(xs, x, bc, nbc_vec, used_cols(bm), texx);
@@ -716,6 +753,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
 #pragma unroll
                     for (int r = 0; r < 8; ++r) sts_f32(q + 4u * r, acc[r]);
                 }
+            }
             }
         }
         __syncwarp();

@@ -55,4 +55,18 @@ M = sp.convert(torch.from_numpy(A.rowptr).cuda(), torch.from_numpy(A.colidx).cud
 X = torch.from_numpy(np.stack([W.vector(A.n, k) for k in range(3)])).pin_memory()
 Y = torch.zeros((3, A.m)).pin_memory()
 M.spmv_host_batched(X, Y)
+# round 2: count pass, fused peer-store epilogue, tensor-core SpMM (fp16, k = 70)
+assert sp.count_blocks(torch.from_numpy(A.rowptr).cuda(), torch.from_numpy(A.colidx).cuda(), A.n) == M.info.Bnnz
+xd = torch.from_numpy(W.vector(A.n, 5)).cuda()
+peers = [torch.zeros(A.m + 8, device="cuda") for _ in range(3)]
+M.spmv_scatter(xd, [t.data_ptr() for t in peers], 4)
+for C in (A, B, W.h2()):
+    Mh = sp.convert(torch.from_numpy(C.rowptr).cuda(), torch.from_numpy(C.colidx).cuda(),
+                    torch.from_numpy(C.values).cuda(), C.n, storage="fp16")
+    Xk = torch.from_numpy(np.stack([W.vector(C.n, k) for k in range(70)])).cuda()
+    Xb = Mh.pack_x_tc(Xk)
+    Yk = torch.zeros((70, C.m), device="cuda")
+    Mh.spmm_tc(Xb, 70, Yk, alpha=0.5, beta=0.5)
+    torch.cuda.synchronize()
+    Mh.free()
 print("sanitize run ok")
