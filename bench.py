@@ -60,7 +60,7 @@ def parse():
     p.add_argument("--no-cusparse", action="store_true")
     p.add_argument("--no-variants", action="store_true", help="skip the other-precision kernel timing")
     p.add_argument("--spmm", default="4", help="comma list of right-hand-side counts for the SpMM extra ('' = skip)")
-    p.add_argument("--spmm-tc", default="128", help="comma list of right-hand-side counts for the tensor-core "
+    p.add_argument("--spmm-tc", default="64,128", help="comma list of right-hand-side counts for the tensor-core "
                                                    "SpMM extra (fp16 storage, tcgen05; '' = skip)")
     p.add_argument("--hybrid", type=int, default=-1,
                    help="hybrid format: blocks with <= HYBRID entries go to a CSR residual (0 = pure bitBSR, "

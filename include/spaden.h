@@ -236,14 +236,21 @@ SPADEN_API spaden_status_t spaden_spmm(spaden_matrix_t A, float alpha, const flo
                                        int32_t k, float beta, float *d_Y, int64_t ldy, void *stream);
 
 /*
- * spaden_spmm_tc_pack_x -- x slabs for spaden_spmm_tc: d_Xb[bc][j][c] =
- * fp16(d_X[j*ldx + 8*bc + c]) for block columns bc < ceil(n/8), vectors j < k,
- * c < 8 (round to nearest even; entries past n are 0).  d_X: float32,
+ * spaden_spmm_tc_pack_x -- x slabs for spaden_spmm_tc, in groups of 128
+ * vectors: d_Xb[g][bc][jj][c] = fp16(d_X[j*ldx + 8*bc + c]) with j = 128g + jj,
+ * for groups g < ceil(k/128), block columns bc < ceil(n/8), jj < 128, c < 8
+ * (round to nearest even; entries past n and vectors j >= k are 0).  The slabs
+ * of one group are contiguous across block columns, so the kernel fetches a
+ * run of consecutive block columns with one bulk copy.  d_X: float32,
  * column-major (vector j at d_X + j*ldx, ldx >= n).  d_Xb: DEVICE buffer of
- * 16 * ceil(n/8) * k bytes, 16-byte aligned, owned by the caller.  Stream-ordered.
+ * 2048 * ceil(n/8) * ceil(k/128) bytes (spaden_spmm_tc_xb_bytes), 16-byte
+ * aligned, owned by the caller.  Stream-ordered.
  */
 SPADEN_API spaden_status_t spaden_spmm_tc_pack_x(int64_t n, int32_t k, const float *d_X, int64_t ldx, void *d_Xb,
                                                  void *stream);
+
+/* Bytes of the slab buffer spaden_spmm_tc_pack_x fills for n columns and k vectors. */
+SPADEN_API int64_t spaden_spmm_tc_xb_bytes(int64_t n, int32_t k);
 
 /*
  * spaden_spmm_tc -- Y[:, j] = alpha * A X[:, j] + beta * Y[:, j], j < k, on the

@@ -84,6 +84,9 @@ spaden_spmm.restype = _ST
 spaden_spmm_tc_pack_x = _lib.spaden_spmm_tc_pack_x
 spaden_spmm_tc_pack_x.argtypes = [_I64, ctypes.c_int32, _P, _I64, _P, _P]
 spaden_spmm_tc_pack_x.restype = _ST
+spaden_spmm_tc_xb_bytes = _lib.spaden_spmm_tc_xb_bytes
+spaden_spmm_tc_xb_bytes.argtypes = [_I64, ctypes.c_int32]
+spaden_spmm_tc_xb_bytes.restype = _I64
 spaden_spmm_tc = _lib.spaden_spmm_tc
 spaden_spmm_tc.argtypes = [_P, _F, _P, ctypes.c_int32, _F, _P, _I64, _P]
 spaden_spmm_tc.restype = _ST
@@ -116,7 +119,7 @@ spaden_version.argtypes = []
 spaden_version.restype = ctypes.c_char_p
 
 EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_count_blocks", "spaden_spmv", "spaden_spmm",
-            "spaden_spmv_scatter", "spaden_spmm_tc_pack_x", "spaden_spmm_tc", "spaden_spmv_host", "spaden_spmv_host_batched",
+            "spaden_spmv_scatter", "spaden_spmm_tc_pack_x", "spaden_spmm_tc_xb_bytes", "spaden_spmm_tc", "spaden_spmv_host", "spaden_spmv_host_batched",
             "spaden_free",
             "spaden_get_info", "spaden_get_arrays", "spaden_spmv_launch_count", "spaden_status_string",
             "spaden_last_error_message", "spaden_version"]
@@ -264,11 +267,11 @@ class Matrix:
 
     def pack_x_tc(self, X, Xb=None, stream=None):
         """fp16 x slabs for spmm_tc (spaden_spmm_tc_pack_x): X is k x n (CUDA float32, rows
-        contiguous); returns a uint8 CUDA tensor of 16 * ceil(n/8) * k bytes."""
+        contiguous); returns a uint8 CUDA tensor of 2048 * ceil(n/8) * ceil(k/128) bytes."""
         torch = _torch()
         k = X.shape[0]
         assert X.dtype == torch.float32 and X.is_cuda and X.shape[1] == self.n and X.stride(1) == 1
-        nbytes = 16 * ((self.n + 7) // 8) * k
+        nbytes = int(spaden_spmm_tc_xb_bytes(self.n, k))
         if Xb is None:
             Xb = torch.empty(max(16, nbytes), dtype=torch.uint8, device=X.device)
         assert Xb.numel() >= nbytes and Xb.is_cuda

@@ -280,6 +280,11 @@ spaden_status_t spaden_spmm(spaden_matrix_t A, float alpha, const float *d_X, in
     return spmm_launch(*A, alpha, d_X, ldx, k, beta, d_Y, ldy, (cudaStream_t)stream);
 }
 
+int64_t spaden_spmm_tc_xb_bytes(int64_t n, int32_t k) {
+    if (n <= 0 || k <= 0) return 0;
+    return 2048 * ((n + 7) / 8) * (((int64_t)k + 127) / 128);
+}
+
 spaden_status_t spaden_spmm_tc_pack_x(int64_t n, int32_t k, const float *d_X, int64_t ldx, void *d_Xb,
                                       void *stream) {
     g_last_error.clear();
@@ -302,7 +307,7 @@ spaden_status_t spaden_spmm_tc(spaden_matrix_t A, float alpha, const void *d_Xb,
         return SPADEN_ERR_UNSUPPORTED;
     }
     if (k > 0 && A->m > 0 && A->n > 0) {
-        const char *xb = (const char *)d_Xb, *xe = xb + 16 * ((A->n + 7) / 8) * (int64_t)k;
+        const char *xb = (const char *)d_Xb, *xe = xb + spaden_spmm_tc_xb_bytes(A->n, k);
         const char *yb = (const char *)d_Y, *ye = (const char *)(d_Y + (int64_t)(k - 1) * ldy + A->m);
         if (xb < ye && yb < xe) {
             set_error("X slabs and Y must not overlap");

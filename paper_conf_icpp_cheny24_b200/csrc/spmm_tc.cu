@@ -32,21 +32,30 @@
 // consecutive blocks [B0, B1); block-rows [brA, brE) end in it, a block-row
 // may start in an earlier chunk (pair pA) and continue into the next (pE).
 // Roles per CTA:
-//   warp 13    producer lane: bulk-copies the chunk's blk_rowptr, bitmap,
-//              blk_col, blk_offset and value slices (4-chunk ring) and, one
-//              chunk behind, walks the staged blk_rowptr into the chunk's MMA
-//              list and the list of block-rows ending in it;
-//   warps 4-11 copy the x slabs of the chunk's blocks (cp.async, 3 slab
-//              buffers) and decode the blocks into dense tiles (4-chunk ring);
-//   warp 12    TMEM allocation + the MMA issue thread;
+//   warp 13    producer lane: bulk-copies the chunk's MMA record (TcRec,
+//              precomputed with the schedule), blk_rowptr, bitmap, blk_col,
+//              blk_offset and value slices (4-chunk ring);
+//   warp 14    x slabs: once a chunk's arrays have landed, its lanes issue one
+//              cp.async.bulk per block (3 slab buffers);
+//   warps 4-11 decode the blocks into dense tiles (4-chunk ring);
+//   warps 12, 15  MMA issue, alternate chunks (warp 12 also allocates TMEM): one elected lane issues the MMAs
+//              (pair o's descriptors are base + o * stride: blocks sit in pair
+//              order, see TcRec; the per-block-row slot comes through redux.sync
+//              so every MMA operand is warp-uniform);
 //   warps 0-3  epilogue (TMEM lanes 32w..32w+31 = vectors): tcgen05.ld of the
 //              accumulators of the block-rows ending in the chunk, alpha*D +
 //              beta*Y written as two 16-byte stores per vector and block-row.
-// mbarriers per ring slot: arrays landed, MMA list written, tiles written,
-// MMAs complete (tcgen05.commit: tiles free + accumulators ready), epilogue
-// done; per slab buffer: slab copies landed (cp.async.mbarrier.arrive), MMAs
+// mbarriers per ring slot: arrays landed, arrays free (epilogue done with the
+// record), tiles written, MMAs complete (tcgen05.commit: tiles free +
+// accumulators ready), epilogue done; per slab buffer: slabs landed, MMAs
 // reading it complete.  The MMAs of chunk c wait for the epilogue of chunk
 // c-3, so at most 3 * kTcPairs < kTcSlots accumulators are live.
+// History (fem1p5m, K = 128, per chunk of ~13 MMAs): a producer lane walking
+// blk_rowptr into the MMA list at run time set the pace (1.81 ms); moving the
+// walk to the schedule left the MMA lane at ~100 cycles per MMA (a per-MMA
+// ELECT loop for non-uniform operands) and the decode warps busy with 16-byte
+// cp.async slab pieces and a proxy fence per chunk (traced with
+// -DSPADEN_TC_TRACE, tools/tc_trace.py).
 #include <algorithm>
 
 #include "internal.cuh"
@@ -62,14 +71,15 @@ constexpr int kTcRows = 48;       // block-rows touched by one chunk (incl. empt
 constexpr int kTcSlots = 64;      // TMEM accumulator slots (8 columns each, 512 columns)
 constexpr int kSlabBytes = kTcM * 16;
 constexpr int kTileBytes = 128;
-constexpr int kTcArrBytes = 5120; // one chunk's staged arrays (brp, bitmap, blk_col, blk_offset, values)
+constexpr int kTcRecBytes = 160;  // a chunk's MMA record (TcRec)
+constexpr int kTcArrBytes = 5120; // one chunk's staged arrays (record, brp, bitmap, blk_col, blk_offset, values)
 constexpr int kTcRing = 4;        // arrays, tiles and accumulator hand-off: 4 chunks in flight
 constexpr int kTcSlabBufs = 3;    // x slabs: 3 chunks (the big buffers)
 constexpr int kTcDecodeWarps = 8;
 constexpr int kTcSlabBytes = kTcBlocks * kSlabBytes;
 constexpr int kTcTileBytes = kTcBlocks * kTileBytes;
-constexpr int kTcSmem = kTcSlabBufs * kTcSlabBytes + kTcRing * (kTcTileBytes + kTcArrBytes) + kSlabBytes + kTileBytes;
-constexpr int kTcThreads = (4 + kTcDecodeWarps + 2) * 32;
+constexpr int kTcSmem = kTcSlabBufs * kTcSlabBytes + kTcRing * (kTcTileBytes + kTcArrBytes);
+constexpr int kTcThreads = (4 + kTcDecodeWarps + 4) * 32;
 
 // one chunk of the schedule (48 bytes)
 struct alignas(16) TcChunk {
@@ -80,6 +90,46 @@ struct alignas(16) TcChunk {
     int V0, V1;      // values [V0, V1) = blk_offset[B0], blk_offset[B1]
     int pad0, pad1, pad2;
 };
+
+// A chunk's MMAs and finished block-rows, precomputed with the schedule and
+// staged with the chunk's arrays (so no thread walks blk_rowptr at run time).
+// The chunk's blocks are placed in *pair order*: pair o of the chunk uses tile
+// and slab positions 2o, 2o+1 (a block-row's lone last block has a zero tile
+// as partner), so the MMA descriptors of pair o are base + o * stride and the
+// issue loop needs no per-MMA operand from memory.
+//   seg[s]  = slot | accumulate << 6 | pairs << 7  (the s-th non-empty block-row
+//             of the chunk: TMEM slot, whether it continues an earlier chunk's
+//             accumulation, its pairs in this chunk)
+//   lone    = bit o: pair o has no second block
+//   pos[q]  = position of the chunk's block q
+//   end[e]  = i | (slot + 1) << 6  (block-row brA + i ends in the chunk; 0 = empty row)
+struct alignas(16) TcRec {
+    uint8_t nseg, nends;
+    uint16_t lone;
+    uint16_t seg[kTcPairs];
+    uint8_t pos[kTcBlocks];
+    uint16_t end[kTcRows];
+};
+static_assert(sizeof(TcRec) == kTcRecBytes && offsetof(TcRec, seg) == 4 && offsetof(TcRec, pos) == 34 &&
+                  offsetof(TcRec, end) == 64,
+              "TcRec layout");
+// worst case of one chunk's staged regions (each rounded out to 16 bytes on both ends)
+static_assert(kTcRecBytes + (4 * (kTcRows + 1) + 30) + (8 * kTcBlocks + 30) + 2 * (4 * kTcBlocks + 30) +
+                      (2 * 64 * kTcBlocks + 30) <= kTcArrBytes,
+              "kTcArrBytes too small");
+
+#ifdef SPADEN_TC_TRACE  // experiment builds only (tools/exp_build.sh): per-role timestamps of CTA 0
+__device__ long long *g_tc_trace;
+constexpr int kTrChunks = 512, kTrEv = 8;
+#define TR(role, c, ev)                                                                         \
+    do {                                                                                        \
+        if (trp && (c) < kTrChunks) trp[((role) * kTrChunks + (c)) * kTrEv + (ev)] = clock64(); \
+    } while (0)
+#else
+#define TR(role, c, ev) \
+    do {                \
+    } while (0)
+#endif
 
 __device__ __forceinline__ uint32_t s_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void tc_mbar_init(uint32_t bar, uint32_t count) {
@@ -107,6 +157,11 @@ __device__ __forceinline__ void tc_bulk(uint32_t dst, const void *src, uint32_t 
         "l"(src), "r"(bytes), "r"(bar)
         : "memory");
 }
+__device__ __forceinline__ uint32_t tc_lds8(uint32_t a) {
+    uint16_t v;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=h"(v) : "r"(a) : "memory");
+    return v;
+}
 __device__ __forceinline__ uint32_t tc_lds(uint32_t a) {
     uint32_t v;
     asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
@@ -117,20 +172,26 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t addr, uint32_t lbo, uint3
     return (uint64_t)((addr & 0x3FFFFu) >> 4) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |
            ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | (1ull << 46);
 }
+// high word of every descriptor here (SBO = 128 bytes, version 1): the MMA
+// lists carry only the low words
+constexpr uint32_t kDescHi = ((128u >> 4) & 0x3FFFu) | (1u << 14);
 // instruction descriptor: kind::f16, A = B = F16 (K-major), D = F32, M = 128, N = 8
 constexpr uint32_t kTcIdesc = (1u << 4) | ((uint32_t)(kTcN >> 3) << 17) | ((uint32_t)(kTcM >> 4) << 24);
 
-__device__ __forceinline__ void umma_f16(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t accumulate) {
+// issued by the whole (converged) warp, one elected lane executes the MMA; the
+// operands must be warp-uniform (see the MMA warp: passed through redux.sync,
+// whose result ptxas keeps in uniform registers, so no per-MMA ELECT loop)
+__device__ __forceinline__ void umma_f16_elect(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t accumulate) {
     asm volatile(
-        "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
-        " tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
+        "{\n .reg .pred p, e;\n setp.ne.b32 p, %4, 0;\n elect.sync _|e, 0xffffffff;\n"
+        " @e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
         "l"(adesc), "l"(bdesc), "r"(kTcIdesc), "r"(accumulate)
         : "memory");
 }
 
 // staged arrays of a chunk inside its buffer (16-byte aligned regions)
 struct TcArr {
-    uint32_t brp, bmp, col, off, val;  // shared addresses of element 0 of each slice
+    uint32_t brp, bmp, col, off, val, rec;  // shared addresses of element 0 of each slice, of the record
 };
 
 // Chunk schedule (built once per handle on the GPU).  Block-rows are grouped in
@@ -204,125 +265,129 @@ __global__ void k_tc_sched(const int32_t *__restrict__ brp, const int32_t *__res
     }
 }
 
+// one thread per chunk: its MMA record (the block-rows it touches, in order)
+__global__ void k_tc_ops(const int32_t *__restrict__ brp, const TcChunk *__restrict__ chunks, int64_t nchunks,
+                         TcRec *__restrict__ recs) {
+    const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nchunks) return;
+    const TcChunk ch = chunks[c];
+    TcRec r;
+    const int rows = ch.brE - ch.brA + (ch.pE > 0 ? 1 : 0);
+    int seq = ch.seq0, ne = 0, ns = 0, o = 0;
+    r.lone = 0;
+    for (int q = 0; q < kTcBlocks; ++q) r.pos[q] = 0;
+    for (int i = 0; i < rows; ++i) {
+        const int s0 = brp[ch.brA + i], nb = brp[ch.brA + i + 1] - s0;
+        const int slot = seq % kTcSlots;
+        if (ch.brA + i < ch.brE) r.end[ne++] = (uint16_t)(i | ((nb ? slot + 1 : 0) << 6));
+        if (nb == 0) continue;
+        const int npr = (nb + 1) >> 1;
+        const int pb = i == 0 ? ch.pA : 0;
+        const int pe = (ch.brA + i < ch.brE) ? npr : ch.pE;
+        r.seg[ns++] = (uint16_t)(slot | ((pb > 0 ? 1 : 0) << 6) | ((pe - pb) << 7));
+        for (int p = pb; p < pe; ++p, ++o) {
+            const int q1 = s0 + 2 * p - ch.B0;
+            r.pos[q1] = (uint8_t)(2 * o);
+            if (2 * p + 1 < nb) r.pos[q1 + 1] = (uint8_t)(2 * o + 1);
+            else r.lone |= (uint16_t)(1u << o);
+        }
+        if (ch.brA + i < ch.brE) ++seq;
+    }
+    r.nseg = (uint8_t)ns;
+    r.nends = (uint8_t)ne;
+    for (int e = ne; e < kTcRows; ++e) r.end[e] = 0;
+    for (int t = ns; t < kTcPairs; ++t) r.seg[t] = 0;
+    const uint4 *src = reinterpret_cast<const uint4 *>(&r);
+    uint4 *dst = reinterpret_cast<uint4 *>(recs + c);
+#pragma unroll
+    for (int w = 0; w < kTcRecBytes / 16; ++w) dst[w] = src[w];
+}
+
 __global__ void __launch_bounds__(kTcThreads, 1)
-k_spmm_tc(int64_t m, const TcChunk *__restrict__ chunks, const int32_t *__restrict__ cta_start,
+k_spmm_tc(int64_t m, const TcChunk *__restrict__ chunks, const TcRec *__restrict__ recs,
+          const int32_t *__restrict__ cta_start,
           const int32_t *__restrict__ brp, const int32_t *__restrict__ bcol, const uint64_t *__restrict__ bitmap,
           const int32_t *__restrict__ boff, const __half *__restrict__ vals, const __half *__restrict__ Xb,
-          int32_t k, int32_t j0, int32_t kv, float alpha, float beta, float *__restrict__ Y, int64_t ldy) {
+          int64_t nbcx, int32_t j0, int32_t kv, float alpha, float beta, float *__restrict__ Y, int64_t ldy) {
     extern __shared__ __align__(1024) unsigned char smem[];
     __shared__ TcChunk cdesc[kTcRing];
     __shared__ TcArr arr[kTcRing];
     // a = c % kTcRing (arrays, tiles, accumulator hand-off), b = c % kTcSlabBufs (x slabs)
     __shared__ __align__(8) uint64_t bar_arr[kTcRing];    // arrays landed (producer, tx)
-    __shared__ __align__(8) uint64_t bar_afree[kTcRing];  // arrays of chunk c no longer read (MMA issued)
+    __shared__ __align__(8) uint64_t bar_afree[kTcRing];  // arrays of chunk c no longer read (4 epilogue warps)
     __shared__ __align__(8) uint64_t bar_epi[kTcRing];    // epilogue done with chunk c (4 warps)
-    __shared__ int2 ends[kTcRing][kTcRows];               // (block-row, slot or -1) ending in chunk c
-    __shared__ int nends[kTcRing];
-    __shared__ uint4 ops[kTcRing][kTcPairs][2];           // the chunk's MMAs: (adesc, bdesc), (d, accumulate)
-    __shared__ int nops[kTcRing];
-    __shared__ __align__(8) uint64_t bar_ops[kTcRing];    // MMA list and ends of chunk c written (producer)
     __shared__ __align__(8) uint64_t bar_tiles[kTcRing];  // tiles decoded (decode warps)
     __shared__ __align__(8) uint64_t bar_mma[kTcRing];    // chunk's MMAs complete (commit): tiles free,
                                                           // accumulators ready
     __shared__ __align__(8) uint64_t bar_sfree[kTcSlabBufs];  // MMAs reading the slabs complete (commit)
-    __shared__ __align__(8) uint64_t bar_slab[kTcSlabBufs];   // slab cp.asyncs landed (every decode thread)
+    __shared__ __align__(8) uint64_t bar_slab[kTcSlabBufs];   // slab bulk copies landed (producer, tx)
     __shared__ uint32_t tmem_base_sh;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t sb = s_u32(smem);
     const uint32_t tiles0 = sb + (uint32_t)kTcSlabBufs * kTcSlabBytes;
     const uint32_t arr0 = tiles0 + (uint32_t)kTcRing * kTcTileBytes;
-    const uint32_t zero_slab = arr0 + (uint32_t)kTcRing * kTcArrBytes, zero_tile = zero_slab + kSlabBytes;
     const int c0 = cta_start[blockIdx.x], nch = cta_start[blockIdx.x + 1] - c0;
-    const int kMma = 4 + kTcDecodeWarps, kProd = kMma + 1;
+    const int kMma = 4 + kTcDecodeWarps, kProd = kMma + 1, kSlab = kMma + 2, kMma2 = kMma + 3;
 
     if (threadIdx.x == 0) {
         for (int a = 0; a < kTcRing; ++a) {
             tc_mbar_init(s_u32(&bar_arr[a]), 1);
-            tc_mbar_init(s_u32(&bar_afree[a]), 1);
-            tc_mbar_init(s_u32(&bar_ops[a]), 1);
+            tc_mbar_init(s_u32(&bar_afree[a]), 4);
             tc_mbar_init(s_u32(&bar_epi[a]), 4);
             tc_mbar_init(s_u32(&bar_tiles[a]), kTcDecodeWarps);
-            tc_mbar_init(s_u32(&bar_mma[a]), 2);  // tcgen05.commit + the MMA thread's own arrive (ends list)
+            tc_mbar_init(s_u32(&bar_mma[a]), 1);  // tcgen05.commit
         }
         for (int b = 0; b < kTcSlabBufs; ++b) {
             tc_mbar_init(s_u32(&bar_sfree[b]), 1);
-            tc_mbar_init(s_u32(&bar_slab[b]), kTcDecodeWarps * 32);
+            tc_mbar_init(s_u32(&bar_slab[b]), 1);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    // zero slab + zero tile (the partner of a block-row's lone last block)
-    for (int i = threadIdx.x; i < (kSlabBytes + kTileBytes) / 16; i += blockDim.x)
-        asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(zero_slab + 16u * i), "r"(0u) : "memory");
+    // the slab buffers start zeroed: a lone block's partner position (zero tile)
+    // then only ever holds zeros or earlier finite slabs, never NaN patterns
+    for (int i = threadIdx.x; i < kTcSlabBufs * kTcSlabBytes / 16; i += blockDim.x)
+        asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(sb + 16u * i), "r"(0u) : "memory");
     if (warp == kMma) {  // TMEM: 512 columns = kTcSlots accumulators of 8 fp32 columns
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(s_u32(&tmem_base_sh))
                      : "memory");
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
     }
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // zero slab/tile -> tensor core
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // zeroed slabs -> tensor core
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     __syncthreads();
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#ifdef SPADEN_TC_TRACE
+    long long *const trp = blockIdx.x == 0 ? g_tc_trace : nullptr;
+#endif
     const uint32_t tmem = tmem_base_sh;
+    const uint32_t tmem_u = __reduce_or_sync(0xffffffffu, tmem);  // warp-uniform copy (MMA operands)
     auto slab_of = [&](int b, int q) { return sb + (uint32_t)b * kTcSlabBytes + (uint32_t)q * kSlabBytes; };
     auto tile_of = [&](int a, int q) { return tiles0 + (uint32_t)a * kTcTileBytes + (uint32_t)q * kTileBytes; };
     auto ring_ph = [](int c) { return (uint32_t)((c / kTcRing) & 1); };
     auto slab_ph = [](int c) { return (uint32_t)((c / kTcSlabBufs) & 1); };
 
-    if (warp == kProd) {  // ------------------------------- producer: arrays, then x slabs
-        if (lane == 0) {
-            // the MMA list and the block-rows ending in chunk cw (walk of its staged
-            // blk_rowptr, one chunk behind the copies); ops / ends of its ring slot were
-            // last read by the MMA thread and the epilogue of chunk cw - kTcRing
-            auto walk = [&](int cw) {
-                const int a = cw % kTcRing, b = cw % kTcSlabBufs;
-                tc_wait(s_u32(&bar_arr[a]), ring_ph(cw));
-                if (cw >= kTcRing) tc_wait(s_u32(&bar_epi[a]), ring_ph(cw - kTcRing));
-                const TcChunk ch = cdesc[a];
-                const TcArr ar = arr[a];
-                const int rows = ch.brE - ch.brA + (ch.pE > 0 ? 1 : 0);
-                int seq = ch.seq0, ne = 0, no = 0;
-                for (int i = 0; i < rows; ++i) {
-                    const int s0 = (int)tc_lds(ar.brp + 4u * i), nb = (int)tc_lds(ar.brp + 4u * i + 4u) - s0;
-                    if (ch.brA + i < ch.brE) ends[a][ne++] = make_int2(ch.brA + i, nb ? seq % kTcSlots : -1);
-                    if (nb == 0) continue;
-                    const int npr = (nb + 1) >> 1;
-                    const int pb = i == 0 ? ch.pA : 0;
-                    const int pe = (ch.brA + i < ch.brE) ? npr : ch.pE;
-                    const uint32_t d = tmem + (uint32_t)((seq % kTcSlots) * kTcN);
-                    for (int p = pb; p < pe; ++p) {
-                        const int q1 = s0 + 2 * p - ch.B0;
-                        const bool two = 2 * p + 1 < nb;
-                        const uint32_t s1 = slab_of(b, q1), t1 = tile_of(a, q1);
-                        const uint32_t s2 = two ? slab_of(b, q1 + 1) : zero_slab;
-                        const uint32_t t2 = two ? tile_of(a, q1 + 1) : zero_tile;
-                        const uint64_t ad = umma_desc(s1, s2 - s1, 128u), bd = umma_desc(t1, t2 - t1, 128u);
-                        ops[a][no][0] = make_uint4((uint32_t)ad, (uint32_t)(ad >> 32), (uint32_t)bd, (uint32_t)(bd >> 32));
-                        ops[a][no][1] = make_uint4(d, p > 0 ? 1u : 0u, 0u, 0u);
-                        ++no;
-                    }
-                    if (ch.brA + i < ch.brE) ++seq;
-                }
-                nends[a] = ne;
-                nops[a] = no;
-                tc_arrive(s_u32(&bar_ops[a]));
-            };
-            TcChunk next = nch > 0 ? chunks[c0] : TcChunk{};  // descriptors one chunk ahead
-            for (int c = 0; c < nch; ++c) {
+    if (warp == kProd) {  // ---------------------------------------------- producer: arrays
+        TcChunk next = nch > 0 ? chunks[c0] : TcChunk{};  // descriptors one chunk ahead
+        for (int c = 0; c < nch; ++c) {
+            if (lane == 0) {  // the chunk's record and array slices (one lane)
                 const int a = c % kTcRing;
                 const TcChunk ch = next;
                 if (c + 1 < nch) next = chunks[c0 + c + 1];
+                TR(0, c, 0);
                 if (c >= kTcRing) tc_wait(s_u32(&bar_afree[a]), ring_ph(c - kTcRing));
+                TR(0, c, 1);
                 cdesc[a] = ch;
                 const int nrows = ch.brE - ch.brA + (ch.pE > 0 ? 1 : 0);
                 const int v0 = ch.V0, v1 = ch.V1;
                 uint32_t cur = arr0 + (uint32_t)a * kTcArrBytes;
                 uint32_t total = 0;
-                const void *srcs[5] = {brp + ch.brA, bitmap + ch.B0, bcol + ch.B0, boff + ch.B0, vals + v0};
-                const uint32_t lens[5] = {4u * (uint32_t)(nrows + 1), 8u * (uint32_t)(ch.B1 - ch.B0),
-                                          4u * (uint32_t)(ch.B1 - ch.B0), 4u * (uint32_t)(ch.B1 - ch.B0),
-                                          2u * (uint32_t)(v1 - v0)};
-                uint32_t addr[5], asrc[5], asz[5];
-                for (int r = 0; r < 5; ++r) {
+                const void *srcs[6] = {recs + c0 + c, brp + ch.brA, bitmap + ch.B0, bcol + ch.B0, boff + ch.B0,
+                                       vals + v0};
+                const uint32_t lens[6] = {(uint32_t)kTcRecBytes, 4u * (uint32_t)(nrows + 1),
+                                          8u * (uint32_t)(ch.B1 - ch.B0), 4u * (uint32_t)(ch.B1 - ch.B0),
+                                          4u * (uint32_t)(ch.B1 - ch.B0), 2u * (uint32_t)(v1 - v0)};
+                uint32_t addr[6], asrc[6], asz[6];
+                for (int r = 0; r < 6; ++r) {
                     const uintptr_t lo = (uintptr_t)srcs[r];
                     const uintptr_t alo = lo & ~(uintptr_t)15;
                     asz[r] = lens[r] ? (uint32_t)(((lo + lens[r] + 15) & ~(uintptr_t)15) - alo) : 0u;
@@ -331,102 +396,167 @@ k_spmm_tc(int64_t m, const TcChunk *__restrict__ chunks, const int32_t *__restri
                     cur += asz[r];
                     total += asz[r];
                 }
-                arr[a] = TcArr{addr[0], addr[1], addr[2], addr[3], addr[4]};
+                arr[a] = TcArr{addr[1], addr[2], addr[3], addr[4], addr[5], addr[0]};
                 const uint32_t fb = s_u32(&bar_arr[a]);
                 tc_arrive_tx(fb, total);
                 uint32_t dst = arr0 + (uint32_t)a * kTcArrBytes;
-                for (int r = 0; r < 5; ++r) {
+                for (int r = 0; r < 6; ++r) {
                     if (asz[r]) tc_bulk(dst, (const void *)((uintptr_t)srcs[r] - asrc[r]), asz[r], fb);
                     dst += asz[r];
                 }
-                if (c >= 1) walk(c - 1);
+                TR(0, c, 2);
             }
-            if (nch > 0) walk(nch - 1);
+        }
+    } else if (warp == kSlab) {  // ------------------------------------------------ x slabs
+        for (int cs = 0; cs < nch; ++cs) {
+            {  // one bulk copy per block, lane per block
+                const int a = cs % kTcRing, b = cs % kTcSlabBufs;
+                tc_wait(s_u32(&bar_arr[a]), ring_ph(cs));
+                if (cs >= kTcSlabBufs) tc_wait(s_u32(&bar_sfree[b]), slab_ph(cs - kTcSlabBufs));
+                const TcArr ar = arr[a];
+                const int nblk = cdesc[a].B1 - cdesc[a].B0;
+                const uint32_t sbar = s_u32(&bar_slab[b]);
+                if (lane == 0) tc_arrive_tx(sbar, (uint32_t)nblk * (uint32_t)kSlabBytes);
+                __syncwarp();
+                // runs of consecutive block columns at consecutive positions are one copy
+                // (a group's slabs are adjacent in Xb)
+                const __half *xg = Xb + (int64_t)(j0 / kTcM) * nbcx * (kTcM * 8);
+                for (int q = lane; q < nblk; q += 32) {
+                    const int bc = (int)tc_lds(ar.col + 4u * q);
+                    const int pos = (int)tc_lds8(ar.rec + 34u + (uint32_t)q);
+                    auto continues = [&](int r, int bcr, int posr) {  // block r extends block r-1's run
+                        return (int)tc_lds(ar.col + 4u * (r - 1)) == bcr - 1 &&
+                               (int)tc_lds8(ar.rec + 34u + (uint32_t)(r - 1)) == posr - 1;
+                    };
+                    if (q > 0 && continues(q, bc, pos)) continue;  // inside a run
+                    int len = 1;
+                    while (q + len < nblk) {
+                        const int r = q + len;
+                        if (!continues(r, (int)tc_lds(ar.col + 4u * r), (int)tc_lds8(ar.rec + 34u + (uint32_t)r))) break;
+                        ++len;
+                    }
+                    tc_bulk(slab_of(b, pos), xg + (int64_t)bc * (kTcM * 8), (uint32_t)(len * kSlabBytes), sbar);
+                }
+            }
         }
     } else if (warp >= 4 && warp < kMma) {  // --------------------------------- decode
         const int dw = warp - 4;
         for (int c = 0; c < nch; ++c) {
-            const int a = c % kTcRing, b = c % kTcSlabBufs;
+            const int a = c % kTcRing;
+            if (lane == 0 && dw == 0) TR(1, c, 0);
             tc_wait(s_u32(&bar_arr[a]), ring_ph(c));
+            if (lane == 0 && dw == 0) TR(1, c, 1);
             const TcChunk ch = cdesc[a];
             const TcArr ar = arr[a];
             const int nblk = ch.B1 - ch.B0;
-            // x slabs: cp.async by the decode warps, a warp per block's slab (16 bytes per
-            // lane and step); many small bulk copies serialise in the copy engine
-            if (c >= kTcSlabBufs) tc_wait(s_u32(&bar_sfree[b]), slab_ph(c - kTcSlabBufs));
-            {
-                // this warp's blocks q = dw + 8i: all their pieces in flight at once
-                // (distinct address registers: an LDGSTS holds its operands until
-                // the data returns, so a reused register would serialise the slabs)
-                constexpr int kPer = (kTcBlocks + kTcDecodeWarps - 1) / kTcDecodeWarps;
-                uint64_t srcs[kPer];
-                uint32_t dsts[kPer];
-#pragma unroll
-                for (int i = 0; i < kPer; ++i) {
-                    const int q = dw + kTcDecodeWarps * i;
-                    const int bc = q < nblk ? (int)tc_lds(ar.col + 4u * q) : 0;
-                    srcs[i] = (uint64_t)(Xb + ((int64_t)bc * k + j0) * 8);
-                    dsts[i] = slab_of(b, q);
-                }
-#pragma unroll
-                for (int r = 0; r < kTcM / 32; ++r) {
-                    const int piece = lane + 32 * r;
-#pragma unroll
-                    for (int i = 0; i < kPer; ++i) {
-                        if (dw + kTcDecodeWarps * i < nblk && piece < kv)
-                            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dsts[i] + 16u * piece),
-                                         "l"(srcs[i] + 16ull * piece)
-                                         : "memory");
-                    }
-                }
-                // the slab buffer's barrier completes when every decode thread's copies
-                // have landed; the decode warps move on without waiting
-                asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(s_u32(&bar_slab[b]))
-                             : "memory");
-            }
+            if (lane == 0 && dw == 0) TR(1, c, 3);
             if (c >= kTcRing) tc_wait(s_u32(&bar_mma[a]), ring_ph(c - kTcRing));  // tile slot free
+            if (lane == 0 && dw == 0) TR(1, c, 4);
             const int v0 = (int)tc_lds(ar.off);  // blk_offset of the chunk's first block
-            // a warp per block, lane l -> bits 2l, 2l+1 (row l/4, columns 2(l%4), 2(l%4)+1)
-            for (int q = dw; q < nblk; q += kTcDecodeWarps) {
-                const uint32_t lo = tc_lds(ar.bmp + 8u * q), hi = tc_lds(ar.bmp + 8u * q + 4u);
-                const uint64_t bm = ((uint64_t)hi << 32) | lo;
-                const int off = (int)tc_lds(ar.off + 4u * q) - v0;
-                const int bit = 2 * lane;
-                const uint32_t two = (uint32_t)(bm >> bit) & 3u;
-                uint32_t word = 0;
-                if (two) {
-                    const int idx = off + __popcll(bm & ((1ull << bit) - 1ull));
-                    const uint32_t a0 = ar.val + 2u * (uint32_t)idx;
-                    uint16_t h0 = 0, h1 = 0;
-                    if (two & 1u) asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h0) : "r"(a0) : "memory");
-                    if (two & 2u)
-                        asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h1) : "r"(a0 + 2u * (two & 1u)) : "memory");
-                    word = (uint32_t)h0 | ((uint32_t)h1 << 16);
-                }
-                asm volatile("st.shared.u32 [%0], %1;" ::"r"(tile_of(a, q) + 4u * lane), "r"(word) : "memory");
+            // a warp per block, lane l -> bits 2l, 2l+1 (row l/4, columns 2(l%4), 2(l%4)+1);
+            // two blocks per step (q, q + 8) so their shared-memory chains overlap
+            const int bit = 2 * lane;
+            for (int q0 = dw; q0 < nblk; q0 += 2 * kTcDecodeWarps) {
+                const int q1 = q0 + kTcDecodeWarps;
+                const bool has1 = q1 < nblk;
+                const uint32_t lo0 = tc_lds(ar.bmp + 8u * q0), hi0 = tc_lds(ar.bmp + 8u * q0 + 4u);
+                const uint32_t lo1 = has1 ? tc_lds(ar.bmp + 8u * q1) : 0u, hi1 = has1 ? tc_lds(ar.bmp + 8u * q1 + 4u) : 0u;
+                const int off0 = (int)tc_lds(ar.off + 4u * q0) - v0;
+                const int off1 = has1 ? (int)tc_lds(ar.off + 4u * q1) - v0 : 0;
+                const uint32_t pos0 = tc_lds8(ar.rec + 34u + (uint32_t)q0);
+                const uint32_t pos1 = has1 ? tc_lds8(ar.rec + 34u + (uint32_t)q1) : 0u;
+                const uint64_t bm0 = ((uint64_t)hi0 << 32) | lo0, bm1 = ((uint64_t)hi1 << 32) | lo1;
+                const uint32_t two0 = (uint32_t)(bm0 >> bit) & 3u, two1 = (uint32_t)(bm1 >> bit) & 3u;
+                const uint32_t a0 = ar.val + 2u * (uint32_t)(off0 + __popcll(bm0 & ((1ull << bit) - 1ull)));
+                const uint32_t a1 = ar.val + 2u * (uint32_t)(off1 + __popcll(bm1 & ((1ull << bit) - 1ull)));
+                uint16_t h00 = 0, h01 = 0, h10 = 0, h11 = 0;
+                if (two0 & 1u) asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h00) : "r"(a0) : "memory");
+                if (two0 & 2u) asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h01) : "r"(a0 + 2u * (two0 & 1u)) : "memory");
+                if (two1 & 1u) asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h10) : "r"(a1) : "memory");
+                if (two1 & 2u) asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h11) : "r"(a1 + 2u * (two1 & 1u)) : "memory");
+                asm volatile("st.shared.u32 [%0], %1;" ::"r"(tile_of(a, (int)pos0) + 4u * lane),
+                             "r"((uint32_t)h00 | ((uint32_t)h01 << 16))
+                             : "memory");
+                if (has1)
+                    asm volatile("st.shared.u32 [%0], %1;" ::"r"(tile_of(a, (int)pos1) + 4u * lane),
+                                 "r"((uint32_t)h10 | ((uint32_t)h11 << 16))
+                                 : "memory");
+            }
+            // zero tiles for the partners of lone blocks (pair o: position 2o+1)
+            for (uint32_t lone = tc_lds(ar.rec) >> 16; lone; lone &= lone - 1) {
+                const int o = __ffs(lone) - 1;
+                if (o % kTcDecodeWarps == dw)
+                    asm volatile("st.shared.u32 [%0], %1;" ::"r"(tile_of(a, 2 * o + 1) + 4u * lane), "r"(0u) : "memory");
             }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // tiles -> tensor core
             __syncwarp();
             if (lane == 0) tc_arrive(s_u32(&bar_tiles[a]));
+            if (lane == 0 && dw == 0) TR(1, c, 5);
         }
-    } else if (warp == kMma) {  // ------------------------------------------- MMA issue
-        for (int c = 0; c < nch; ++c) {
+    } else if (warp == kMma || warp == kMma2) {  // ------------------------------- MMA issue
+        // two issuing warps take alternate chunks: one chunk's waits and record
+        // reads overlap the other's MMAs (each commits its own MMAs)
+        for (int c = warp == kMma ? 0 : 1; c < nch; c += 2) {
             const int a = c % kTcRing, b = c % kTcSlabBufs;
+            if (lane == 0) TR(2, c, 0);
+            tc_wait(s_u32(&bar_arr[a]), ring_ph(c));
+            if (lane == 0) TR(2, c, 1);
             tc_wait(s_u32(&bar_tiles[a]), ring_ph(c));
-            tc_wait(s_u32(&bar_ops[a]), ring_ph(c));
+            if (lane == 0) TR(2, c, 2);
             tc_wait(s_u32(&bar_slab[b]), slab_ph(c));
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // cp.async slabs -> tensor core
-            // accumulator slots: the epilogue has finished chunk c-3 (chunks c-2 .. c
-            // hold at most 3 * kTcPairs < kTcSlots started block-rows)
+            if (lane == 0) TR(2, c, 3);
+            // accumulator slots: the epilogue has finished chunk c-3
+            // (chunks c-2 .. c hold at most 3 * kTcPairs < kTcSlots started block-rows)
             if (c >= 3) tc_wait(s_u32(&bar_epi[(c - 3) % kTcRing]), ring_ph(c - 3));
+            // a block-row continued from the previous chunk accumulates after that
+            // chunk's MMAs (issued by the other warp) have completed
+            if (c >= 1 && cdesc[a].pA > 0) tc_wait(s_u32(&bar_mma[(c - 1) % kTcRing]), ring_ph(c - 1));
+            if (lane == 0) TR(2, c, 4);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-            if (lane == 0) {
-                tc_arrive(s_u32(&bar_afree[a]));  // decoding is done: the staged arrays are free
-                const int no = nops[a];
-                for (int o = 0; o < no; ++o) {
-                    const uint4 dd = ops[a][o][0], dx = ops[a][o][1];
-                    umma_f16(dx.x, ((uint64_t)dd.y << 32) | dd.x, ((uint64_t)dd.w << 32) | dd.z, dx.y);
+            // the record's head and segments (bytes 0..33): three loads in flight at once
+            const uint32_t rec = arr[a].rec;
+            uint32_t r0, r1, r2, r3, r4, r5, r6, r7, r8;
+            asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                         : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
+                         : "r"(rec)
+                         : "memory");
+            asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                         : "=r"(r4), "=r"(r5), "=r"(r6), "=r"(r7)
+                         : "r"(rec + 16u)
+                         : "memory");
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(r8) : "r"(rec + 32u) : "memory");
+            // segments: warp-uniform through redux.sync (one per non-empty block-row);
+            // seg[t] is the low half of word 1 + t/2 for even t, the high half for odd t
+            const uint32_t nseg = __reduce_or_sync(0xffffffffu, r0 & 0xffu);
+            TR(2, c, 5);
+            // pair o: slabs at positions 2o, 2o+1 (LBO one slab), tiles at 2o, 2o+1 (LBO one tile)
+            const uint32_t ad0 = (uint32_t)umma_desc(slab_of(b, 0), (uint32_t)kSlabBytes, 128u);
+            const uint32_t bd0 = (uint32_t)umma_desc(tile_of(a, 0), (uint32_t)kTileBytes, 128u);
+            uint32_t o = 0;
+#pragma unroll 1
+            for (uint32_t t = 0; t < nseg; ++t) {
+                const uint32_t i = t >> 1;
+                const uint32_t w = i < 4 ? (i < 2 ? (i == 0 ? r1 : r2) : (i == 2 ? r3 : r4))
+                                         : (i < 6 ? (i == 4 ? r5 : r6) : (i == 6 ? r7 : r8));
+                const uint32_t sg = __reduce_or_sync(0xffffffffu, (t & 1u) ? (w >> 16) : (w & 0xffffu));
+                const uint32_t d = tmem_u + (sg & 63u) * (uint32_t)kTcN;
+                const uint32_t acc0 = (sg >> 6) & 1u, np = sg >> 7;
+                // descriptors of pair o: base + o * stride (two MMAs per step)
+                uint32_t ad = ad0 + o * (2u * kSlabBytes >> 4), bd = bd0 + o * (2u * kTileBytes >> 4);
+                uint32_t p = 0;
+#pragma unroll 1
+                for (; p + 1 < np; p += 2) {
+                    umma_f16_elect(d, ((uint64_t)kDescHi << 32) | ad, ((uint64_t)kDescHi << 32) | bd, p > 0 ? 1u : acc0);
+                    umma_f16_elect(d, ((uint64_t)kDescHi << 32) | (ad + (2u * kSlabBytes >> 4)),
+                                   ((uint64_t)kDescHi << 32) | (bd + (2u * kTileBytes >> 4)), 1u);
+                    ad += 2u * (2u * kSlabBytes >> 4);
+                    bd += 2u * (2u * kTileBytes >> 4);
                 }
+                if (p < np)
+                    umma_f16_elect(d, ((uint64_t)kDescHi << 32) | ad, ((uint64_t)kDescHi << 32) | bd, p > 0 ? 1u : acc0);
+                o += np;
+            }
+            if (lane == 0) {
                 // completion of every MMA issued so far: slabs of buffer b free, tiles of
                 // slot a free + accumulators of the chunk ready
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
@@ -435,7 +565,7 @@ k_spmm_tc(int64_t m, const TcChunk *__restrict__ chunks, const int32_t *__restri
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
                                  s_u32(&bar_mma[a]))
                              : "memory");
-                tc_arrive(s_u32(&bar_mma[a]));  // release: the ends list written above
+                TR(2, c, 6);
             }
             __syncwarp();
         }
@@ -443,16 +573,23 @@ k_spmm_tc(int64_t m, const TcChunk *__restrict__ chunks, const int32_t *__restri
         const int vec = warp * 32 + lane;  // TMEM lane = vector within the group
         for (int c = 0; c < nch; ++c) {
             const int a = c % kTcRing;
+            if (threadIdx.x == 0) TR(3, c, 0);
             tc_wait(s_u32(&bar_mma[a]), ring_ph(c));
+            if (threadIdx.x == 0) TR(3, c, 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-            const int ne = nends[a];
-            for (int e = 0; e < ne; ++e) {  // block-rows ending in this chunk
-                const int2 en = ends[a][e];
-                const int br = en.x;
+            // block-rows ending in this chunk, from the staged record
+            const uint32_t rec = arr[a].rec;
+            const int ne = (int)((tc_lds(rec) >> 8) & 0xffu);
+            const int brA = cdesc[a].brA;
+            for (int e = 0; e < ne; ++e) {
+                const uint32_t ea = rec + 64u + 2u * (uint32_t)e;
+                const uint32_t w = tc_lds(ea & ~3u);
+                const uint32_t en = (ea & 2u) ? (w >> 16) : (w & 0xffffu);
+                const int br = brA + (int)(en & 63u), slot = (int)(en >> 6) - 1;
                 float v[8];
-                if (en.y >= 0) {
+                if (slot >= 0) {
                     uint32_t r[8];
-                    const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(en.y * kTcN);
+                    const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)(slot * kTcN);
                     asm volatile(
                         "tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
                         : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
@@ -497,7 +634,11 @@ k_spmm_tc(int64_t m, const TcChunk *__restrict__ chunks, const int32_t *__restri
             }
             asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
             __syncwarp();
-            if (lane == 0) tc_arrive(s_u32(&bar_epi[a]));
+            if (lane == 0) {
+                tc_arrive(s_u32(&bar_epi[a]));
+                tc_arrive(s_u32(&bar_afree[a]));  // the chunk's staged arrays and record are no longer read
+            }
+            if (threadIdx.x == 0) TR(3, c, 2);
         }
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -507,28 +648,46 @@ k_spmm_tc(int64_t m, const TcChunk *__restrict__ chunks, const int32_t *__restri
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem) : "memory");
 }
 
-// Xb[bc][j][c] = fp16(X[j*ldx + 8bc + c]) (round to nearest even), 0 past n
-__global__ void k_pack_x_f16(int64_t n, int32_t k, const float *__restrict__ X, int64_t ldx, __half *__restrict__ Xb) {
+// Xb[g][bc][jj][c] = fp16(X[(128g + jj)*ldx + 8bc + c]) (round to nearest even),
+// 0 past n and past k.  A transpose through shared memory: a CTA takes 32
+// vectors x 16 block columns, reads each vector's 128 consecutive floats
+// coalesced, and writes each block column's 32 slab rows (512 contiguous bytes)
+// as 16-byte stores.
+constexpr int kPackJ = 32, kPackBC = 16, kPackRow = 8 * kPackBC + 8;  // halves per smem row (+8: no conflicts)
+__global__ void __launch_bounds__(256) k_pack_x_f16(int64_t n, int32_t k, const float *__restrict__ X, int64_t ldx,
+                                                    __half *__restrict__ Xb) {
+    __shared__ __align__(16) __half sh[kPackJ * kPackRow];
     const int64_t nbc = (n + 7) / 8;
-    const int64_t total = nbc * (int64_t)k;
-    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
-         t += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t bc = t / k;
-        const int j = (int)(t - bc * k);
-        const float *src = X + (int64_t)j * ldx + 8 * bc;
-        __align__(16) __half h[8];
-#pragma unroll
-        for (int c = 0; c < 8; ++c) h[c] = (8 * bc + c < n) ? __float2half_rn(src[c]) : __float2half_rn(0.f);
-        *reinterpret_cast<uint4 *>(Xb + t * 8) = *reinterpret_cast<const uint4 *>(h);
+    const int64_t bc0 = (int64_t)blockIdx.x * kPackBC;
+    const int j0 = blockIdx.y * kPackJ;  // vectors up to the padded group end (a multiple of 128)
+#pragma unroll 4
+    for (int idx = threadIdx.x; idx < kPackJ * 8 * kPackBC; idx += 256) {
+        const int r = idx / (8 * kPackBC), c = idx % (8 * kPackBC);
+        const int j = j0 + r;
+        const int64_t f = 8 * bc0 + c;
+        float v = 0.f;
+        if (j < k && f < n) v = __ldg(X + (int64_t)j * ldx + f);
+        sh[r * kPackRow + c] = __float2half_rn(v);
+    }
+    __syncthreads();
+    for (int idx = threadIdx.x; idx < kPackJ * kPackBC; idx += 256) {
+        const int b = idx / kPackJ, r = idx % kPackJ;
+        const int j = j0 + r;
+        const int64_t bc = bc0 + b;
+        if (bc < nbc) {
+            const int64_t slot = ((int64_t)(j / kTcM) * nbc + bc) * kTcM + (j % kTcM);
+            *reinterpret_cast<uint4 *>(Xb + slot * 8) = *reinterpret_cast<const uint4 *>(sh + r * kPackRow + 8 * b);
+        }
     }
 }
 
 }  // namespace
 
 spaden_status_t spmm_tc_pack_x(int64_t n, int32_t k, const float *X, int64_t ldx, void *Xb, cudaStream_t st) {
-    const int64_t total = ((n + 7) / 8) * (int64_t)k;
-    if (total == 0) return SPADEN_OK;
-    const unsigned grid = (unsigned)std::min<int64_t>((total + 255) / 256, 148 * 32);
+    const int64_t nbc = (n + 7) / 8;
+    if (nbc == 0 || k == 0) return SPADEN_OK;
+    const int64_t kpad = ((int64_t)k + kTcM - 1) / kTcM * kTcM;  // groups are zero-padded to 128 vectors
+    const dim3 grid((unsigned)((nbc + kPackBC - 1) / kPackBC), (unsigned)(kpad / kPackJ));
     k_pack_x_f16<<<grid, 256, 0, st>>>(n, k, X, ldx, (__half *)Xb);
     SPADEN_CUDA_TRY(cudaGetLastError());
     return SPADEN_OK;
@@ -544,19 +703,30 @@ static spaden_status_t build_tc_schedule(Matrix &A, int G, cudaStream_t st) {
     int32_t total = 0;
     if (e == cudaSuccess) e = cudaMemcpyAsync(&total, A.tc_cta_start + G, sizeof(int32_t), cudaMemcpyDeviceToHost, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-    if (e == cudaSuccess) e = cudaMalloc(&A.tc_chunks, sizeof(TcChunk) * (size_t)std::max(1, total));
+    // chunk descriptors, then the chunks' MMA records (16-byte aligned: bulk-copied)
+    const size_t rec_off = (sizeof(TcChunk) * (size_t)std::max(1, total) + 127) & ~(size_t)127;
+    if (e == cudaSuccess) e = cudaMalloc(&A.tc_chunks, rec_off + sizeof(TcRec) * (size_t)std::max(1, total));
     if (e == cudaSuccess) {
         k_tc_sched<<<1, 1, 0, st>>>(A.blk_rowptr, A.blk_offset, A.Bnrow, G, nullptr, cnt + ntmp, A.tc_cta_start,
                                     (TcChunk *)A.tc_chunks);
+        if (total > 0)
+            k_tc_ops<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(
+                A.blk_rowptr, (const TcChunk *)A.tc_chunks, total, (TcRec *)((char *)A.tc_chunks + rec_off));
         e = cudaGetLastError();
     }
     cudaFreeAsync(cnt, st);
     if (e != cudaSuccess) return cuda_status(e, "tensor-core SpMM schedule");
     A.tc_nchunks = total;
     A.tc_grid = G;
-    A.aux_bytes += (int64_t)(sizeof(TcChunk) * (size_t)total + sizeof(int32_t) * (G + 1));
+    A.aux_bytes += (int64_t)(rec_off + sizeof(TcRec) * (size_t)total + sizeof(int32_t) * (G + 1));
     return SPADEN_OK;
 }
+
+#ifdef SPADEN_TC_TRACE
+extern "C" __attribute__((visibility("default"))) int spaden_debug_tc_trace(void *buf) {
+    return (int)cudaMemcpyToSymbol(g_tc_trace, &buf, sizeof(buf));
+}
+#endif
 
 spaden_status_t spmm_tc_launch(Matrix &A, float alpha, const void *Xb, int32_t k, float beta, float *Y,
                                int64_t ldy, cudaStream_t st) {
@@ -577,9 +747,12 @@ spaden_status_t spmm_tc_launch(Matrix &A, float alpha, const void *Xb, int32_t k
     }
     for (int32_t j0 = 0; j0 < k; j0 += kTcM) {
         const int32_t kv = std::min<int32_t>(kTcM, k - j0);
-        k_spmm_tc<<<A.tc_grid, kTcThreads, kTcSmem, st>>>(A.m, (const TcChunk *)A.tc_chunks, A.tc_cta_start,
+        const size_t rec_off = (sizeof(TcChunk) * (size_t)std::max<int64_t>(1, A.tc_nchunks) + 127) & ~(size_t)127;
+        k_spmm_tc<<<A.tc_grid, kTcThreads, kTcSmem, st>>>(A.m, (const TcChunk *)A.tc_chunks,
+                                                            (const TcRec *)((const char *)A.tc_chunks + rec_off),
+                                                            A.tc_cta_start,
                                                             A.blk_rowptr, A.blk_col, A.bitmap, A.blk_offset,
-                                                            (const __half *)A.values, (const __half *)Xb, k, j0, kv,
+                                                            (const __half *)A.values, (const __half *)Xb, (A.n + 7) / 8, j0, kv,
                                                             alpha, beta, Y, ldy);
         SPADEN_CUDA_TRY(cudaGetLastError());
     }

@@ -181,12 +181,13 @@ class FusedIteratedSpMV:
         return self.x
 
 
-def _symmetric_buffers(L: int, world: int, rank: int, group, device):
-    """Two length-L fp32 buffers visible to every rank (peer views) + a barrier."""
+def _symmetric_buffers(L: int, world: int, rank: int, group, device, force_symmetric: bool = False):
+    """Two length-L fp32 buffers visible to every rank (peer views) + a barrier.
+    ``force_symmetric`` takes the symmetric-memory path even for one rank (tests)."""
     import torch
     import torch.distributed as dist
 
-    if world == 1 or not (dist.is_available() and dist.is_initialized()):
+    if (world == 1 and not force_symmetric) or not (dist.is_available() and dist.is_initialized()):
         if world != 1:
             raise RuntimeError("world > 1 needs an initialised process group")
         a = torch.zeros(L, dtype=torch.float32, device=device)
