@@ -138,6 +138,9 @@ typedef struct {
  * its bit (the round trip bitBSR -> CSR is the identity).  Invalid CSR is
  * reported as INVALID_ARGUMENT / INDEX_OUT_OF_RANGE / UNSORTED_OR_DUPLICATE;
  * nothing is leaked on error.  m == 0, n == 0 or nnz == 0 give a valid handle.
+ * The handle's arrays are stream-ordered allocations (on `stream`) from a
+ * library-private memory pool per device that keeps up to 4 GiB of freed
+ * memory mapped, so converting again after spaden_free reuses it.
  */
 SPADEN_API spaden_status_t spaden_convert_csr_to_bitmap(int64_t m, int64_t n, int64_t nnz,
                                              const int32_t *d_rowptr, const int32_t *d_colidx,
@@ -294,8 +297,10 @@ SPADEN_API spaden_status_t spaden_spmv_host_batched(spaden_matrix_t A, float alp
                                                     int64_t ldx, float beta, float *h_y, int64_t ldy,
                                                     int64_t nvec, void *stream);
 
-/* spaden_free -- synchronises the handle's device, then releases all device
- * arrays owned by A.  spaden_free(NULL) returns SPADEN_OK. */
+/* spaden_free -- synchronises the handle's device, then returns all device
+ * arrays owned by A to the library's pool (up to 4 GiB stays mapped for later
+ * conversions, the rest goes back to the driver).  spaden_free(NULL) returns
+ * SPADEN_OK. */
 SPADEN_API spaden_status_t spaden_free(spaden_matrix_t A);
 
 /* Introspection (tests, bench, the bytes-per-nnz metric). */

@@ -4,6 +4,7 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstdlib>
+#include <mutex>
 #include <new>
 #include <string>
 
@@ -42,23 +43,61 @@ static spaden_status_t check_device_ptr(const void *p, const char *name, int dev
     return SPADEN_OK;
 }
 
+// ---------------------------------------------------------- memory pool
+namespace {
+std::mutex g_pool_mu;
+cudaMemPool_t g_pool[64] = {};
+}  // namespace
+
+cudaError_t dev_alloc(void **ptr, size_t bytes, cudaStream_t st) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+    cudaMemPool_t pool;
+    {
+        std::lock_guard<std::mutex> lock(g_pool_mu);
+        if (!g_pool[dev]) {
+            cudaMemPoolProps props = {};
+            props.allocType = cudaMemAllocationTypePinned;
+            props.location.type = cudaMemLocationTypeDevice;
+            props.location.id = dev;
+            e = cudaMemPoolCreate(&g_pool[dev], &props);
+            if (e != cudaSuccess) {
+                g_pool[dev] = nullptr;
+                return e;
+            }
+            uint64_t keep = kPoolKeepBytes;
+            cudaMemPoolSetAttribute(g_pool[dev], cudaMemPoolAttrReleaseThreshold, &keep);
+        }
+        pool = g_pool[dev];
+    }
+    return cudaMallocFromPoolAsync(ptr, bytes, pool, st);
+}
+
+void dev_free(void *ptr, cudaStream_t st) {
+    if (ptr) cudaFreeAsync(ptr, st);
+}
+
 static void release(Matrix *A) {
     if (!A) return;
+    // the handle's arrays may still be read by work on any stream the caller
+    // used (spaden_free's contract says none is in flight; cudaFree used to
+    // synchronise the device implicitly): keep that behaviour
+    cudaDeviceSynchronize();
     void *ptrs[] = {A->blk_rowptr, A->blk_col, A->bitmap,   A->blk_offset, A->values,
                     A->stage_x,     A->stage_y,  A->tiles, A->rot,
                     A->long_rows,   A->chunk_start, A->chunk_row, A->carry, A->chunk_done,
                     A->spmm_tiles[0], A->spmm_tiles[1], A->spmm_tiles[2], A->tc_chunks, A->tc_cta_start};
-    for (void *p : ptrs)
-        if (p) cudaFree(p);
+    for (void *p : ptrs) dev_free(p, 0);
     for (int j = 0; j < Matrix::kMaxPipe; ++j) {
-        if (A->pipe_x[j]) cudaFree(A->pipe_x[j]);
-        if (A->pipe_y[j]) cudaFree(A->pipe_y[j]);
+        dev_free(A->pipe_x[j], 0);
+        dev_free(A->pipe_y[j], 0);
     }
     for (int q = 0; q < A->n_res_parts; ++q) {
         const spaden::ResPart &P = A->res[q];
         void *rp[] = {P.rowptr, P.colidx, P.values, P.long_rows, P.chunk_start, P.chunk_row, P.carry, P.done, P.perm};
-        for (void *p : rp)
-            if (p) cudaFree(p);
+        for (void *p : rp) dev_free(p, 0);
     }
     for (cudaEvent_t e : A->ev)
         if (e) cudaEventDestroy(e);
@@ -77,9 +116,10 @@ static spaden_status_t ensure_pipeline(Matrix *A) {
     if (const char *e = getenv("SPADEN_PIPE_SLOTS")) slots = atoi(e);
     A->pipe_slots = slots < 2 ? 2 : (slots > Matrix::kMaxPipe ? Matrix::kMaxPipe : slots);
     for (int j = 0; j < A->pipe_slots; ++j) {
-        if (A->n > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->pipe_x[j], pad16(4 * A->n)));
-        if (A->m > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->pipe_y[j], pad16(4 * A->m)));
+        if (A->n > 0) SPADEN_CUDA_TRY(dmalloc(&A->pipe_x[j], pad16(4 * A->n), 0));
+        if (A->m > 0) SPADEN_CUDA_TRY(dmalloc(&A->pipe_y[j], pad16(4 * A->m), 0));
     }
+    SPADEN_CUDA_TRY(cudaStreamSynchronize(0));  // pool allocations visible to the non-blocking copy streams
     for (cudaEvent_t &e : A->ev) SPADEN_CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     SPADEN_CUDA_TRY(cudaStreamCreateWithFlags(&A->s_d2h, cudaStreamNonBlocking));
     SPADEN_CUDA_TRY(cudaStreamCreateWithFlags(&A->s_h2d, cudaStreamNonBlocking));
@@ -324,8 +364,8 @@ spaden_status_t spaden_spmv_host(spaden_matrix_t A, float alpha, const float *h_
         return SPADEN_ERR_INVALID_ARGUMENT;
     }
     cudaStream_t st = (cudaStream_t)stream;
-    if (!A->stage_x && A->n > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->stage_x, pad16(4 * A->n)));
-    if (!A->stage_y && A->m > 0) SPADEN_CUDA_TRY(cudaMalloc(&A->stage_y, pad16(4 * A->m)));
+    if (!A->stage_x && A->n > 0) SPADEN_CUDA_TRY(dmalloc(&A->stage_x, pad16(4 * A->n), st));
+    if (!A->stage_y && A->m > 0) SPADEN_CUDA_TRY(dmalloc(&A->stage_y, pad16(4 * A->m), st));
     if (A->n > 0)
         SPADEN_CUDA_TRY(cudaMemcpyAsync(A->stage_x, h_x, 4 * A->n, cudaMemcpyHostToDevice, st));
     if (beta != 0.f && A->m > 0)

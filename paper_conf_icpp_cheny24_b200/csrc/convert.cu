@@ -378,7 +378,7 @@ spaden_status_t convert_csr(int64_t m, int64_t n, int64_t nnz, const int32_t *ro
     // ---- owned arrays
     A->m = m; A->n = n; A->nnz = nnz; A->Bnrow = Bnrow; A->Bnnz = Bnnz; A->storage = sdt;
     auto alloc = [&](void **ptr, size_t bytes) -> cudaError_t {
-        cudaError_t e = cudaMalloc(ptr, pad16(bytes));
+        cudaError_t e = dmalloc(ptr, pad16(bytes), st);
         if (e == cudaSuccess) e = cudaMemsetAsync(*ptr, 0, pad16(bytes), st);
         return e;
     };

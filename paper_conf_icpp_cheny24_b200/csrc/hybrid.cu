@@ -410,8 +410,8 @@ spaden_status_t residual_schedule(Matrix *A, ResPart &P, cudaStream_t st) {
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     if (e == cudaSuccess && nl > 0) {
         P.n_long = nl;
-        e = cudaMalloc(&P.long_rows, 4 * (size_t)nl);
-        if (e == cudaSuccess) e = cudaMalloc(&P.chunk_start, 4 * ((size_t)nl + 1));
+        e = dmalloc(&P.long_rows, 4 * (size_t)nl, st);
+        if (e == cudaSuccess) e = dmalloc(&P.chunk_start, 4 * ((size_t)nl + 1), st);
         if (e == cudaSuccess) {
             k_res_long_list<<<g, 256, 0, st>>>(m, P.rowptr, flag, P.long_rows, P.chunk_start);
             e = exclusive_scan_i32(P.chunk_start, P.chunk_start, nl, scan_tmp, st);
@@ -421,11 +421,11 @@ spaden_status_t residual_schedule(Matrix *A, ResPart &P, cudaStream_t st) {
         if (e == cudaSuccess) e = cudaStreamSynchronize(st);
         if (e == cudaSuccess) {
             P.n_chunks = nc;
-            e = cudaMalloc(&P.chunk_row, 4 * (size_t)std::max(1, nc));
+            e = dmalloc(&P.chunk_row, 4 * (size_t)std::max(1, nc), st);
         }
         constexpr int SL = Matrix::kScratchSlots;
-        if (e == cudaSuccess) e = cudaMalloc(&P.carry, 4 * (size_t)std::max(1, nc) * SL);
-        if (e == cudaSuccess) e = cudaMalloc(&P.done, 4 * (size_t)nl * SL);
+        if (e == cudaSuccess) e = dmalloc(&P.carry, 4 * (size_t)std::max(1, nc) * SL, st);
+        if (e == cudaSuccess) e = dmalloc(&P.done, 4 * (size_t)nl * SL, st);
         if (e == cudaSuccess) e = cudaMemsetAsync(P.done, 0, 4 * (size_t)nl * SL, st);
         if (e == cudaSuccess) {
             k_res_chunk_rows<<<(unsigned)((nl + 255) / 256), 256, 0, st>>>(nl, P.chunk_start, P.chunk_row);
@@ -437,7 +437,7 @@ spaden_status_t residual_schedule(Matrix *A, ResPart &P, cudaStream_t st) {
     int32_t *perm_pos = nullptr;
     ResBins bins{};
     int64_t total = 0;
-    if (e == cudaSuccess) e = cudaMalloc(&perm_pos, 4 * (size_t)std::max<int64_t>(1, m));
+    if (e == cudaSuccess) e = dmalloc(&perm_pos, 4 * (size_t)std::max<int64_t>(1, m), st);
     for (int c = 0; c <= kResClasses && e == cudaSuccess; ++c) {
         bins.row_start[c] = total;
         k_res_class_flag<<<g, 256, 0, st>>>(m, P.rowptr, c, flag);
@@ -463,7 +463,7 @@ spaden_status_t residual_schedule(Matrix *A, ResPart &P, cudaStream_t st) {
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     cudaFreeAsync(tmp, st);
     if (e != cudaSuccess) {
-        if (perm_pos) cudaFree(perm_pos);
+        if (perm_pos) dev_free(perm_pos, st);
         return cuda_status(e, "hybrid residual schedule");
     }
     P.perm = perm_pos;
@@ -535,9 +535,9 @@ static spaden_status_t segment_residual(Matrix *A, cudaStream_t st) {
     int32_t *cnt = nullptr, *scan_tmp = nullptr;
     int32_t **d_cols = nullptr;
     void **d_vals = nullptr;
-    cudaError_t e = cudaMalloc(&cnt, 4 * (size_t)S * (m + 1));
-    if (e == cudaSuccess) e = cudaMalloc(&scan_tmp, 4 * (nt + 4));
-    if (e == cudaSuccess) e = cudaMalloc(&d_cols, sizeof(void *) * 2 * S);
+    cudaError_t e = dmalloc(&cnt, 4 * (size_t)S * (m + 1), st);
+    if (e == cudaSuccess) e = dmalloc(&scan_tmp, 4 * (nt + 4), st);
+    if (e == cudaSuccess) e = dmalloc(&d_cols, sizeof(void *) * 2 * S, st);
     d_vals = (void **)(d_cols + S);
     const unsigned g = (unsigned)((32 * m + 255) / 256);
     if (e == cudaSuccess) {
@@ -557,9 +557,9 @@ static spaden_status_t segment_residual(Matrix *A, cudaStream_t st) {
         if (e == cudaSuccess) e = cudaMemcpyAsync(&tot, c + m, 4, cudaMemcpyDeviceToHost, st);
         if (e == cudaSuccess) e = cudaStreamSynchronize(st);
         P.nnz = tot;
-        if (e == cudaSuccess) e = cudaMalloc(&P.rowptr, pad16(4 * (m + 1)));
-        if (e == cudaSuccess) e = cudaMalloc(&P.colidx, pad16(4 * (size_t)tot));
-        if (e == cudaSuccess) e = cudaMalloc(&P.values, pad16(sv * (size_t)tot));
+        if (e == cudaSuccess) e = dmalloc(&P.rowptr, pad16(4 * (m + 1)), st);
+        if (e == cudaSuccess) e = dmalloc(&P.colidx, pad16(4 * (size_t)tot), st);
+        if (e == cudaSuccess) e = dmalloc(&P.values, pad16(sv * (size_t)tot), st);
         if (e == cudaSuccess) e = cudaMemcpyAsync(P.rowptr, c, 4 * (m + 1), cudaMemcpyDeviceToDevice, st);
         h_cols[q] = P.colidx;
         h_vals[q] = P.values;
@@ -577,12 +577,12 @@ static spaden_status_t segment_residual(Matrix *A, cudaStream_t st) {
         e = cudaGetLastError();
     }
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-    cudaFree(full.rowptr);
-    cudaFree(full.colidx);
-    cudaFree(full.values);
-    if (cnt) cudaFree(cnt);
-    if (scan_tmp) cudaFree(scan_tmp);
-    if (d_cols) cudaFree(d_cols);
+    dev_free(full.rowptr, st);
+    dev_free(full.colidx, st);
+    dev_free(full.values, st);
+    if (cnt) dev_free(cnt, st);
+    if (scan_tmp) dev_free(scan_tmp, st);
+    if (d_cols) dev_free(d_cols, st);
     if (e != cudaSuccess) return cuda_status(e, "hybrid residual column segmentation");
     A->res_aux_bytes += 4 * (int64_t)(S - 1) * (m + 1);  // rowptrs beyond the first
     return SPADEN_OK;
@@ -619,17 +619,17 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
     int32_t *n_col = nullptr, *n_off = nullptr, *r_col = nullptr;
     uint64_t *n_bmp = nullptr;
     void *n_vals = nullptr, *r_vals = nullptr;
-    e = cudaMalloc(&n_col, pad16(4 * nB));
-    if (e == cudaSuccess) e = cudaMalloc(&n_bmp, pad16(8 * nB));
-    if (e == cudaSuccess) e = cudaMalloc(&n_off, pad16(4 * (nB + 1)));
-    if (e == cudaSuccess) e = cudaMalloc(&n_vals, pad16(sv * nV));
+    e = dmalloc(&n_col, pad16(4 * nB), st);
+    if (e == cudaSuccess) e = dmalloc(&n_bmp, pad16(8 * nB), st);
+    if (e == cudaSuccess) e = dmalloc(&n_off, pad16(4 * (nB + 1)), st);
+    if (e == cudaSuccess) e = dmalloc(&n_vals, pad16(sv * nV), st);
     ResPart &P0 = A->res[0];
-    if (e == cudaSuccess) e = cudaMalloc(&P0.rowptr, pad16(4 * (m + 1)));
-    if (e == cudaSuccess) e = cudaMalloc(&r_col, pad16(4 * res_nnz));
-    if (e == cudaSuccess) e = cudaMalloc(&r_vals, pad16(sv * res_nnz));
+    if (e == cudaSuccess) e = dmalloc(&P0.rowptr, pad16(4 * (m + 1)), st);
+    if (e == cudaSuccess) e = dmalloc(&r_col, pad16(4 * res_nnz), st);
+    if (e == cudaSuccess) e = dmalloc(&r_vals, pad16(sv * res_nnz), st);
     if (e != cudaSuccess) {
         for (void *p : {(void *)n_col, (void *)n_bmp, (void *)n_off, n_vals, (void *)r_col, r_vals})
-            if (p) cudaFree(p);
+            if (p) dev_free(p, st);
         return fail(e, "hybrid split (allocation)");
     }
     cudaMemsetAsync(n_off, 0, pad16(4 * (nB + 1)), st);
@@ -647,10 +647,10 @@ spaden_status_t split_residual(Matrix *A, int t, cudaStream_t st) {
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     cudaFreeAsync(tmp, st);
     // install the compacted bitBSR (free the old arrays) and the residual
-    cudaFree(A->blk_col);
-    cudaFree(A->bitmap);
-    cudaFree(A->blk_offset);
-    cudaFree(A->values);
+    dev_free(A->blk_col, st);
+    dev_free(A->bitmap, st);
+    dev_free(A->blk_offset, st);
+    dev_free(A->values, st);
     A->blk_col = n_col;
     A->bitmap = n_bmp;
     A->blk_offset = n_off;

@@ -323,4 +323,16 @@ __device__ __forceinline__ int warp_excl_scan_i32(int v, int lane, int *total) {
 
 inline size_t pad16(size_t bytes) { return ((bytes + 15) / 16) * 16 + 16; }
 
+// Device memory of handles and conversion scratch: stream-ordered allocations
+// from a library-private pool per device (capi.cu) that keeps up to
+// kPoolKeepBytes of freed memory mapped, so converting again after
+// spaden_free does not pay the driver's map/unmap (conversion time is then
+// stable from the second conversion on).  dev_free is stream ordered as well.
+constexpr uint64_t kPoolKeepBytes = 4ull << 30;
+cudaError_t dev_alloc(void **ptr, size_t bytes, cudaStream_t st);
+void dev_free(void *ptr, cudaStream_t st);
+template <typename T> inline cudaError_t dmalloc(T **ptr, size_t bytes, cudaStream_t st) {
+    return dev_alloc(reinterpret_cast<void **>(ptr), bytes, st);
+}
+
 }  // namespace spaden

@@ -273,8 +273,8 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     A->n_long = h[1];
     const size_t tile_bytes = sizeof(TileDesc) * (size_t)std::max<int64_t>(1, A->n_tiles + 1);
     const size_t long_bytes = sizeof(int32_t) * (size_t)std::max<int64_t>(1, A->n_long);
-    e = cudaMalloc(&A->tiles, tile_bytes);
-    if (e == cudaSuccess) e = cudaMalloc(&A->long_rows, long_bytes);
+    e = dmalloc(&A->tiles, tile_bytes, st);
+    if (e == cudaSuccess) e = dmalloc(&A->long_rows, long_bytes, st);
     if (e != cudaSuccess) {
         cudaFreeAsync(tmp, st);
         return cuda_status(e, "allocating SpMV schedule");
@@ -286,7 +286,7 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     cudaFreeAsync(tmp, st);
     if (e != cudaSuccess) return cuda_status(e, "packing SpMV schedule");
     if (use_rot && A->n_tiles > 0 && A->Bnnz > 0) {  // bank-conflict row rotations (slot decode)
-        e = cudaMalloc(&A->rot, pad16((size_t)A->Bnnz));
+        e = dmalloc(&A->rot, pad16((size_t)A->Bnnz), st);
         if (e == cudaSuccess) e = cudaMemsetAsync(A->rot, 0, pad16((size_t)A->Bnnz), st);
         if (e == cudaSuccess) {
             const unsigned g = (unsigned)((A->n_tiles + kRotWarps - 1) / kRotWarps);
@@ -306,7 +306,7 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     int32_t *ltmp = nullptr;
     const size_t lt = scan_tmp_ints(nl + 1);
     SPADEN_CUDA_TRY(cudaMallocAsync(&ltmp, (lt + 4) * sizeof(int32_t), st));
-    e = cudaMalloc(&A->chunk_start, sizeof(int32_t) * (nl + 1));
+    e = dmalloc(&A->chunk_start, sizeof(int32_t) * (nl + 1), st);
     if (e == cudaSuccess) {
         k_long_chunks<<<(nl + 255) / 256, 256, 0, st>>>(nl, A->long_rows, A->blk_rowptr, A->chunk_start);
         e = exclusive_scan_i32(A->chunk_start, A->chunk_start, nl, ltmp, st);
@@ -317,11 +317,11 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
     cudaFreeAsync(ltmp, st);
     if (e == cudaSuccess) {
         A->n_chunks = nch;
-        e = cudaMalloc(&A->chunk_row, sizeof(int32_t) * std::max(1, nch));
+        e = dmalloc(&A->chunk_row, sizeof(int32_t) * std::max(1, nch), st);
     }
     constexpr int SL = Matrix::kScratchSlots;
-    if (e == cudaSuccess) e = cudaMalloc(&A->carry, sizeof(float) * 8 * std::max(1, nch) * SL);
-    if (e == cudaSuccess) e = cudaMalloc(&A->chunk_done, sizeof(int32_t) * nl * SL);
+    if (e == cudaSuccess) e = dmalloc(&A->carry, sizeof(float) * 8 * std::max(1, nch) * SL, st);
+    if (e == cudaSuccess) e = dmalloc(&A->chunk_done, sizeof(int32_t) * nl * SL, st);
     if (e == cudaSuccess) e = cudaMemsetAsync(A->chunk_done, 0, sizeof(int32_t) * nl * SL, st);
     if (e == cudaSuccess) {
         k_chunk_rows<<<(nl + 255) / 256, 256, 0, st>>>(nl, A->chunk_start, A->chunk_row);
@@ -371,7 +371,7 @@ spaden_status_t build_spmm_schedule(Matrix *A, int kidx, int K, cudaStream_t st)
         return SPADEN_ERR_UNSUPPORTED;
     }
     const size_t tile_bytes = sizeof(TileDesc) * (size_t)std::max(1, h[0] + 1);
-    e = cudaMalloc(&A->spmm_tiles[kidx], tile_bytes);
+    e = dmalloc(&A->spmm_tiles[kidx], tile_bytes, st);
     if (e == cudaSuccess) {
         k_pack<true><<<grid, 128, 0, st>>>(Bnrow, A->blk_rowptr, A->blk_offset, sv, cap, long_cost, pack_bytes,
                                            hyb, nullptr, nullptr, nullptr, seg_tiles, seg_long, A->spmm_tiles[kidx],

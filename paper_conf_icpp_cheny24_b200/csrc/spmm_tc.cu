@@ -695,7 +695,7 @@ spaden_status_t spmm_tc_pack_x(int64_t n, int32_t k, const float *X, int64_t ldx
 
 static spaden_status_t build_tc_schedule(Matrix &A, int G, cudaStream_t st) {
     int32_t *cnt = nullptr;
-    SPADEN_CUDA_TRY(cudaMalloc(&A.tc_cta_start, sizeof(int32_t) * (G + 1)));
+    SPADEN_CUDA_TRY(dmalloc(&A.tc_cta_start, sizeof(int32_t) * (G + 1), st));
     const size_t ntmp = scan_tmp_ints(G + 1);
     SPADEN_CUDA_TRY(cudaMallocAsync(&cnt, sizeof(int32_t) * (ntmp + G + 1), st));
     k_tc_sched<<<1, 1, 0, st>>>(A.blk_rowptr, A.blk_offset, A.Bnrow, G, A.tc_cta_start, nullptr, nullptr, nullptr);
@@ -705,7 +705,7 @@ static spaden_status_t build_tc_schedule(Matrix &A, int G, cudaStream_t st) {
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     // chunk descriptors, then the chunks' MMA records (16-byte aligned: bulk-copied)
     const size_t rec_off = (sizeof(TcChunk) * (size_t)std::max(1, total) + 127) & ~(size_t)127;
-    if (e == cudaSuccess) e = cudaMalloc(&A.tc_chunks, rec_off + sizeof(TcRec) * (size_t)std::max(1, total));
+    if (e == cudaSuccess) e = dmalloc(&A.tc_chunks, rec_off + sizeof(TcRec) * (size_t)std::max(1, total), st);
     if (e == cudaSuccess) {
         k_tc_sched<<<1, 1, 0, st>>>(A.blk_rowptr, A.blk_offset, A.Bnrow, G, nullptr, cnt + ntmp, A.tc_cta_start,
                                     (TcChunk *)A.tc_chunks);

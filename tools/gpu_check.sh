@@ -1,9 +1,17 @@
 #!/bin/bash
-mkdir -p gpurun_out
-timeout 1500 python -m pytest tests -m gpu -q -x --timeout 900 > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
-nvidia-smi --query-gpu=index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active --format=csv -lms 200 > gpurun_out/clocks.csv &
-SMI=$!
-timeout 900 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
-kill $SMI
-nvidia-smi -q | grep -i -A3 "PCIe Generation\|Link Width" > gpurun_out/pcie.txt 2>&1
-echo done
+# health check at HEAD: smoke, pytest -m gpu, default bench lines (fp32 / fp16)
+O=gpurun_out/chk; mkdir -p $O
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?" >> $O/smoke.log
+timeout 1800 python -m pytest tests -m gpu -q -x --timeout 900 > $O/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $O/pytest_gpu.log
+timeout 600 python bench.py > $O/bench_fp32.json 2> $O/bench_fp32.err
+timeout 600 python bench.py --dtype fp16 --spmm "" --spmm-tc "" --no-cpu-baseline > $O/bench_fp16.json 2> $O/bench_fp16.err
+tail -3 $O/pytest_gpu.log; tail -2 $O/smoke.log
+python - <<'PY'
+import json
+for f in ['gpurun_out/chk/bench_fp32.json', 'gpurun_out/chk/bench_fp16.json']:
+    try:
+        d = json.loads(open(f).read().strip().splitlines()[-1])
+        print(f, d['value'], d['roofline']['frac'], d.get('convert'))
+    except Exception as e:
+        print(f, 'ERR', e)
+PY
