@@ -65,6 +65,10 @@ def parse():
     p.add_argument("--hybrid", type=int, default=-1,
                    help="hybrid format: blocks with <= HYBRID entries go to a CSR residual (0 = pure bitBSR, "
                         "-1 = automatic by mean block fill)")
+    p.add_argument("--reorder", default="none", choices=["none", "degree"],
+                   help="degree: symmetric degree ordering P A P^T before conversion (spaden_degree_order + "
+                        "spaden_permute_csr, SURVEY.md NEXT-1); the iteration runs in the permuted space "
+                        "(one GPU only)")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     p.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
                    help="x rebuild for N>1: NCCL all-gather after the SpMV, or peer stores fused into the "
@@ -257,7 +261,7 @@ def reference_arm(args):
 class Workload:
     """This rank's slice of the benchmark matrix plus the iteration it runs."""
 
-    def __init__(self, name, rank, world, dev):
+    def __init__(self, name, rank, world, dev, reorder="none"):
         import torch
 
         from paper_conf_icpp_cheny24_b200.dist import RowPartition
@@ -290,6 +294,23 @@ class Workload:
             self.x0 = torch.from_numpy(W.vector(A.n, 2)).to(dev)
             self.step_desc = "x <- A x / ||A||_inf"
         self.r0, self.r1 = self.part.range(rank)
+        self.reorder_s = None
+        if reorder == "degree":  # B = P A P^T; x kept in the permuted space (x'[k] = x[perm[k]])
+            import paper_conf_icpp_cheny24_b200 as sp
+            if world > 1:
+                raise SystemExit("bench.py: --reorder needs the whole matrix on one GPU (--gpus 1)")
+            times = []
+            for _ in range(3):  # first call loads the sort kernels; median of the 3
+                torch.cuda.synchronize(dev)
+                t0 = time.perf_counter()
+                perm = sp.degree_order(self.local[0])
+                B = sp.permute_csr(*self.local, perm)
+                torch.cuda.synchronize(dev)
+                times.append(time.perf_counter() - t0)
+            self.reorder_s = statistics.median(times)
+            self.local = B
+            self.x0 = self.x0[perm.long()].contiguous()
+            self.host = None
 
 
 def main():
@@ -316,7 +337,7 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
 
     # ---- workload (identical on every rank), this rank's 8-row-aligned slice
-    wl = Workload(args.workload, rank, world, dev)
+    wl = Workload(args.workload, rank, world, dev, args.reorder)
     sv = 2 if args.dtype == "fp16" else 4
     stream = torch.cuda.current_stream(dev)
     # warm-up conversion of the same matrix: loads every kernel the conversion
@@ -641,6 +662,10 @@ def main():
                               if flush else "inputs larger than L2 (A > 126 MB), no flush"
                               if info.format_bytes > L2_BYTES else "matrix fits L2, no flush (--l2 warm): warm-L2 number"),
                        "step": wl.step_desc,
+                       "reorder": args.reorder if args.reorder == "none" else {
+                           "kind": args.reorder, "seconds": wl.reorder_s,
+                           "what": "spaden_degree_order + spaden_permute_csr on the GPU (median of 3, wall clock); "
+                                   "x and y stay in the permuted space"},
                        **({"exchange": args.exchange} if world > 1 else {})},
             "hbm_gbs": achieved,
             "bytes_per_nnz": {"stored": info.format_bytes / max(1, info.nnz),

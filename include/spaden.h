@@ -161,6 +161,45 @@ SPADEN_API spaden_status_t spaden_count_blocks(int64_t m, int64_t n, int64_t nnz
                                                const int32_t *d_colidx, void *stream, int64_t *Bnnz);
 
 /*
+ * Reordering before conversion (second half).  The
+ * paper names reordering (degree-based, Gorder, Rabbit) as the usual remedy
+ * for irregular, low-degree matrices (§6) -- the regime where
+ * bitmaps cost more than they save.  Placing high-degree
+ * rows/columns first raises the fill of the 8x8 blocks they share and puts the
+ * hub entries of x on common cache lines.
+ *
+ * spaden_degree_order -- d_perm[k] = the row placed k-th: rows by descending
+ * degree (rowptr[i+1] - rowptr[i]), equal degrees in ascending row order.
+ *   m         rows, 0 <= m < 2^31.
+ *   d_rowptr  int32[m+1] device CSR row pointers (non-decreasing).
+ *   d_perm    int32[m] device output (caller-owned).
+ * Stream-ordered, no host synchronisation; temporaries from the library pool.
+ * Deterministic (a stable radix sort).
+ *
+ * spaden_permute_csr -- the symmetric permutation B = P A P^T of a square CSR
+ * matrix A (m x m): row k of B is row perm[k] of A with every column j renamed
+ * iperm[j] (iperm[perm[k]] = k) and the row's entries sorted by the new column.
+ * Hence B (P x) = P (A x) with (P x)[k] = x[perm[k]]: an iteration on B runs
+ * in the permuted space (PageRank keeps x permuted; only its start and end are
+ * mapped).
+ *   m, nnz            shape (square) and entries; A must be a valid CSR with
+ *                     columns in [0, m) (as spaden_convert_csr_to_bitmap checks;
+ *                     violations return INDEX_OUT_OF_RANGE).
+ *   d_rowptr, d_colidx, d_values  A on the device, values of dtype (16F or 32F,
+ *                     moved as raw bits).
+ *   d_perm            int32[m], a permutation of [0, m) (e.g. spaden_degree_order).
+ *   d_out_rowptr, d_out_colidx, d_out_values  B, caller-owned device arrays of
+ *                     m+1, nnz and nnz elements (must not alias the inputs).
+ * Stream-ordered; one host synchronisation (the column range check).
+ */
+SPADEN_API spaden_status_t spaden_degree_order(int64_t m, const int32_t *d_rowptr, int32_t *d_perm, void *stream);
+SPADEN_API spaden_status_t spaden_permute_csr(int64_t m, int64_t nnz, const int32_t *d_rowptr,
+                                              const int32_t *d_colidx, const void *d_values,
+                                              spaden_dtype_t dtype, const int32_t *d_perm,
+                                              int32_t *d_out_rowptr, int32_t *d_out_colidx,
+                                              void *d_out_values, void *stream);
+
+/*
  * spaden_convert_csr_to_bitmap_ex -- as spaden_convert_csr_to_bitmap, with options
  * (opts may be NULL = defaults).  With residual_max_popc = t > 0 the matrix is
  * split by block: 8x8 blocks with <= t entries go to a CSR residual (row-sorted,

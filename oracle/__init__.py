@@ -228,3 +228,32 @@ def hybrid_split(m, n, rowptr, colidx, values, t: int):
         return rp, colidx[mask], values[mask]
 
     return sub(~res), sub(res)
+
+
+def degree_order(rowptr) -> np.ndarray:
+    """Degree ordering (SURVEY.md §8(f) NEXT-1 reordering; degree-based ordering is
+    one of the remedies PAPER.md §6 cites): perm[k] = the row placed k-th,
+    rows by descending degree rowptr[i+1]-rowptr[i], equal degrees in ascending
+    row order (a stable sort of -degree).  Definition only."""
+    deg = np.diff(np.asarray(rowptr, dtype=np.int64))
+    return np.argsort(-deg, kind="stable").astype(np.int32)
+
+
+def permute_csr(rowptr, colidx, values, perm):
+    """Symmetric permutation B = P A P^T of a square CSR matrix, written from its
+    definition B[k, l] = A[perm[k], perm[l]]: every entry (i, j, v) of A becomes
+    (iperm[i], iperm[j], v) with iperm[perm[k]] = k, entries then in (row, column)
+    order.  Returns (rowptr, colidx, values) numpy arrays."""
+    rowptr = np.asarray(rowptr, dtype=np.int64)
+    m = rowptr.size - 1
+    perm = np.asarray(perm, dtype=np.int64)
+    iperm = np.empty(m, dtype=np.int64)
+    iperm[perm] = np.arange(m, dtype=np.int64)
+    rows = np.repeat(np.arange(m, dtype=np.int64), np.diff(rowptr))
+    nr = iperm[rows]
+    nc = iperm[np.asarray(colidx, dtype=np.int64)]
+    order = np.lexsort((nc, nr))
+    counts = np.bincount(nr, minlength=m) if m else np.zeros(0, np.int64)
+    rp = np.zeros(m + 1, np.int64)
+    np.cumsum(counts, out=rp[1:])
+    return rp.astype(np.int32), nc[order].astype(np.int32), np.asarray(values)[order]

@@ -72,6 +72,12 @@ spaden_convert_csr_to_bitmap_ex.restype = _ST
 spaden_count_blocks = _lib.spaden_count_blocks
 spaden_count_blocks.argtypes = [_I64, _I64, _I64, _P, _P, _P, ctypes.POINTER(_I64)]
 spaden_count_blocks.restype = _ST
+spaden_degree_order = _lib.spaden_degree_order
+spaden_degree_order.argtypes = [_I64, _P, _P, _P]
+spaden_degree_order.restype = _ST
+spaden_permute_csr = _lib.spaden_permute_csr
+spaden_permute_csr.argtypes = [_I64, _I64, _P, _P, _P, ctypes.c_int, _P, _P, _P, _P, _P]
+spaden_permute_csr.restype = _ST
 spaden_spmv = _lib.spaden_spmv
 spaden_spmv.argtypes = [_P, _F, _P, _F, _P, _P]
 spaden_spmv.restype = _ST
@@ -118,7 +124,8 @@ spaden_version = _lib.spaden_version
 spaden_version.argtypes = []
 spaden_version.restype = ctypes.c_char_p
 
-EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_count_blocks", "spaden_spmv", "spaden_spmm",
+EXPORTED = ["spaden_convert_csr_to_bitmap", "spaden_convert_csr_to_bitmap_ex", "spaden_count_blocks",
+            "spaden_degree_order", "spaden_permute_csr", "spaden_spmv", "spaden_spmm",
             "spaden_spmv_scatter", "spaden_spmm_tc_pack_x", "spaden_spmm_tc_xb_bytes", "spaden_spmm_tc", "spaden_spmv_host", "spaden_spmv_host_batched",
             "spaden_free",
             "spaden_get_info", "spaden_get_arrays", "spaden_spmv_launch_count", "spaden_status_string",
@@ -329,6 +336,37 @@ def count_blocks(rowptr, colidx, n: int, stream=None) -> int:
                                ctypes.c_void_p(colidx.data_ptr()), _stream_ptr(stream), ctypes.byref(out)),
            "spaden_count_blocks")
     return out.value
+
+
+def degree_order(rowptr, stream=None):
+    """perm (int32 CUDA tensor): rows by descending degree, ties by ascending index
+    (spaden_degree_order; SURVEY.md §8(f) NEXT-1 reordering)."""
+    torch = _torch()
+    assert rowptr.dtype == torch.int32 and rowptr.is_cuda
+    m = rowptr.numel() - 1
+    perm = torch.empty(max(m, 0), dtype=torch.int32, device=rowptr.device)
+    _check(spaden_degree_order(m, ctypes.c_void_p(rowptr.data_ptr()), ctypes.c_void_p(perm.data_ptr()),
+                               _stream_ptr(stream)), "spaden_degree_order")
+    return perm
+
+
+def permute_csr(rowptr, colidx, values, perm, stream=None):
+    """B = P A P^T of a square CSR matrix (spaden_permute_csr): row k of B is row
+    perm[k] of A, columns renamed by the inverse permutation and sorted.  Returns
+    (rowptr, colidx, values) CUDA tensors."""
+    torch = _torch()
+    assert rowptr.dtype == torch.int32 and colidx.dtype == torch.int32 and perm.dtype == torch.int32
+    m = rowptr.numel() - 1
+    nnz = colidx.numel()
+    rp = torch.empty(m + 1, dtype=torch.int32, device=rowptr.device)
+    ci = torch.empty(nnz, dtype=torch.int32, device=rowptr.device)
+    v = torch.empty(nnz, dtype=values.dtype, device=rowptr.device)
+    _check(spaden_permute_csr(m, nnz, ctypes.c_void_p(rowptr.data_ptr()), ctypes.c_void_p(colidx.data_ptr()),
+                              ctypes.c_void_p(values.data_ptr()), _dtype_code(values.dtype),
+                              ctypes.c_void_p(perm.data_ptr()), ctypes.c_void_p(rp.data_ptr()),
+                              ctypes.c_void_p(ci.data_ptr()), ctypes.c_void_p(v.data_ptr()), _stream_ptr(stream)),
+           "spaden_permute_csr")
+    return rp, ci, v
 
 
 def convert(rowptr, colidx, values, n: int, storage=None, stream=None, residual_max_popc: int = 0,

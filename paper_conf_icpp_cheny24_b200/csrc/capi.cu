@@ -227,6 +227,75 @@ spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n, int64_t nn
     return SPADEN_OK;
 }
 
+namespace spaden_capi_kernels {
+__global__ void k_col_range(int64_t nnz, int64_t n, const int32_t *__restrict__ colidx, uint32_t *flag) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x)
+        if (colidx[e] < 0 || colidx[e] >= n) atomicOr(flag, 1u);
+}
+}  // namespace spaden_capi_kernels
+
+spaden_status_t spaden_degree_order(int64_t m, const int32_t *d_rowptr, int32_t *d_perm, void *stream) {
+    g_last_error.clear();
+    if (m < 0 || m >= (1LL << 31) - 8) {
+        set_error("m must be in [0, 2^31)");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (m == 0) return SPADEN_OK;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_status(e, "cudaGetDevice");
+    spaden_status_t s = check_device_ptr(d_rowptr, "rowptr", dev);
+    if (s == SPADEN_OK) s = check_device_ptr(d_perm, "perm", dev);
+    if (s != SPADEN_OK) return s;
+    return degree_order(m, d_rowptr, d_perm, (cudaStream_t)stream);
+}
+
+spaden_status_t spaden_permute_csr(int64_t m, int64_t nnz, const int32_t *d_rowptr, const int32_t *d_colidx,
+                                   const void *d_values, spaden_dtype_t dtype, const int32_t *d_perm,
+                                   int32_t *d_out_rowptr, int32_t *d_out_colidx, void *d_out_values,
+                                   void *stream) {
+    g_last_error.clear();
+    if (m < 0 || nnz < 0 || m >= (1LL << 31) - 8 || nnz >= (1LL << 31) - 1) {
+        set_error("m, nnz must be in [0, 2^31)");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
+    if (dtype != SPADEN_R_32F && dtype != SPADEN_R_16F) {
+        set_error("dtype must be SPADEN_R_32F or SPADEN_R_16F");
+        return SPADEN_ERR_UNSUPPORTED;
+    }
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_status(e, "cudaGetDevice");
+    spaden_status_t s = check_device_ptr(d_rowptr, "rowptr", dev);
+    if (s == SPADEN_OK) s = check_device_ptr(d_out_rowptr, "out_rowptr", dev);
+    if (s == SPADEN_OK && m > 0) s = check_device_ptr(d_perm, "perm", dev);
+    if (s == SPADEN_OK && nnz > 0) s = check_device_ptr(d_colidx, "colidx", dev);
+    if (s == SPADEN_OK && nnz > 0) s = check_device_ptr(d_values, "values", dev);
+    if (s == SPADEN_OK && nnz > 0) s = check_device_ptr(d_out_colidx, "out_colidx", dev);
+    if (s == SPADEN_OK && nnz > 0) s = check_device_ptr(d_out_values, "out_values", dev);
+    if (s != SPADEN_OK) return s;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (nnz > 0) {
+        uint32_t *flag = nullptr, h = 0;
+        e = dmalloc(&flag, sizeof(uint32_t), st);
+        if (e == cudaSuccess) e = cudaMemsetAsync(flag, 0, sizeof(uint32_t), st);
+        if (e == cudaSuccess) {
+            spaden_capi_kernels::k_col_range<<<(unsigned)std::min<int64_t>((nnz + 255) / 256, 148 * 64), 256, 0, st>>>(nnz, m, d_colidx,
+                                                                                                   flag);
+            e = cudaMemcpyAsync(&h, flag, sizeof(h), cudaMemcpyDeviceToHost, st);
+        }
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        dev_free(flag, st);
+        if (e != cudaSuccess) return cuda_status(e, "checking column range");
+        if (h) {
+            set_error("a column index is outside [0, m)");
+            return SPADEN_ERR_INDEX_OUT_OF_RANGE;
+        }
+    }
+    return permute_csr(m, nnz, d_rowptr, d_colidx, d_values, dtype == SPADEN_R_16F ? 2 : 4, d_perm, d_out_rowptr,
+                       d_out_colidx, d_out_values, st);
+}
+
 spaden_status_t spaden_count_blocks(int64_t m, int64_t n, int64_t nnz, const int32_t *d_rowptr,
                                     const int32_t *d_colidx, void *stream, int64_t *Bnnz) {
     g_last_error.clear();

@@ -269,6 +269,12 @@ spaden_status_t spmm_tc_pack_x(int64_t n, int32_t k, const float *X, int64_t ldx
 spaden_status_t spmm_tc_launch(Matrix &A, float alpha, const void *Xb, int32_t k, float beta, float *Y,
                                int64_t ldy, cudaStream_t stream);  // builds the chunk schedule at the first call
 
+// reordering (reorder.cu)
+spaden_status_t degree_order(int64_t m, const int32_t *rowptr, int32_t *perm, cudaStream_t st);
+spaden_status_t permute_csr(int64_t m, int64_t nnz, const int32_t *rowptr, const int32_t *colidx, const void *values,
+                            int value_bytes, const int32_t *perm, int32_t *out_rowptr, int32_t *out_colidx,
+                            void *out_values, cudaStream_t st);
+
 // exclusive scan of int32 (scan.cu): out[i] = sum_{j<i} in[j], out[count] = total.
 // `in` and `out` may alias.  tmp must hold scan_tmp_ints(count) int32.
 size_t scan_tmp_ints(int64_t count);

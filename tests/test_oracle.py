@@ -389,3 +389,43 @@ def test_hybrid_split_partitions_entries(t):
     yk, _ = oracle.spmv(krp, kci, kv, x)
     yr, _ = oracle.spmv(rrp, rci, rv, x)
     np.testing.assert_allclose(yk + yr, y, rtol=1e-12, atol=1e-12)
+
+
+# ------------------------------------------------ reordering (NEXT-1)
+def test_degree_order_hand_worked():
+    """Degrees [1, 3, 0, 3, 2] -> descending, ties in ascending row order:
+    rows 1, 3 (degree 3), 4 (2), 0 (1), 2 (0)."""
+    rp = np.array([0, 1, 4, 4, 7, 9], np.int32)
+    assert oracle.degree_order(rp).tolist() == [1, 3, 4, 0, 2]
+
+
+def test_degree_order_closed_forms():
+    n = 37
+    eye = W.from_dense(np.eye(n, dtype=np.float32))
+    assert np.array_equal(oracle.degree_order(eye.rowptr), np.arange(n))        # all equal: identity
+    low = W.from_dense(np.tril(np.ones((n, n), np.float32)))
+    assert np.array_equal(oracle.degree_order(low.rowptr), np.arange(n)[::-1])  # degree i+1: reversal
+    assert oracle.degree_order(np.zeros(1, np.int32)).size == 0                  # m = 0
+
+
+@pytest.mark.parametrize("m,dens,seed", [(1, 1.0, 0), (13, 0.3, 1), (64, 0.08, 2), (200, 0.02, 3)])
+def test_permute_csr_vs_dense(m, dens, seed):
+    """B = P A P^T against dense indexing B = A[perm][:, perm] (a different
+    mechanism than the oracle's entry relabelling + lexsort), and the SpMV
+    identity B (P x) = P (A x)."""
+    A = W.random_sparse(m, m, dens, seed)
+    for perm in (oracle.degree_order(A.rowptr), W.random_perm(m, seed + 7)):
+        rp, ci, v = oracle.permute_csr(A.rowptr, A.colidx, A.values, perm)
+        B = W.CSR(m, m, rp, ci, v)
+        dense_a = np.zeros((m, m), np.float32)
+        for i in range(m):
+            dense_a[i, A.colidx[A.rowptr[i]:A.rowptr[i + 1]]] = A.values[A.rowptr[i]:A.rowptr[i + 1]]
+        dense_b = np.zeros((m, m), np.float32)
+        for i in range(m):
+            dense_b[i, ci[rp[i]:rp[i + 1]]] = v[rp[i]:rp[i + 1]]
+        assert np.array_equal(dense_b, dense_a[perm][:, perm])
+        assert all(np.all(np.diff(ci[rp[i]:rp[i + 1]]) > 0) for i in range(m))   # canonical rows
+        x = W.vector(m, seed)
+        y, _ = oracle.spmv(A.rowptr, A.colidx, A.values, x)
+        yb, _ = oracle.spmv(rp, ci, v, x[perm])
+        assert np.allclose(yb, y[perm], rtol=1e-12, atol=1e-12)
