@@ -160,6 +160,11 @@ constexpr int kBlockStageBytes = 16 + 36;
 // + 1 byte per block when the schedule carries row rotations (the rotation region);
 // the long-row cost (kLongRowBytes) is computed with kBlockStageBytes alone
 constexpr int kBlockRotBytes = 1;
+// row-rotated decode stores a block's 8 row partials as two 16-byte stores
+// (spmv.cu block_slots_rot_v4): the rotation pass then models the value loads only
+#ifndef SPADEN_ROT_V4
+#define SPADEN_ROT_V4 1
+#endif
 // A block-row whose stage cost (kBlockStageBytes per block + its values + 4)
 // exceeds kLongRowBytes is "long" (chunk path) whatever the tile config: the
 // split between the tile path and the chunk path -- two different summation

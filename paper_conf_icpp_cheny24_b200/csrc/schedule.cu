@@ -146,9 +146,10 @@ k_rot_greedy(const TileDesc *__restrict__ tiles, int ntiles, const uint64_t *__r
                 }
             }
             // the block's partial stores: step t writes row (t + r) & 7 at word
-            // 9 * lane + row of the unit's scratch (kPartStride = 36 bytes)
+            // 9 * lane + row of the unit's scratch (kPartStride = 36 bytes); the
+            // vectorised stores (SPADEN_ROT_V4) are conflict free whatever r
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
+            for (int h = 0; h < (SPADEN_ROT_V4 ? 0 : 2); ++h) {
                 const int tt = 2 * (j >> 3) + h;
                 const int bank = (9 * l + ((tt + r) & 7)) & 31;
                 delta += (sload[w][tt][bank] + 1 > smx[w][tt]) ? 1 : 0;

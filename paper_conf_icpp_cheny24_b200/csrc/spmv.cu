@@ -138,6 +138,10 @@ __device__ __forceinline__ void sts_f32(uint32_t a, float v) {
 // row partials of a block: 8 floats at a 9-word stride (bank-conflict-free
 // per-lane stores and phase-2 reads)
 constexpr uint32_t kPartStride = 36;
+// row-rotated decode (ROT): the 8 row partials of a block, un-rotated in
+// registers, leave as two 16-byte stores at a 32-byte stride (conflict free)
+constexpr bool kRotV4 = SPADEN_ROT_V4 != 0;
+constexpr uint32_t kPartStrideV4 = 32;
 
 // Value source of a block's packed run: shared-memory stage or global memory.
 template <typename V> struct SmemVals {
@@ -253,6 +257,55 @@ __device__ __forceinline__ void block_slots_rot(uint2 bm, uint32_t rho, typename
     }
 }
 
+__device__ __forceinline__ void sts_v4(uint32_t a, float x, float y, float z, float w) {
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"(x), "f"(y), "f"(z), "f"(w) : "memory");
+}
+
+// block_slots_rot with the partials kept in registers: step t computes original
+// row (t + rho) & 7; a two-stage select network rotates the 8 sums back into
+// row order (by rho & 3), rotation by 4 swaps the two 16-byte stores.  Same
+// fma chains as block_slots_rot.
+template <class VS>
+__device__ __forceinline__ void block_slots_rot_v4(uint2 bm, uint32_t rho, typename VS::P p0, const XSeg &xs,
+                                                   uint32_t q) {
+    const uint64_t b = ((uint64_t)bm.y << 32) | bm.x;
+    const uint32_t sh = 8u * rho;
+    const uint64_t rb = sh ? ((b >> sh) | (b << (64u - sh))) : b;
+    const int P = __popcll(b);
+    const int B = __popcll(b & ((1ull << sh) - 1ull));
+    const uint32_t rlo = (uint32_t)rb, rhi = (uint32_t)(rb >> 32);
+    float acc[8];
+#pragma unroll
+    for (int t = 0; t < 8; ++t) {
+        const uint32_t w = t < 4 ? rlo : rhi;
+        const uint32_t byte = (w >> (8 * (t & 3))) & 0xffu;
+        int below = (t & 3) == 0 ? 0 : __popc(w & ((1u << (8 * (t & 3))) - 1u));
+        if (t >= 4) below += __popc(rlo);
+        int start = below + B;
+        start = start >= P ? start - P : start;
+        typename VS::P p = p0 + start * VS::step;
+        float a = 0.f;
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+            if ((byte >> c) & 1u) {
+                a = fmaf(VS::get(p), xs.v[c], a);
+                p += VS::step;
+            }
+        }
+        acc[t] = a;
+    }
+    // row r = (t + rho) & 7 holds acc[t]: o[r] = acc[(r - rho) & 7]
+    float s1[8], s2[8];
+    const bool r1 = rho & 1u, r2 = rho & 2u;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) s1[i] = r1 ? acc[(i + 7) & 7] : acc[i];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) s2[i] = r2 ? s1[(i + 6) & 7] : s1[i];
+    const uint32_t lo = (rho & 4u) ? 16u : 0u;
+    sts_v4(q + lo, s2[0], s2[1], s2[2], s2[3]);
+    sts_v4(q + (16u - lo), s2[4], s2[5], s2[6], s2[7]);
+}
+
 template <class VS>
 __device__ __forceinline__ void block_slots(uint2 bm, typename VS::P p0, const XSeg &xs, float acc[8]) {
     block_slots_at<VS>(bm, p0, p0 + __popc(bm.x) * VS::step, xs, acc);
@@ -306,6 +359,7 @@ __device__ __forceinline__ void store_y(float *__restrict__ y, int64_t row, floa
 // Phase 2: y for every block-row of a tile from the per-block row partials
 // (9-word stride), 4 block-rows x 8 rows per warp pass, 4 chains per row
 // indexed by block position within the block-row, combined (c0+c1)+(c2+c3).
+template <uint32_t kStride = kPartStride>
 __device__ __forceinline__ void reduce_tile(uint32_t a_rp, uint32_t a_part, int nbr, int b0, int br0, int lane,
                                             int64_t m, float alpha, float beta, float *__restrict__ y,
                                             const PeerOut &po) {
@@ -316,17 +370,17 @@ __device__ __forceinline__ void reduce_tile(uint32_t a_rp, uint32_t a_part, int 
             const int k0 = lds_i32(a_rp + 4u * brl) - b0;
             const int k1 = lds_i32(a_rp + 4u * (brl + 1)) - b0;
             float c0 = 0.f, c1 = 0.f, c2 = 0.f, c3 = 0.f;
-            uint32_t q = a_part + kPartStride * k0 + 4u * r;
+            uint32_t q = a_part + kStride * k0 + 4u * r;
             int k = k0;
-            for (; k + 3 < k1; k += 4, q += 4 * kPartStride) {
+            for (; k + 3 < k1; k += 4, q += 4 * kStride) {
                 c0 += lds_f32(q);
-                c1 += lds_f32(q + kPartStride);
-                c2 += lds_f32(q + 2 * kPartStride);
-                c3 += lds_f32(q + 3 * kPartStride);
+                c1 += lds_f32(q + kStride);
+                c2 += lds_f32(q + 2 * kStride);
+                c3 += lds_f32(q + 3 * kStride);
             }
             if (k < k1) c0 += lds_f32(q);
-            if (k + 1 < k1) c1 += lds_f32(q + kPartStride);
-            if (k + 2 < k1) c2 += lds_f32(q + 2 * kPartStride);
+            if (k + 1 < k1) c1 += lds_f32(q + kStride);
+            if (k + 2 < k1) c2 += lds_f32(q + 2 * kStride);
             const float sum = (c0 + c1) + (c2 + c3);
             const int64_t row = 8 * ((int64_t)br0 + brl) + r;
             if (row < m) {
@@ -717,10 +771,12 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
                 for (int h = 0; h < BPL; ++h) {
                     const int lb = lbs[h];
                     if (lb >= nb) continue;
-                    const uint32_t q = a_part + kPartStride * lb;
-                    if constexpr (ROT) {
-                        block_slots_rot<SmemVals<V>>(bms[h], rhos[h], ps[h], xss[h], q);
+                    if constexpr (ROT && kRotV4) {
+                        block_slots_rot_v4<SmemVals<V>>(bms[h], rhos[h], ps[h], xss[h], a_part + kPartStrideV4 * lb);
+                    } else if constexpr (ROT) {
+                        block_slots_rot<SmemVals<V>>(bms[h], rhos[h], ps[h], xss[h], a_part + kPartStride * lb);
                     } else {
+                        const uint32_t q = a_part + kPartStride * lb;
                         float acc[8];
                         const uint2 bm = bms[h];
                         const SwapHalves sw{sizeof(V) == 2 && ((lane >> 1) & 1)};
@@ -768,6 +824,8 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
             const int4 h2 = lds_i4_volatile(a_hdr + 32u);  // br0, nbr, b0, a_rp
             if constexpr (K > 1)
                 reduce_tile_k<K>((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, ldy);
+            else if constexpr (DEC == 1 && ROT && kRotV4)
+                reduce_tile<kPartStrideV4>((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, po);
             else
                 reduce_tile((uint32_t)h2.w, a_part, h2.y, h2.z, h2.x, lane, m, alpha, beta, y, po);
             __syncwarp();
