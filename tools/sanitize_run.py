@@ -69,4 +69,13 @@ for C in (A, B, W.h2()):
     Mh.spmm_tc(Xb, 70, Yk, alpha=0.5, beta=0.5)
     torch.cuda.synchronize()
     Mh.free()
+# reordering (NEXT-1): degree order + P A P^T, then the hybrid SpMV on it
+P = W.powerlaw(12, 5, 1, relabel=True)
+rp, ci, v = (torch.from_numpy(a).cuda() for a in (P.rowptr, P.colidx, P.values))
+perm = sp.degree_order(rp)
+rp2, ci2, v2 = sp.permute_csr(rp, ci, v, perm)
+MR = sp.convert(rp2, ci2, v2, P.n, residual_max_popc=-1)
+MR.spmv(torch.from_numpy(W.vector(P.n, 3)).cuda())
+torch.cuda.synchronize()
+MR.free()
 print("sanitize run ok")
