@@ -38,9 +38,9 @@ __global__ void k_entry_keys(int64_t m, int cb, const int32_t *__restrict__ rowp
     const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < m; i += warps) {
         const uint64_t hi = (uint64_t)(uint32_t)iperm[i] << cb;
-        for (int e = rowptr[i] + lane; e < rowptr[i + 1]; e += 32) {
+        for (int64_t e = (int64_t)rowptr[i] + lane; e < rowptr[i + 1]; e += 32) {  // int64: nnz may reach 2^31 - 2
             key[e] = hi | (uint32_t)iperm[colidx[e]];
-            idx[e] = e;
+            idx[e] = (int32_t)e;
         }
     }
 }
