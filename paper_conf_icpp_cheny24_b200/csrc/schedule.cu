@@ -113,8 +113,9 @@ constexpr int kRotWarps = 8;
 template <int SV>
 __global__ void __launch_bounds__(32 * kRotWarps)
 k_rot_greedy(const TileDesc *__restrict__ tiles, int ntiles, const uint64_t *__restrict__ bitmap,
-             const int32_t *__restrict__ blk_offset, uint8_t *__restrict__ rot) {
+             const int32_t *__restrict__ blk_offset, uint8_t *__restrict__ rot, int passes) {
     __shared__ uint8_t load[kRotWarps][64][32];  // words per (slot instruction, bank) so far
+    __shared__ uint8_t rho_s[kRotWarps][32];     // the unit's chosen rotations (local-search passes)
     __shared__ uint8_t mx[kRotWarps][64];        // max over banks = wavefronts of the instruction
     __shared__ uint8_t sload[kRotWarps][8][32];  // the 8 partial stores (step t -> row (t+rho)&7)
     __shared__ uint8_t smx[kRotWarps][8];
@@ -179,10 +180,84 @@ k_rot_greedy(const TileDesc *__restrict__ tiles, int ntiles, const uint64_t *__r
                 sload[w][j][bank] = (uint8_t)nl;
                 if (nl > smx[w][j]) smx[w][j] = (uint8_t)nl;
             }
-            if (j == 0) rot[ub + l] = (uint8_t)best;
+            if (j == 0) {
+                rot[ub + l] = (uint8_t)best;
+                rho_s[w][l] = (uint8_t)best;
+            }
             __syncwarp();
         }
+        // local search (value loads only, SPADEN_ROT_V4): take each lane's block out
+        // again, recompute the maxima it may have set, and re-pick its rotation
+        // against all the other lanes of the unit (never worse than the greedy)
+        for (int pass = 0; SPADEN_ROT_V4 && pass < passes; ++pass) {
+            for (int l = 0; l < nbu; ++l) {
+                const uint64_t bm = __ldg(bitmap + ub + l);
+                const int off = __ldg(blk_offset + ub + l);
+                const int cur = rho_s[w][l];
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {  // remove
+                    const int sl = j + 32 * h;
+                    if ((bm >> sl) & 1ull) {
+                        const int rank = __popcll(bm & ((1ull << sl) - 1ull));
+                        const int bank = (int)((((int64_t)off + rank) * SV) >> 2) & 31;
+                        const int ins = 8 * (((sl >> 3) - cur) & 7) + (sl & 7);
+                        load[w][ins][bank] = (uint8_t)(load[w][ins][bank] - 1);
+                    }
+                }
+                __syncwarp();
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {  // maxima of every instruction (lane j: j, j + 32)
+                    const int ins = j + 32 * h;
+                    int mm = 0;
+                    for (int bk = 0; bk < 32; ++bk) mm = max(mm, (int)load[w][ins][(bk + j) & 31]);
+                    mx[w][ins] = (uint8_t)mm;
+                }
+                __syncwarp();
+                int delta = 0;
+#pragma unroll 4
+                for (int k = 0; k < 16; ++k) {
+                    const int sl = (j >> 3) + 4 * k;
+                    if ((bm >> sl) & 1ull) {
+                        const int rank = __popcll(bm & ((1ull << sl) - 1ull));
+                        const int bank = (int)((((int64_t)off + rank) * SV) >> 2) & 31;
+                        const int ins = 8 * (((sl >> 3) - r) & 7) + (sl & 7);
+                        delta += (load[w][ins][bank] + 1 > mx[w][ins]) ? 1 : 0;
+                    }
+                }
+                delta += __shfl_xor_sync(0xffffffffu, delta, 8);
+                delta += __shfl_xor_sync(0xffffffffu, delta, 16);
+                // prefer the current rotation on ties (the search then only moves downhill)
+                int key = delta * 16 + (r == cur ? 0 : 8) + r;
+                key = min(key, __shfl_xor_sync(0xffffffffu, key, 1));
+                key = min(key, __shfl_xor_sync(0xffffffffu, key, 2));
+                key = min(key, __shfl_xor_sync(0xffffffffu, key, 4));
+                const int best = key & 7;
+                __syncwarp();
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {  // add back with the chosen rotation
+                    const int sl = j + 32 * h;
+                    if ((bm >> sl) & 1ull) {
+                        const int rank = __popcll(bm & ((1ull << sl) - 1ull));
+                        const int bank = (int)((((int64_t)off + rank) * SV) >> 2) & 31;
+                        const int ins = 8 * (((sl >> 3) - best) & 7) + (sl & 7);
+                        const int nl = load[w][ins][bank] + 1;
+                        load[w][ins][bank] = (uint8_t)nl;
+                        if (nl > mx[w][ins]) mx[w][ins] = (uint8_t)nl;
+                    }
+                }
+                if (j == 0) {
+                    rot[ub + l] = (uint8_t)best;
+                    rho_s[w][l] = (uint8_t)best;
+                }
+                __syncwarp();
+            }
+        }
     }
+}
+
+int rotation_passes() {  // SPADEN_ROT_PASSES: local-search passes after the greedy (default 1), read per conversion
+    const char *e = getenv("SPADEN_ROT_PASSES");
+    return e ? atoi(e) : 1;
 }
 
 bool rotation_enabled() {  // SPADEN_ROT=0 disables (A/B, tests), read per conversion
@@ -292,9 +367,11 @@ spaden_status_t build_schedule(Matrix *A, cudaStream_t st) {
         if (e == cudaSuccess) {
             const unsigned g = (unsigned)((A->n_tiles + kRotWarps - 1) / kRotWarps);
             if (sv == 2)
-                k_rot_greedy<2><<<g, 32 * kRotWarps, 0, st>>>(A->tiles, (int)A->n_tiles, A->bitmap, A->blk_offset, A->rot);
+                k_rot_greedy<2><<<g, 32 * kRotWarps, 0, st>>>(A->tiles, (int)A->n_tiles, A->bitmap, A->blk_offset, A->rot,
+                                                              rotation_passes());
             else
-                k_rot_greedy<4><<<g, 32 * kRotWarps, 0, st>>>(A->tiles, (int)A->n_tiles, A->bitmap, A->blk_offset, A->rot);
+                k_rot_greedy<4><<<g, 32 * kRotWarps, 0, st>>>(A->tiles, (int)A->n_tiles, A->bitmap, A->blk_offset, A->rot,
+                                                              rotation_passes());
             e = cudaGetLastError();
         }
         if (e != cudaSuccess) return cuda_status(e, "row-rotation schedule");
