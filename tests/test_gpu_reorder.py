@@ -125,3 +125,37 @@ def test_empty_matrix(sp, torch):
                                   torch.zeros(0, dtype=torch.float32, device="cuda"), perm)
     torch.cuda.synchronize()
     assert brp.cpu().tolist() == [0]
+
+
+def test_rmat25_reordered_hybrid_sampled(sp, torch):
+    """The bench's `--workload rmat25 --reorder degree` path at full size (1.05B
+    nnz): degree order and P A P^T on the GPU, automatic hybrid; the permutation is
+    checked against the oracle's definition on the row degrees, and y' = B (P x)
+    on 4096 sampled rows (incl. the hubs) against the fp64 oracle's P (A x) rows."""
+    rp, ci, v, n, nnz = W.pagerank_slice_torch(25, 32, 0, 1 << 25, seed=0, device="cuda")
+    perm = sp.degree_order(rp)
+    torch.cuda.synchronize()
+    rph = rp.cpu().numpy().astype(np.int64)
+    assert np.array_equal(perm.cpu().numpy(), oracle.degree_order(rph))
+    brp, bci, bv = sp.permute_csr(rp, ci, v, perm)
+    M = sp.convert(brp, bci, bv, n, residual_max_popc=-1)
+    torch.cuda.synchronize()
+    assert M.info.nnz == nnz
+    g = torch.Generator(device="cuda")
+    g.manual_seed(7)
+    x = torch.rand(n, generator=g, device="cuda")
+    xp = x[perm.long()].contiguous()
+    y = M.spmv(xp)
+    torch.cuda.synchronize()
+    p = perm.cpu().numpy()
+    lens = np.diff(rph)
+    rng = np.random.default_rng(5)
+    krows = np.unique(np.concatenate([rng.choice(n, 4064, replace=False), np.arange(32)]))  # B's first rows = hubs
+    orig = p[krows]  # row k of B is row perm[k] of A
+    sub_rp = np.zeros(orig.size + 1, np.int64)
+    sub_rp[1:] = np.cumsum(lens[orig])
+    idx = torch.from_numpy(np.concatenate([np.arange(rph[r], rph[r + 1]) for r in orig])).cuda()
+    ys, s = oracle.spmv(sub_rp, ci[idx].cpu().numpy(), v[idx].cpu().numpy(), x.cpu().numpy())
+    err = oracle.componentwise_error(y[torch.from_numpy(krows).cuda()].cpu().numpy(), ys, s)
+    assert err <= TOL32, err
+    M.free()
