@@ -151,6 +151,28 @@ __device__ __forceinline__ void tc_wait(uint32_t bar, uint32_t parity) {
             : "memory");
     }
 }
+// MMA-issue warps: poll without the suspend hint and back off with __nanosleep
+// (their polls otherwise take issue slots from the decode warps)
+#ifndef SPADEN_TC_MMA_BACKOFF
+#define SPADEN_TC_MMA_BACKOFF 64
+#endif
+__device__ __forceinline__ void tc_wait_mma(uint32_t bar, uint32_t parity) {
+    if (!SPADEN_TC_MMA_BACKOFF) {
+        tc_wait(bar, parity);
+        return;
+    }
+    uint32_t ok = 0, ns = 32;
+    while (true) {
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(ok)
+            : "r"(bar), "r"(parity)
+            : "memory");
+        if (ok) return;
+        __nanosleep(ns);
+        ns = ns < SPADEN_TC_MMA_BACKOFF ? 2 * ns : ns;
+    }
+}
 __device__ __forceinline__ void tc_bulk(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
     asm volatile(
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
@@ -499,18 +521,18 @@ k_spmm_tc(int64_t m, const TcChunk *__restrict__ chunks, const TcRec *__restrict
         for (int c = warp == kMma ? 0 : 1; c < nch; c += 2) {
             const int a = c % kTcRing, b = c % kTcSlabBufs;
             if (lane == 0) TR(2, c, 0);
-            tc_wait(s_u32(&bar_arr[a]), ring_ph(c));
+            tc_wait_mma(s_u32(&bar_arr[a]), ring_ph(c));
             if (lane == 0) TR(2, c, 1);
-            tc_wait(s_u32(&bar_tiles[a]), ring_ph(c));
+            tc_wait_mma(s_u32(&bar_tiles[a]), ring_ph(c));
             if (lane == 0) TR(2, c, 2);
-            tc_wait(s_u32(&bar_slab[b]), slab_ph(c));
+            tc_wait_mma(s_u32(&bar_slab[b]), slab_ph(c));
             if (lane == 0) TR(2, c, 3);
             // accumulator slots: the epilogue has finished chunk c-3
             // (chunks c-2 .. c hold at most 3 * kTcPairs < kTcSlots started block-rows)
-            if (c >= 3) tc_wait(s_u32(&bar_epi[(c - 3) % kTcRing]), ring_ph(c - 3));
+            if (c >= 3) tc_wait_mma(s_u32(&bar_epi[(c - 3) % kTcRing]), ring_ph(c - 3));
             // a block-row continued from the previous chunk accumulates after that
             // chunk's MMAs (issued by the other warp) have completed
-            if (c >= 1 && cdesc[a].pA > 0) tc_wait(s_u32(&bar_mma[(c - 1) % kTcRing]), ring_ph(c - 1));
+            if (c >= 1 && cdesc[a].pA > 0) tc_wait_mma(s_u32(&bar_mma[(c - 1) % kTcRing]), ring_ph(c - 1));
             if (lane == 0) TR(2, c, 4);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
             // the record's head and segments (bytes 0..33): three loads in flight at once
