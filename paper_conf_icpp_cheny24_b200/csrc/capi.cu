@@ -8,7 +8,20 @@
 #include <new>
 #include <string>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "internal.cuh"
+
+
+// NVTX range over a C-ABI call (named after the entry point): profilers (ncu
+// --nvtx, nsys) can attribute the call's kernels; near free without a tool
+namespace {
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+}  // namespace
+#define SPADEN_NVTX(name) NvtxRange nvtx_range_(name)
 
 namespace spaden {
 
@@ -162,6 +175,7 @@ spaden_status_t spaden_convert_csr_to_bitmap_ex(int64_t m, int64_t n, int64_t nn
                                                 spaden_dtype_t values_dtype, spaden_dtype_t storage_dtype,
                                                 const spaden_convert_opts_t *opts, void *stream,
                                                 spaden_matrix_t *out) {
+    SPADEN_NVTX("spaden_convert_csr_to_bitmap_ex");
     g_last_error.clear();
     int res_t = 0;
     float auto_fill = 0.f;
@@ -235,6 +249,7 @@ __global__ void k_col_range(int64_t nnz, int64_t n, const int32_t *__restrict__ 
 }  // namespace spaden_capi_kernels
 
 spaden_status_t spaden_degree_order(int64_t m, const int32_t *d_rowptr, int32_t *d_perm, void *stream) {
+    SPADEN_NVTX("spaden_degree_order");
     g_last_error.clear();
     if (m < 0 || m >= (1LL << 31) - 8) {
         set_error("m must be in [0, 2^31)");
@@ -254,6 +269,7 @@ spaden_status_t spaden_permute_csr(int64_t m, int64_t nnz, const int32_t *d_rowp
                                    const void *d_values, spaden_dtype_t dtype, const int32_t *d_perm,
                                    int32_t *d_out_rowptr, int32_t *d_out_colidx, void *d_out_values,
                                    void *stream) {
+    SPADEN_NVTX("spaden_permute_csr");
     g_last_error.clear();
     if (m < 0 || nnz < 0 || m >= (1LL << 31) - 8 || nnz >= (1LL << 31) - 1) {
         set_error("m, nnz must be in [0, 2^31)");
@@ -298,6 +314,7 @@ spaden_status_t spaden_permute_csr(int64_t m, int64_t nnz, const int32_t *d_rowp
 
 spaden_status_t spaden_count_blocks(int64_t m, int64_t n, int64_t nnz, const int32_t *d_rowptr,
                                     const int32_t *d_colidx, void *stream, int64_t *Bnnz) {
+    SPADEN_NVTX("spaden_count_blocks");
     g_last_error.clear();
     if (!Bnnz) {
         set_error("Bnnz must not be NULL");
@@ -332,6 +349,7 @@ spaden_status_t spaden_count_blocks(int64_t m, int64_t n, int64_t nnz, const int
 
 spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const float *d_x, float beta, float *d_y,
                             void *stream) {
+    SPADEN_NVTX("spaden_spmv");
     if (!A) {
         set_error("NULL matrix handle");
         return SPADEN_ERR_INVALID_ARGUMENT;
@@ -353,6 +371,7 @@ spaden_status_t spaden_spmv(spaden_matrix_t A, float alpha, const float *d_x, fl
 
 spaden_status_t spaden_spmv_scatter(spaden_matrix_t A, float alpha, const float *d_x, float beta, float *d_y,
                                     float *const *h_out_ptrs, int32_t npeers, int64_t out_offset, void *stream) {
+    SPADEN_NVTX("spaden_spmv_scatter");
     if (!A || npeers < 1 || npeers > kMaxPeers || !h_out_ptrs || out_offset < 0 ||
         (A->Bnnz > 0 && !d_x) || (beta != 0.f && A->m > 0 && !d_y)) {
         set_error("bad arguments (handle, 1 <= npeers <= 8, out pointers, x, y with beta != 0)");
@@ -373,6 +392,7 @@ spaden_status_t spaden_spmv_scatter(spaden_matrix_t A, float alpha, const float 
 
 spaden_status_t spaden_spmm(spaden_matrix_t A, float alpha, const float *d_X, int64_t ldx, int32_t k, float beta,
                             float *d_Y, int64_t ldy, void *stream) {
+    SPADEN_NVTX("spaden_spmm");
     if (!A || k < 0 || ldx < A->n || ldy < A->m || (k > 0 && ((A->m > 0 && !d_Y) || (A->Bnnz > 0 && !d_X)))) {
         set_error("NULL handle/matrices, k < 0, or ldx < n / ldy < m");
         return SPADEN_ERR_INVALID_ARGUMENT;
@@ -396,6 +416,7 @@ int64_t spaden_spmm_tc_xb_bytes(int64_t n, int32_t k) {
 
 spaden_status_t spaden_spmm_tc_pack_x(int64_t n, int32_t k, const float *d_X, int64_t ldx, void *d_Xb,
                                       void *stream) {
+    SPADEN_NVTX("spaden_spmm_tc_pack_x");
     g_last_error.clear();
     if (n < 0 || k < 0 || ldx < n || (n > 0 && k > 0 && (!d_X || !d_Xb)) || ((uintptr_t)d_Xb & 15u)) {
         set_error("bad arguments (n, k >= 0, ldx >= n, non-NULL 16-byte aligned d_Xb)");
@@ -406,6 +427,7 @@ spaden_status_t spaden_spmm_tc_pack_x(int64_t n, int32_t k, const float *d_X, in
 
 spaden_status_t spaden_spmm_tc(spaden_matrix_t A, float alpha, const void *d_Xb, int32_t k, float beta, float *d_Y,
                                int64_t ldy, void *stream) {
+    SPADEN_NVTX("spaden_spmm_tc");
     g_last_error.clear();
     if (!A || k < 0 || ldy < A->m || (k > 0 && A->m > 0 && (!d_Y || !d_Xb)) || ((uintptr_t)d_Xb & 15u)) {
         set_error("NULL handle/matrices, k < 0, ldy < m, or d_Xb not 16-byte aligned");
@@ -428,6 +450,7 @@ spaden_status_t spaden_spmm_tc(spaden_matrix_t A, float alpha, const void *d_Xb,
 
 spaden_status_t spaden_spmv_host(spaden_matrix_t A, float alpha, const float *h_x, float beta, float *h_y,
                                  void *stream) {
+    SPADEN_NVTX("spaden_spmv_host");
     if (!A || (A->n > 0 && !h_x) || (A->m > 0 && !h_y)) {
         set_error("NULL handle or host vector");
         return SPADEN_ERR_INVALID_ARGUMENT;
@@ -449,6 +472,7 @@ spaden_status_t spaden_spmv_host(spaden_matrix_t A, float alpha, const float *h_
 
 spaden_status_t spaden_spmv_host_batched(spaden_matrix_t A, float alpha, const float *h_x, int64_t ldx,
                                          float beta, float *h_y, int64_t ldy, int64_t nvec, void *stream) {
+    SPADEN_NVTX("spaden_spmv_host_batched");
     if (!A || nvec < 0 || (nvec > 0 && ((A->n > 0 && !h_x) || (A->m > 0 && !h_y))) || ldx < A->n ||
         ldy < A->m) {
         set_error("NULL handle/vectors, nvec < 0, or ldx < n / ldy < m");
@@ -493,6 +517,7 @@ spaden_status_t spaden_spmv_host_batched(spaden_matrix_t A, float alpha, const f
 }
 
 spaden_status_t spaden_free(spaden_matrix_t A) {
+    SPADEN_NVTX("spaden_free");
     if (!A) return SPADEN_OK;
     int cur = 0;
     const int dev = A->device;
