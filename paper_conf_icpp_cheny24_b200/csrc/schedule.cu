@@ -194,6 +194,7 @@ k_rot_greedy(const TileDesc *__restrict__ tiles, int ntiles, const uint64_t *__r
                 const uint64_t bm = __ldg(bitmap + ub + l);
                 const int off = __ldg(blk_offset + ub + l);
                 const int cur = rho_s[w][l];
+                int touched[2] = {-1, -1};  // instructions this lane's slots j, j + 32 used
 #pragma unroll
                 for (int h = 0; h < 2; ++h) {  // remove
                     const int sl = j + 32 * h;
@@ -202,15 +203,18 @@ k_rot_greedy(const TileDesc *__restrict__ tiles, int ntiles, const uint64_t *__r
                         const int bank = (int)((((int64_t)off + rank) * SV) >> 2) & 31;
                         const int ins = 8 * (((sl >> 3) - cur) & 7) + (sl & 7);
                         load[w][ins][bank] = (uint8_t)(load[w][ins][bank] - 1);
+                        touched[h] = ins;
                     }
                 }
                 __syncwarp();
 #pragma unroll
-                for (int h = 0; h < 2; ++h) {  // maxima of every instruction (lane j: j, j + 32)
-                    const int ins = j + 32 * h;
-                    int mm = 0;
-                    for (int bk = 0; bk < 32; ++bk) mm = max(mm, (int)load[w][ins][(bk + j) & 31]);
-                    mx[w][ins] = (uint8_t)mm;
+                for (int h = 0; h < 2; ++h) {  // new maxima of the instructions the block left
+                    const int ins = touched[h];
+                    if (ins >= 0) {
+                        int mm = 0;
+                        for (int bk = 0; bk < 32; ++bk) mm = max(mm, (int)load[w][ins][(bk + j) & 31]);
+                        mx[w][ins] = (uint8_t)mm;
+                    }
                 }
                 __syncwarp();
                 int delta = 0;
