@@ -22,7 +22,7 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:spmm
 python tools/ncu_summary.py $O/ncu_spmm_tc.ncu-rep > $O/ncu_summary_spmm_tc.txt 2>&1
 timeout 900 ncu --set full --clock-control none -k regex:residual -s 3 -c 1 -o $O/ncu_residual_rmat22 python bench.py --workload rmat22 --steps 5 --warmup 3 --no-cpu-baseline --no-cusparse --no-variants --spmm "" --spmm-tc "" > /dev/null 2>&1
 python tools/ncu_summary.py $O/ncu_residual_rmat22.ncu-rep > $O/ncu_summary_residual_rmat22.txt 2>&1
-for tool in memcheck synccheck initcheck; do
+for tool in ${SANITIZERS:-}; do
   timeout 900 compute-sanitizer --tool $tool --target-processes all python tools/sanitize_run.py > $O/sanitizer_$tool.log 2>&1; echo "rc=$?" >> $O/sanitizer_$tool.log
 done
 rm -f $O/*.ncu-rep.tmp
