@@ -68,7 +68,7 @@ def parse():
     p.add_argument("--reorder", default="none", choices=["none", "degree"],
                    help="degree: symmetric degree ordering P A P^T before conversion (spaden_degree_order + "
                         "spaden_permute_csr, SURVEY.md NEXT-1); the iteration runs in the permuted space "
-                        "(one GPU only)")
+                        "(with N ranks every rank permutes the whole matrix and keeps its row slice)")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     p.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
                    help="x rebuild for N>1: NCCL all-gather after the SpMV, or peer stores fused into the "
@@ -297,18 +297,30 @@ class Workload:
         self.reorder_s = None
         if reorder == "degree":  # B = P A P^T; x kept in the permuted space (x'[k] = x[perm[k]])
             import paper_conf_icpp_cheny24_b200 as sp
-            if world > 1:
-                raise SystemExit("bench.py: --reorder needs the whole matrix on one GPU (--gpus 1)")
+            full = self.local
+            if world > 1:  # every rank permutes the whole matrix (the same B) and keeps its rows
+                if name.startswith("rmat"):
+                    rp, ci, v, _, _ = W.pagerank_slice_torch(int(name[4:]), 32, 0, self.m, seed=0, device=dev)
+                    full = (rp, ci, v)
+                else:
+                    full = tuple(torch.from_numpy(a).to(dev) for a in (A.rowptr, A.colidx, A.values))
             times = []
             for _ in range(3):  # first call loads the sort kernels; median of the 3
                 torch.cuda.synchronize(dev)
                 t0 = time.perf_counter()
-                perm = sp.degree_order(self.local[0])
-                B = sp.permute_csr(*self.local, perm)
+                perm = sp.degree_order(full[0])
+                B = sp.permute_csr(*full, perm)
                 torch.cuda.synchronize(dev)
                 times.append(time.perf_counter() - t0)
             self.reorder_s = statistics.median(times)
+            if world > 1:  # rows [r0, r1) of B, local rowptr
+                brp, bci, bv = B
+                a, b = int(brp[self.r0].item()), int(brp[self.r1].item())
+                B = ((brp[self.r0:self.r1 + 1] - a).contiguous(), bci[a:b].contiguous(), bv[a:b].contiguous())
+                del brp, bci, bv
+            del full
             self.local = B
+            self.local_nnz = int(B[1].numel())
             self.x0 = self.x0[perm.long()].contiguous()
             self.host = None
 
