@@ -187,10 +187,12 @@ SPADEN_API spaden_status_t spaden_count_blocks(int64_t m, int64_t n, int64_t nnz
  *                     violations return INDEX_OUT_OF_RANGE).
  *   d_rowptr, d_colidx, d_values  A on the device, values of dtype (16F or 32F,
  *                     moved as raw bits).
- *   d_perm            int32[m], a permutation of [0, m) (e.g. spaden_degree_order).
+ *   d_perm            int32[m], a permutation of [0, m) (e.g. spaden_degree_order);
+ *                     anything else returns INVALID_ARGUMENT (checked first).
  *   d_out_rowptr, d_out_colidx, d_out_values  B, caller-owned device arrays of
  *                     m+1, nnz and nnz elements (must not alias the inputs).
- * Stream-ordered; one host synchronisation (the column range check).
+ * Stream-ordered; two host synchronisations (the column range and the
+ * permutation checks).
  */
 SPADEN_API spaden_status_t spaden_degree_order(int64_t m, const int32_t *d_rowptr, int32_t *d_perm, void *stream);
 SPADEN_API spaden_status_t spaden_permute_csr(int64_t m, int64_t nnz, const int32_t *d_rowptr,

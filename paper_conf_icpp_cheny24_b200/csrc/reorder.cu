@@ -25,9 +25,19 @@ __global__ void k_degree_keys(int64_t m, const int32_t *__restrict__ rowptr, uin
     }
 }
 
-__global__ void k_inverse(int64_t m, const int32_t *__restrict__ perm, int32_t *__restrict__ iperm) {
-    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < m; k += (int64_t)gridDim.x * blockDim.x)
-        iperm[perm[k]] = (int32_t)k;
+// iperm[perm[k]] = k (iperm pre-filled with -1); entries outside [0, m) set *bad
+__global__ void k_inverse(int64_t m, const int32_t *__restrict__ perm, int32_t *__restrict__ iperm, uint32_t *bad) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < m; k += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t p = perm[k];
+        if (p < 0 || p >= m) atomicOr(bad, 1u);
+        else iperm[p] = (int32_t)k;
+    }
+}
+
+// a permutation leaves no -1 in iperm (a repeated entry leaves a hole)
+__global__ void k_check_inverse(int64_t m, const int32_t *__restrict__ iperm, uint32_t *bad) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x)
+        if (iperm[i] < 0) atomicOr(bad, 1u);
 }
 
 // entry e of row i -> key (iperm[i] << cb) | iperm[col], value e (one warp per row)
@@ -111,14 +121,29 @@ spaden_status_t permute_csr(int64_t m, int64_t nnz, const int32_t *rowptr, const
     cudaError_t e = cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, (const uint64_t *)nullptr,
                                                     (uint64_t *)nullptr, (const int32_t *)nullptr,
                                                     (int32_t *)nullptr, (int)nz, 0, 2 * cb, st);
+    uint32_t *bad = nullptr, hbad = 0;
     if (e == cudaSuccess) e = dmalloc(&iperm, sizeof(int32_t) * (size_t)m, st);
+    if (e == cudaSuccess) e = dmalloc(&bad, sizeof(uint32_t), st);
     if (e == cudaSuccess) e = dmalloc(&cnt, sizeof(int32_t) * (size_t)(m + 1), st);
     if (e == cudaSuccess) e = dmalloc(&scan_tmp, sizeof(int32_t) * scan_tmp_ints(m + 1), st);
     if (e == cudaSuccess) e = dmalloc(&key, 2 * sizeof(uint64_t) * nz, st);
     if (e == cudaSuccess) e = dmalloc(&idx, 2 * sizeof(int32_t) * nz, st);
     if (e == cudaSuccess) e = dmalloc(&tmp, std::max<size_t>(16, tmp_bytes), st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(iperm, 0xff, sizeof(int32_t) * (size_t)m, st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(bad, 0, sizeof(uint32_t), st);
+    if (e == cudaSuccess) {  // the permutation is checked before it indexes anything
+        k_inverse<<<grid_for(m, 256), 256, 0, st>>>(m, perm, iperm, bad);
+        k_check_inverse<<<grid_for(m, 256), 256, 0, st>>>(m, iperm, bad);
+        e = cudaMemcpyAsync(&hbad, bad, sizeof(hbad), cudaMemcpyDeviceToHost, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    }
+    if (e == cudaSuccess && hbad) {
+        for (void *p : {(void *)iperm, (void *)cnt, (void *)scan_tmp, (void *)key, (void *)idx, tmp, (void *)bad})
+            dev_free(p, st);
+        set_error("perm is not a permutation of [0, m)");
+        return SPADEN_ERR_INVALID_ARGUMENT;
+    }
     if (e == cudaSuccess) {
-        k_inverse<<<grid_for(m, 256), 256, 0, st>>>(m, perm, iperm);
         k_perm_counts<<<grid_for(m, 256), 256, 0, st>>>(m, rowptr, perm, cnt);
         e = exclusive_scan_i32(cnt, out_rowptr, m, scan_tmp, st);
     }
@@ -138,7 +163,8 @@ spaden_status_t permute_csr(int64_t m, int64_t nnz, const int32_t *rowptr, const
             e = cudaGetLastError();
         }
     }
-    for (void *p : {(void *)iperm, (void *)cnt, (void *)scan_tmp, (void *)key, (void *)idx, tmp}) dev_free(p, st);
+    for (void *p : {(void *)iperm, (void *)cnt, (void *)scan_tmp, (void *)key, (void *)idx, tmp, (void *)bad})
+        dev_free(p, st);
     return e == cudaSuccess ? SPADEN_OK : cuda_status(e, "permuting CSR");
 }
 

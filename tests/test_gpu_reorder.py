@@ -159,3 +159,18 @@ def test_rmat25_reordered_hybrid_sampled(sp, torch):
     err = oracle.componentwise_error(y[torch.from_numpy(krows).cuda()].cpu().numpy(), ys, s)
     assert err <= TOL32, err
     M.free()
+
+
+@pytest.mark.parametrize("kind", ["range", "duplicate"])
+def test_permute_rejects_bad_permutation(sp, torch, kind):
+    A = W.random_sparse(40, 40, 0.1, 2)
+    rp, ci, v = to_dev(torch, A.rowptr, A.colidx, A.values)
+    p = np.arange(40, dtype=np.int32)
+    if kind == "range":
+        p[7] = 40
+    else:
+        p[7] = 3  # 3 twice, 7 missing
+    (pd,) = to_dev(torch, p)
+    with pytest.raises(sp.SpadenError) as ei:
+        sp.permute_csr(rp, ci, v, pd)
+    assert ei.value.status == 1  # SPADEN_ERR_INVALID_ARGUMENT
