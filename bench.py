@@ -411,6 +411,7 @@ def main():
         dist.barrier()
     torch.cuda.synchronize(dev)
     with Clocks(local) as clk:
+        torch.cuda.nvtx.range_push("bench_timed_region")  # ncu --nvtx --nvtx-include bench_timed_region/
         start.record(stream)
         for i in range(args.steps):
             if flush:  # evict A, x and y from L2 (outside the step's events)
@@ -424,6 +425,7 @@ def main():
             it.gather_events = None
         end.record(stream)
         torch.cuda.synchronize(dev)
+        torch.cuda.nvtx.range_pop()
     if world > 1:
         dist.barrier()
     kernel_ms = [a.elapsed_time(b) for a, b in evs]
