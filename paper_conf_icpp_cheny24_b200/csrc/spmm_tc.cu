@@ -18,9 +18,12 @@
 //              core matrices (SBO = 128 B between 8-vector groups, LBO = slab2 -
 //              slab1), staged by cp.async.bulk straight from Xb;
 //   B operand: the two blocks decoded into dense 8x8 fp16 tiles (row-major, one
-//              core matrix each, LBO = tile2 - tile1): a warp decodes a block
-//              with lane l owning bits 2l, 2l+1 -- exactly the paper's Alg. 2
-//              lane mapping, value index = offset + popcount rank.
+//              core matrix each, LBO = tile2 - tile1): 8 lanes per block, lane
+//              r walking row r's bits in column order (value index = offset +
+//              popcount rank, P:L138 / Alg. 2 semantics P:L172-177) and storing
+//              the dense row as one 16-byte store (a warp decodes 4 blocks at
+//              once; the paper's lane-per-2-bits mapping took 20 instructions
+//              per block instead of ~7: K = 64 1.221 -> 1.187 ms).
 // The pairs of a block-row accumulate in its own 8 TMEM columns in block order
 // (deterministic, a function of the block-row alone); the epilogue reads the
 // 128 x 8 fp32 accumulator with tcgen05.ld and writes alpha*D + beta*Y.
@@ -475,34 +478,40 @@ k_spmm_tc(int64_t m, const TcChunk *__restrict__ chunks, const TcRec *__restrict
             if (c >= kTcRing) tc_wait(s_u32(&bar_mma[a]), ring_ph(c - kTcRing));  // tile slot free
             if (lane == 0 && dw == 0) TR(1, c, 4);
             const int v0 = (int)tc_lds(ar.off);  // blk_offset of the chunk's first block
-            // a warp per block, lane l -> bits 2l, 2l+1 (row l/4, columns 2(l%4), 2(l%4)+1);
-            // two blocks per step (q, q + 8) so their shared-memory chains overlap
-            const int bit = 2 * lane;
-            for (int q0 = dw; q0 < nblk; q0 += 2 * kTcDecodeWarps) {
-                const int q1 = q0 + kTcDecodeWarps;
-                const bool has1 = q1 < nblk;
-                const uint32_t lo0 = tc_lds(ar.bmp + 8u * q0), hi0 = tc_lds(ar.bmp + 8u * q0 + 4u);
-                const uint32_t lo1 = has1 ? tc_lds(ar.bmp + 8u * q1) : 0u, hi1 = has1 ? tc_lds(ar.bmp + 8u * q1 + 4u) : 0u;
-                const int off0 = (int)tc_lds(ar.off + 4u * q0) - v0;
-                const int off1 = has1 ? (int)tc_lds(ar.off + 4u * q1) - v0 : 0;
-                const uint32_t pos0 = tc_lds8(ar.rec + 34u + (uint32_t)q0);
-                const uint32_t pos1 = has1 ? tc_lds8(ar.rec + 34u + (uint32_t)q1) : 0u;
-                const uint64_t bm0 = ((uint64_t)hi0 << 32) | lo0, bm1 = ((uint64_t)hi1 << 32) | lo1;
-                const uint32_t two0 = (uint32_t)(bm0 >> bit) & 3u, two1 = (uint32_t)(bm1 >> bit) & 3u;
-                const uint32_t a0 = ar.val + 2u * (uint32_t)(off0 + __popcll(bm0 & ((1ull << bit) - 1ull)));
-                const uint32_t a1 = ar.val + 2u * (uint32_t)(off1 + __popcll(bm1 & ((1ull << bit) - 1ull)));
-                uint16_t h00 = 0, h01 = 0, h10 = 0, h11 = 0;
-                if (two0 & 1u) asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h00) : "r"(a0) : "memory");
-                if (two0 & 2u) asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h01) : "r"(a0 + 2u * (two0 & 1u)) : "memory");
-                if (two1 & 1u) asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h10) : "r"(a1) : "memory");
-                if (two1 & 2u) asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h11) : "r"(a1 + 2u * (two1 & 1u)) : "memory");
-                asm volatile("st.shared.u32 [%0], %1;" ::"r"(tile_of(a, (int)pos0) + 4u * lane),
-                             "r"((uint32_t)h00 | ((uint32_t)h01 << 16))
-                             : "memory");
-                if (has1)
-                    asm volatile("st.shared.u32 [%0], %1;" ::"r"(tile_of(a, (int)pos1) + 4u * lane),
-                                 "r"((uint32_t)h10 | ((uint32_t)h11 << 16))
-                                 : "memory");
+            // 8 lanes per block, lane = row r: the row's set bits in ascending
+            // column order take the row's values (popcount rank of the row start,
+            // P:L138), the dense 8-half row leaves as one 16-byte store; a warp
+            // decodes 4 blocks per step
+            {
+                const int qs = lane >> 3, r = lane & 7;
+                for (int qb = 4 * dw; qb < nblk; qb += 4 * kTcDecodeWarps) {
+                    const int q = qb + qs;
+                    if (q < nblk) {
+                        const uint32_t lo = tc_lds(ar.bmp + 8u * q), hi = tc_lds(ar.bmp + 8u * q + 4u);
+                        const int off = (int)tc_lds(ar.off + 4u * q) - v0;
+                        const uint32_t pos = tc_lds8(ar.rec + 34u + (uint32_t)q);
+                        const uint64_t bm = ((uint64_t)hi << 32) | lo;
+                        const uint32_t byte = (uint32_t)(bm >> (8 * r)) & 0xffu;
+                        uint32_t va = ar.val + 2u * (uint32_t)(off + __popcll(bm & ((1ull << (8 * r)) - 1ull)));
+                        uint32_t w[4];
+#pragma unroll
+                        for (int c2 = 0; c2 < 4; ++c2) {
+                            uint16_t h0 = 0, h1 = 0;
+                            if ((byte >> (2 * c2)) & 1u) {
+                                asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h0) : "r"(va) : "memory");
+                                va += 2u;
+                            }
+                            if ((byte >> (2 * c2 + 1)) & 1u) {
+                                asm volatile("ld.shared.u16 %0, [%1];" : "=h"(h1) : "r"(va) : "memory");
+                                va += 2u;
+                            }
+                            w[c2] = (uint32_t)h0 | ((uint32_t)h1 << 16);
+                        }
+                        asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(tile_of(a, (int)pos) + 16u * (uint32_t)r),
+                                     "r"(w[0]), "r"(w[1]), "r"(w[2]), "r"(w[3])
+                                     : "memory");
+                    }
+                }
             }
             // zero tiles for the partners of lone blocks (pair o: position 2o+1)
             for (uint32_t lone = tc_lds(ar.rec) >> 16; lone; lone &= lone - 1) {
