@@ -35,13 +35,13 @@
 // consecutive blocks [B0, B1); block-rows [brA, brE) end in it, a block-row
 // may start in an earlier chunk (pair pA) and continue into the next (pE).
 // Roles per CTA:
-//   warp 13    producer lane: bulk-copies the chunk's MMA record (TcRec,
+//   warp 9     producer lane: bulk-copies the chunk's MMA record (TcRec,
 //              precomputed with the schedule), blk_rowptr, bitmap, blk_col,
 //              blk_offset and value slices (4-chunk ring);
-//   warp 14    x slabs: once a chunk's arrays have landed, its lanes issue one
+//   warp 10    x slabs: once a chunk's arrays have landed, its lanes issue one
 //              cp.async.bulk per block (3 slab buffers);
-//   warps 4-11 decode the blocks into dense tiles (4-chunk ring);
-//   warps 12, 15  MMA issue, alternate chunks (warp 12 also allocates TMEM): one elected lane issues the MMAs
+//   warps 4-7  decode the blocks into dense tiles (4-chunk ring);
+//   warps 8, 11  MMA issue, alternate chunks (warp 8 also allocates TMEM): one elected lane issues the MMAs
 //              (pair o's descriptors are base + o * stride: blocks sit in pair
 //              order, see TcRec; the per-block-row slot comes through redux.sync
 //              so every MMA operand is warp-uniform);
@@ -78,7 +78,10 @@ constexpr int kTcRecBytes = 160;  // a chunk's MMA record (TcRec)
 constexpr int kTcArrBytes = 5120; // one chunk's staged arrays (record, brp, bitmap, blk_col, blk_offset, values)
 constexpr int kTcRing = 4;        // arrays, tiles and accumulator hand-off: 4 chunks in flight
 constexpr int kTcSlabBufs = 3;    // x slabs: 3 chunks (the big buffers)
-constexpr int kTcDecodeWarps = 8;
+#ifndef SPADEN_TC_DECODE_WARPS
+#define SPADEN_TC_DECODE_WARPS 4  // 8 measured slower once a warp decodes 4 blocks at a time
+#endif
+constexpr int kTcDecodeWarps = SPADEN_TC_DECODE_WARPS;
 constexpr int kTcSlabBytes = kTcBlocks * kSlabBytes;
 constexpr int kTcTileBytes = kTcBlocks * kTileBytes;
 constexpr int kTcSmem = kTcSlabBufs * kTcSlabBytes + kTcRing * (kTcTileBytes + kTcArrBytes);
