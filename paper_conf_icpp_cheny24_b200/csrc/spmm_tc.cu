@@ -76,8 +76,14 @@ constexpr int kSlabBytes = kTcM * 16;
 constexpr int kTileBytes = 128;
 constexpr int kTcRecBytes = 160;  // a chunk's MMA record (TcRec)
 constexpr int kTcArrBytes = 5120; // one chunk's staged arrays (record, brp, bitmap, blk_col, blk_offset, values)
-constexpr int kTcRing = 4;        // arrays, tiles and accumulator hand-off: 4 chunks in flight
-constexpr int kTcSlabBufs = 3;    // x slabs: 3 chunks (the big buffers)
+#ifndef SPADEN_TC_RING
+#define SPADEN_TC_RING 4
+#endif
+#ifndef SPADEN_TC_SLABS
+#define SPADEN_TC_SLABS 3
+#endif
+constexpr int kTcRing = SPADEN_TC_RING;  // arrays, tiles and accumulator hand-off: chunks in flight
+constexpr int kTcSlabBufs = SPADEN_TC_SLABS;  // x slabs: chunks (the big buffers)
 #ifndef SPADEN_TC_DECODE_WARPS
 #define SPADEN_TC_DECODE_WARPS 4  // 8 measured slower once a warp decodes 4 blocks at a time
 #endif
