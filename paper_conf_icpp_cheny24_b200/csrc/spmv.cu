@@ -70,6 +70,9 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t byt
 // try_wait suspends the warp (up to the hint) instead of spinning: waiting
 // warps then cost no issue slots
 constexpr uint32_t kSuspendHintNs = 0x989680;
+#ifndef SPADEN_AVAIL_SLEEP_NS
+#define SPADEN_AVAIL_SLEEP_NS 64  // back-off of a consumer waiting for its unit's tile to be published
+#endif
 __device__ __forceinline__ bool mbar_try_wait(uint32_t bar, uint32_t parity) {
     uint32_t ok;
     asm volatile(
@@ -710,7 +713,7 @@ k_spmv_tiled(int stages, int stage_bytes, int64_t m, const TileDesc *__restrict_
         if (g >= total) break;
         while (avail <= g) {  // the producer has not published the tile yet
             asm volatile("ld.acquire.cta.shared.s32 %0, [%1];" : "=r"(avail) : "r"(a_avail) : "memory");
-            if (avail <= g) __nanosleep(64);
+            if (avail <= g) __nanosleep(SPADEN_AVAIL_SLEEP_NS);
         }
         int s = 0, us = 0, par = 0;
         for (; s < stages; ++s) {  // the stage whose tile holds unit g (its current fill:
